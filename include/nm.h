@@ -1,0 +1,205 @@
+/*
+ * nm.h -- C ABI of libnm, the B200-native (sm_100a) hot path of
+ *   Chen, Sung, Zhang, Li, Shen, "Accelerating GNNs on GPU Sparse Tensor Cores through N:M
+ *   Sparsity-Oriented Graph Reordering", PPoPP'25   ("PAPER.md:Lxxx" = line of the paper text).
+ *
+ * The method (§3, §4): reorder the vertices of a graph so that
+ * the symmetric adjacency matrix B = P A P^T meets the V:N:M structured-sparsity pattern of
+ * sparse tensor cores "as much as possible" (SGRP, L188-199), pack it into the SPTC form
+ * (compressed values + 2-bit metadata + per-meta-block column indices, L492), and run the
+ * aggregation SpMM Y = B (P X) on sparse tensor cores (L182, L492).  This library adds a
+ * residual CSR for whatever still violates the pattern, so the result is always lossless
+ * (L128: reordering "does not cause any accuracy loss").
+ *
+ * Conventions (all entry points):
+ *  - Every function returns nm_status; no exception or longjmp crosses the ABI.  On error
+ *    the out-parameters are left untouched and nm_last_error() (thread-local) says why.
+ *  - perm[p] = old vertex id placed at new position p (the paper's phi' as a list, Alg. 1
+ *    output L358).  B[p][q] = A[perm[p]][perm[q]];  (P X)[p] = X[perm[p]]  (Fig. 1 caption
+ *    L38: "the corresponding rows in the dense matrix ... must be swapped too").
+ *  - Graphs are CSR: rowptr int64[n+1], col int32[nnz], columns sorted ascending, no
+ *    duplicates, symmetric pattern (undirected graph, L188), self-loops allowed.
+ *  - Ownership: the caller owns every array it passes (graph, perm, X, Y, W, bias) and every
+ *    output buffer; the library owns nm_packed (device memory on the device current at pack
+ *    time) until nm_packed_free.
+ *  - Streams: `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *    Device-side calls are stream-ordered and asynchronous unless stated otherwise.
+ *  - There is no CPU fallback: without a usable sm_100 device the device entry points
+ *    return NM_ERR_CUDA.
+ */
+#ifndef NM_H_
+#define NM_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define NM_API __attribute__((visibility("default")))
+#else
+#define NM_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  NM_OK = 0,
+  NM_ERR_INVALID_ARG = 1,  /* NULL pointer, negative size, bad flag combination            */
+  NM_ERR_UNSUPPORTED = 2,  /* V, N, M, F or dtype outside the supported set (see below)     */
+  NM_ERR_BAD_CSR = 3,      /* rowptr not monotone, column out of range, unsorted or dup     */
+  NM_ERR_NOT_SYMMETRIC = 4,/* pattern of A is not symmetric                                 */
+  NM_ERR_CUDA = 5,         /* CUDA runtime/driver error (message in nm_last_error)          */
+  NM_ERR_OOM = 6           /* device or host allocation failed                              */
+} nm_status;
+
+typedef enum { NM_F16 = 0, NM_BF16 = 1, NM_F32 = 2 } nm_dtype;
+
+/* A square sparse matrix in CSR form.  `val` (length nnz, dtype val_dtype) may be NULL,
+ * meaning every stored entry is 1.0 (binary adjacency, L484).  on_device = 1 when the three
+ * arrays are device pointers, 0 for host pointers. */
+typedef struct {
+  int64_t n, nnz;
+  const int64_t* rowptr;
+  const int32_t* col;
+  const void* val;
+  nm_dtype val_dtype;
+  int on_device;
+} nm_csr;
+
+/* Reordering options (Alg. 1-3).  Zero-initialise and set what you need, or pass NULL for
+ * the defaults {10, 10, 10, 0, 1}. */
+typedef struct {
+  int max_outer;   /* Alg. 1 loop cap ("max. iteration", L359; MAXITER = 10, L496)        */
+  int max_stage1;  /* Alg. 2 MAXITER (L421)                                                */
+  int max_stage2;  /* Alg. 3 MAXITER (L451)                                                */
+  int gain_rule;   /* 0 = paper: freshtop() takes the best fresh pair whatever its gain
+                      (footnote L440); 1 = only pairs with positive gain                   */
+  int keep_best;   /* 1 = return the visited order with the fewest violations (never worse
+                      than the input order); 0 = return the last order (literal Alg. 1)    */
+} nm_reorder_opts;
+
+typedef struct {
+  int64_t omega_init, omega_final; /* #segment vectors violating N:M (omega, L203)         */
+  int64_t mb_init, mb_final;       /* #meta-blocks violating the vertical constraint (MBscore, L382) */
+  int64_t outer_iters, stage1_iters, stage2_passes;
+  int64_t max_pairs_per_primary;   /* <= M by construction (L562-569)                      */
+  double seconds;
+} nm_reorder_stats;
+
+/* ---------------------------------------------------------------------------------------
+ * nm_reorder -- the SGRP heuristic (Alg. 1: repeat Stage-1 (Alg. 2, vertical
+ * constraint, Hamming position codes + sort, L366-384) and Stage-2 (Alg. 3, horizontal
+ * constraint, greedy pair swaps, L386-422) while violations remain).  Deterministic; the
+ * permutation is bit-identical to the CPU oracle's (DESIGN.md §3 readings).
+ *   A        : input graph (host or device CSR), symmetric pattern.
+ *   V, N, M  : pattern; V >= 1, 1 <= N < M <= 32.
+ *   perm_out : host int32[n], caller-allocated; receives perm.
+ *   st       : optional statistics.
+ * Synchronous.  Errors: INVALID_ARG, UNSUPPORTED (M > 32), BAD_CSR, NOT_SYMMETRIC, OOM, CUDA.
+ * ------------------------------------------------------------------------------------- */
+NM_API nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
+                     int32_t* perm_out, nm_reorder_stats* st);
+
+/* nm_count_violations -- omega (L203), MBscore (L382) and optionally PScore per segment
+ * (L396) of B = P A P^T, computed on the GPU.  perm: host int32[n] or NULL (identity).
+ * pscore: host int32[ceil(n/M)] or NULL.  Synchronous. */
+NM_API nm_status nm_count_violations(const nm_csr* A, const int32_t* perm, int V, int N, int M,
+                              int64_t* omega, int64_t* mbscore, int32_t* pscore);
+
+/* ---------------------------------------------------------------------------------------
+ * Packed V:N:M matrix (the SPTC form of L492).  Rows of B are grouped in
+ * panels of Vp = 128 rows; columns in segments of Mp columns, Mp = 4 when V == 1 (2:4 at
+ * V = 1) and Mp = M otherwise; per non-empty (panel, segment) meta-block the k = 4 columns
+ * with the most nonzeros are selected (vertical constraint, L338-339) and each row keeps
+ * its first <= 2 nonzeros among them (N = 2, horizontal constraint L340-341) as two 16-bit
+ * values plus a 4-bit index pair.  Everything else goes to a residual CSR.  Device memory
+ * holds the MMA-native image consumed by nm_spmm (tcgen05.mma.sp operands).
+ * Supported: N = 2; M in {4, 8, 16}; any V >= 1 (V = 1 -> Mp = 4); Vp = 128 (pass 0 or
+ * 128); dtype NM_F16 or NM_BF16 (values are rounded from val_dtype to dtype).
+ * ------------------------------------------------------------------------------------- */
+typedef struct nm_packed nm_packed;
+
+/* Packs rows [0, n) of B = P A P^T.  perm: host int32[n] (NULL = identity).
+ * The call blocks until the pack is complete; the handle is then immutable. */
+NM_API nm_status nm_pack(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
+                  nm_dtype dtype, void* stream, nm_packed** out);
+
+/* Packs only rows [row_begin, row_end) of B (a row shard for multi-GPU runs); row_begin
+ * must be a multiple of Vp.  Columns still range over all n vertices. */
+NM_API nm_status nm_pack_rows(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
+                       nm_dtype dtype, int64_t row_begin, int64_t row_end, void* stream,
+                       nm_packed** out);
+
+/* Sizes: #meta-blocks, #values kept in MMA slots, #residual nonzeros, device bytes held,
+ * #K=32 chunks (8 meta-blocks each, padded per panel).  Any pointer may be NULL. */
+NM_API nm_status nm_packed_info(const nm_packed* P, int64_t* n_mb, int64_t* packed_nnz,
+                         int64_t* residual_nnz, int64_t* device_bytes, int64_t* n_chunks);
+
+/* Copies the canonical form back to host arrays (caller-allocated, sizes from
+ * nm_packed_info; rows = row_end - row_begin, panels = ceil(rows / Vp)):
+ *   panel_ptr int64[panels+1], mb_seg int32[n_mb], sel uint8[n_mb*4] (ascending offsets),
+ *   nib uint8[n_mb*Vp] (idx0 | idx1 << 2 per row of the meta-block's panel),
+ *   vals uint16[n_mb*Vp*2] (16-bit value bits of the two slots),
+ *   res_rowptr int64[rows+1], res_col int32[residual_nnz], res_val uint16[residual_nnz].
+ * Any pointer may be NULL to skip that array.  Synchronous. */
+NM_API nm_status nm_export_canonical(const nm_packed* P, int64_t* panel_ptr, int32_t* mb_seg,
+                              uint8_t* sel, uint8_t* nib, uint16_t* vals, int64_t* res_rowptr,
+                              int32_t* res_col, uint16_t* res_val);
+
+NM_API void nm_packed_free(nm_packed* P);
+
+/* ---------------------------------------------------------------------------------------
+ * Row permutation of a dense matrix (Fig. 1 caption L38).  Device pointers, row-major,
+ * leading dimension ld (elements), F columns, n rows; dtype of X/Y elements.
+ *   nm_permute_rows   : PX[p] = X[perm[p]]      (X -> permuted order)
+ *   nm_unpermute_rows : Y[perm[p]] = Yp[p]      (permuted order -> original order)
+ * perm_dev: device int32[n].  In-place (X == PX) is not allowed. */
+NM_API nm_status nm_permute_rows(const void* X, void* PX, const int32_t* perm_dev, int64_t n, int F,
+                          int64_t ld, nm_dtype dtype, void* stream);
+NM_API nm_status nm_unpermute_rows(const void* Yp, void* Y, const int32_t* perm_dev, int64_t n, int F,
+                            int64_t ld, nm_dtype dtype, void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * nm_spmm -- Yp = B[rows of P] * PX on sparse tensor cores (tcgen05.mma.sp.kind::f16,
+ * fp32 accumulation in tensor memory) plus the residual CSR (CUDA cores), i.e. exactly
+ * (P A P^T)(P X) for the packed rows (the aggregation SpMM of L182, L492).
+ *   PX : device, n x F, leading dimension ldx (elements), dtype of the pack, permuted order.
+ *        ldx must be a multiple of 8 (16-byte rows).
+ *   Yp : device fp32, (row_end-row_begin) x F, leading dimension ldy; overwritten.
+ *   F  : 1 <= F <= 4096.
+ * Stream-ordered, asynchronous.  Errors: INVALID_ARG, UNSUPPORTED, CUDA. */
+NM_API nm_status nm_spmm(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy,
+                  int F, void* stream);
+
+/* Same as nm_spmm, but only the tensor-core part (no residual) or only the residual part
+ * (adds into Yp).  For profiling and tests. */
+NM_API nm_status nm_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy,
+                       int F, void* stream);
+NM_API nm_status nm_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
+                           int64_t ldy, int F, void* stream);
+
+/* ---------------------------------------------------------------------------------------
+ * nm_gcn_layer -- one GCN layer (Eq. 1): Hout = act(Ahat (H W) + bias), linear first
+ * (GCN "aggregates after its linear layer", L564).  Ahat: packed normalised adjacency in
+ * permuted order (P Ahat P^T), H: device [rows(Ahat.n) x F_in] dtype of the pack (permuted
+ * order), W: device [F_in x F_out] same dtype, row-major; bias: device fp32[F_out] or NULL;
+ * Hout: device [rows x F_out] same dtype.  flags: NM_RELU.  ws: device workspace of at
+ * least nm_gcn_workspace_bytes(...) bytes.  The dense H W runs on cuBLASLt (a plain
+ * library GEMM); the aggregation on nm_spmm.
+ * ------------------------------------------------------------------------------------- */
+#define NM_RELU 1
+NM_API size_t nm_gcn_workspace_bytes(int64_t n, int F_out);
+NM_API nm_status nm_gcn_layer(const nm_packed* Ahat, const void* H, const void* W, const float* bias,
+                       void* Hout, int F_in, int F_out, int flags, void* ws, size_t ws_bytes,
+                       void* stream);
+
+/* ------------------------------------------------------------------------------------- */
+NM_API const char* nm_status_string(nm_status s);
+NM_API const char* nm_last_error(void);   /* thread-local detail of the last failure on this thread */
+NM_API int nm_version(void);              /* ABI version, currently 1 */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NM_H_ */

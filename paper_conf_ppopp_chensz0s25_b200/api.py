@@ -1,0 +1,182 @@
+"""Thin Pythonic layer over the C ABI (argument marshalling only; every step runs in libnm).
+
+numpy arrays are passed for host-side graph data, torch CUDA tensors for device buffers
+(torch is used for device memory and streams only).
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+
+from . import _lib as L
+
+_DT = {"f16": L.NM_F16, "bf16": L.NM_BF16, "f32": L.NM_F32}
+
+
+def _ptr(a):
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        return ctypes.c_void_p(a.ctypes.data)
+    return ctypes.c_void_p(a.data_ptr())  # torch tensor
+
+
+def _csr_struct(indptr, indices, val=None, val_dtype="f16"):
+    rp = np.ascontiguousarray(indptr, dtype=np.int64)
+    ci = np.ascontiguousarray(indices, dtype=np.int32)
+    keep = [rp, ci]
+    c = L.nm_csr()
+    c.n = len(rp) - 1
+    c.nnz = int(rp[-1])
+    c.rowptr = rp.ctypes.data
+    c.col = ci.ctypes.data
+    if val is not None:
+        v = np.ascontiguousarray(val)
+        keep.append(v)
+        c.val = v.ctypes.data
+    else:
+        c.val = None
+    c.val_dtype = _DT[val_dtype]
+    c.on_device = 0
+    return c, keep
+
+
+def _stream_ptr(stream=None):
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def reorder(indptr, indices, V: int, N: int, M: int, max_outer=10, max_stage1=10, max_stage2=10,
+            gain_rule=0, keep_best=1):
+    """nm_reorder: returns (perm int32[n], stats dict)."""
+    c, keep = _csr_struct(indptr, indices)
+    perm = np.zeros(c.n, np.int32)
+    o = L.nm_reorder_opts(max_outer, max_stage1, max_stage2, gain_rule, keep_best)
+    st = L.nm_reorder_stats()
+    L.check(L.load().nm_reorder(ctypes.byref(c), V, N, M, ctypes.byref(o),
+                                perm.ctypes.data_as(L.P32), ctypes.byref(st)), "nm_reorder")
+    return perm, {f: getattr(st, f) for f, _ in L.nm_reorder_stats._fields_}
+
+
+def count_violations(indptr, indices, perm, V: int, N: int, M: int):
+    """nm_count_violations (GPU): returns (omega, mbscore, pscore int32[ceil(n/M)])."""
+    c, keep = _csr_struct(indptr, indices)
+    S = (c.n + M - 1) // M
+    ps = np.zeros(S, np.int32)
+    w = ctypes.c_int64()
+    mb = ctypes.c_int64()
+    pm = None if perm is None else np.ascontiguousarray(perm, np.int32)
+    L.check(L.load().nm_count_violations(ctypes.byref(c), None if pm is None else pm.ctypes.data_as(L.P32),
+                                         V, N, M, ctypes.byref(w), ctypes.byref(mb),
+                                         ps.ctypes.data_as(L.P32)), "nm_count_violations")
+    return int(w.value), int(mb.value), ps
+
+
+class Packed:
+    """Owns an nm_packed handle (device memory on the current device)."""
+
+    def __init__(self, handle, n, row_begin, row_end, dtype):
+        self.handle = handle
+        self.n = n
+        self.row_begin = row_begin
+        self.row_end = row_end
+        self.dtype = dtype
+
+    @property
+    def rows(self):
+        return self.row_end - self.row_begin
+
+    def info(self):
+        vals = [ctypes.c_int64() for _ in range(5)]
+        L.check(L.load().nm_packed_info(self.handle, *[ctypes.byref(v) for v in vals]),
+                "nm_packed_info")
+        keys = ("n_mb", "packed_nnz", "residual_nnz", "device_bytes", "n_chunks")
+        return {k: int(v.value) for k, v in zip(keys, vals)}
+
+    def export_canonical(self):
+        inf = self.info()
+        m, r = inf["n_mb"], inf["residual_nnz"]
+        P = (self.rows + 127) // 128
+        out = dict(panel_ptr=np.zeros(P + 1, np.int64), mb_seg=np.zeros(max(m, 1), np.int32),
+                   sel=np.zeros(max(m, 1) * 4, np.uint8), nib=np.zeros(max(m, 1) * 128, np.uint8),
+                   vals=np.zeros(max(m, 1) * 256, np.uint16),
+                   res_rowptr=np.zeros(self.rows + 1, np.int64),
+                   res_col=np.zeros(max(r, 1), np.int32), res_val=np.zeros(max(r, 1), np.uint16))
+        L.check(L.load().nm_export_canonical(
+            self.handle, out["panel_ptr"].ctypes.data_as(L.P64), out["mb_seg"].ctypes.data_as(L.P32),
+            out["sel"].ctypes.data_as(L.PU8), out["nib"].ctypes.data_as(L.PU8),
+            out["vals"].ctypes.data_as(L.PU16), out["res_rowptr"].ctypes.data_as(L.P64),
+            out["res_col"].ctypes.data_as(L.P32), out["res_val"].ctypes.data_as(L.PU16)),
+            "nm_export_canonical")
+        out["mb_seg"] = out["mb_seg"][:m]
+        out["sel"] = out["sel"][:m * 4]
+        out["nib"] = out["nib"][:m * 128]
+        out["vals"] = out["vals"][:m * 256]
+        out["res_col"] = out["res_col"][:r]
+        out["res_val"] = out["res_val"][:r]
+        out["n_mb"], out["res_nnz"] = m, r
+        return out
+
+    def free(self):
+        if self.handle:
+            L.load().nm_packed_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def pack(indptr, indices, perm, V: int, N: int, M: int, dtype="f16", val=None, val_dtype=None,
+         row_begin=None, row_end=None, stream=None):
+    """nm_pack / nm_pack_rows of B = P A P^T.  val: values per CSR entry (numpy, dtype
+    val_dtype in {'f16','bf16' (uint16 bits),'f32'}) or None for a binary adjacency."""
+    if val is not None and val_dtype is None:
+        val_dtype = "f32" if val.dtype == np.float32 else ("f16" if val.dtype == np.float16 else "bf16")
+    c, keep = _csr_struct(indptr, indices, val, val_dtype or "f16")
+    pm = None if perm is None else np.ascontiguousarray(perm, np.int32)
+    h = ctypes.c_void_p()
+    pp = None if pm is None else pm.ctypes.data_as(L.P32)
+    sp = _stream_ptr(stream)
+    if row_begin is None:
+        L.check(L.load().nm_pack(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], sp, ctypes.byref(h)),
+                "nm_pack")
+        rb, re = 0, c.n
+    else:
+        rb, re = int(row_begin), int(row_end)
+        L.check(L.load().nm_pack_rows(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], rb, re, sp,
+                                      ctypes.byref(h)), "nm_pack_rows")
+    return Packed(h, c.n, rb, re, dtype)
+
+
+def spmm(P: Packed, PX, Yp, F=None, stream=None, part="all"):
+    """Yp (fp32 CUDA tensor, rows x F) = packed B * PX (16-bit CUDA tensor, n x F)."""
+    F = PX.shape[1] if F is None else F
+    fn = {"all": "nm_spmm", "sptc": "nm_spmm_sptc", "residual": "nm_spmm_residual"}[part]
+    L.check(getattr(L.load(), fn)(P.handle, _ptr(PX), PX.stride(0), _ptr(Yp), Yp.stride(0), F,
+                                  _stream_ptr(stream)), fn)
+
+
+def permute_rows(X, PX, perm_dev, dtype, stream=None):
+    L.check(L.load().nm_permute_rows(_ptr(X), _ptr(PX), _ptr(perm_dev), X.shape[0], X.shape[1],
+                                     X.stride(0), _DT[dtype], _stream_ptr(stream)), "nm_permute_rows")
+
+
+def unpermute_rows(Yp, Y, perm_dev, dtype, stream=None):
+    L.check(L.load().nm_unpermute_rows(_ptr(Yp), _ptr(Y), _ptr(perm_dev), Yp.shape[0], Yp.shape[1],
+                                       Yp.stride(0), _DT[dtype], _stream_ptr(stream)),
+            "nm_unpermute_rows")
+
+
+def gcn_workspace_bytes(n, F_out):
+    return int(L.load().nm_gcn_workspace_bytes(n, F_out))
+
+
+def gcn_layer(P: Packed, H, W, bias, Hout, ws, relu=True, stream=None):
+    L.check(L.load().nm_gcn_layer(P.handle, _ptr(H), _ptr(W), _ptr(bias), _ptr(Hout), H.shape[1],
+                                  W.shape[1], L.NM_RELU if relu else 0, _ptr(ws), ws.numel(),
+                                  _stream_ptr(stream)), "nm_gcn_layer")

@@ -1,0 +1,252 @@
+// libnm: status/error plumbing, CSR validation and upload, packed-handle queries and the
+// canonical export (decoding the MMA-native image back to the canonical arrays of nm.h).
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "nm_internal.h"
+
+namespace nm {
+
+static thread_local std::string g_last_error;
+
+void set_error(const std::string& msg) { g_last_error = msg; }
+
+nm_status fail(nm_status s, const std::string& msg) {
+  g_last_error = msg;
+  return s;
+}
+
+nm_status cuda_fail(cudaError_t e, const char* what) {
+  g_last_error = std::string(what) + ": " + cudaGetErrorString(e);
+  return e == cudaErrorMemoryAllocation ? NM_ERR_OOM : NM_ERR_CUDA;
+}
+
+uint16_t one_bits(nm_dtype dt) { return dt == NM_BF16 ? (uint16_t)0x3F80 : (uint16_t)0x3C00; }
+
+nm_status validate_csr_host(int64_t n, const int64_t* rp, const int32_t* ci, bool check_sym) {
+  if (n < 0) return fail(NM_ERR_INVALID_ARG, "n < 0");
+  if (rp[0] != 0) return fail(NM_ERR_BAD_CSR, "rowptr[0] != 0");
+  for (int64_t i = 0; i < n; ++i) {
+    if (rp[i + 1] < rp[i]) return fail(NM_ERR_BAD_CSR, "rowptr not monotone at row " + std::to_string(i));
+    for (int64_t k = rp[i]; k < rp[i + 1]; ++k) {
+      if (ci[k] < 0 || ci[k] >= n)
+        return fail(NM_ERR_BAD_CSR, "column out of range in row " + std::to_string(i));
+      if (k > rp[i] && ci[k] <= ci[k - 1])
+        return fail(NM_ERR_BAD_CSR, "columns unsorted or duplicated in row " + std::to_string(i));
+    }
+  }
+  if (check_sym) {
+    // symmetric pattern: for every (i, j) the entry (j, i) exists.  Count-based check: walk
+    // rows in order and keep a cursor per row; each row j must see its entries (j, i) in
+    // increasing i as the outer loop advances.
+    std::vector<int64_t> cur(rp, rp + n);
+    for (int64_t i = 0; i < n; ++i)
+      for (int64_t k = rp[i]; k < rp[i + 1]; ++k) {
+        int64_t j = ci[k];
+        if (cur[j] >= rp[j + 1] || ci[cur[j]] != i)
+          return fail(NM_ERR_NOT_SYMMETRIC, "pattern not symmetric at (" + std::to_string(i) +
+                                                "," + std::to_string(j) + ")");
+        cur[j]++;
+      }
+    for (int64_t j = 0; j < n; ++j)
+      if (cur[j] != rp[j + 1])
+        return fail(NM_ERR_NOT_SYMMETRIC, "pattern not symmetric in row " + std::to_string(j));
+  }
+  return NM_OK;
+}
+
+void DevCsr::release() {
+  if (rp) cudaFree(rp);
+  if (ci) cudaFree(ci);
+  if (val) cudaFree(val);
+  rp = nullptr;
+  ci = nullptr;
+  val = nullptr;
+}
+
+__global__ void k_convert_vals(const void* __restrict__ src, int src_dt, uint16_t* __restrict__ dst,
+                               int dst_dt, int64_t nnz) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  for (; i < nnz; i += (int64_t)gridDim.x * blockDim.x) {
+    float v;
+    if (src_dt == NM_F32) v = ((const float*)src)[i];
+    else if (src_dt == NM_F16) v = __half2float(((const __half*)src)[i]);
+    else v = __bfloat162float(((const __nv_bfloat16*)src)[i]);
+    uint16_t b;
+    if (dst_dt == NM_F16) {
+      __half h = __float2half_rn(v);
+      memcpy(&b, &h, 2);
+    } else {
+      __nv_bfloat16 h = __float2bfloat16_rn(v);
+      memcpy(&b, &h, 2);
+    }
+    dst[i] = b;
+  }
+}
+
+nm_status upload_csr(const nm_csr* A, nm_dtype dtype, DevCsr* out, cudaStream_t s) {
+  out->release();
+  out->n = A->n;
+  out->nnz = A->nnz;
+  cudaMemcpyKind kind = A->on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+  NM_CUDA(cudaMalloc(&out->rp, sizeof(int64_t) * (A->n + 1)));
+  NM_CUDA(cudaMalloc(&out->ci, sizeof(int32_t) * (A->nnz > 0 ? A->nnz : 1)));
+  NM_CUDA(cudaMemcpyAsync(out->rp, A->rowptr, sizeof(int64_t) * (A->n + 1), kind, s));
+  if (A->nnz > 0)
+    NM_CUDA(cudaMemcpyAsync(out->ci, A->col, sizeof(int32_t) * A->nnz, kind, s));
+  if (A->val) {
+    NM_CUDA(cudaMalloc(&out->val, sizeof(uint16_t) * (A->nnz > 0 ? A->nnz : 1)));
+    if (A->nnz > 0) {
+      if (A->val_dtype == dtype) {
+        NM_CUDA(cudaMemcpyAsync(out->val, A->val, sizeof(uint16_t) * A->nnz, kind, s));
+      } else {
+        const void* src = A->val;
+        void* tmp = nullptr;
+        size_t esz = A->val_dtype == NM_F32 ? 4 : 2;
+        if (!A->on_device) {
+          NM_CUDA(cudaMalloc(&tmp, esz * A->nnz));
+          NM_CUDA(cudaMemcpyAsync(tmp, A->val, esz * A->nnz, cudaMemcpyHostToDevice, s));
+          src = tmp;
+        }
+        k_convert_vals<<<1184, 256, 0, s>>>(src, A->val_dtype, out->val, dtype, A->nnz);
+        NM_CUDA(cudaGetLastError());
+        if (tmp) {
+          NM_CUDA(cudaStreamSynchronize(s));
+          cudaFree(tmp);
+        }
+      }
+    }
+  }
+  return NM_OK;
+}
+
+nm_status host_csr(const nm_csr* A, int64_t** rp, int32_t** ci) {
+  *rp = (int64_t*)malloc(sizeof(int64_t) * (A->n + 1));
+  *ci = (int32_t*)malloc(sizeof(int32_t) * (A->nnz > 0 ? A->nnz : 1));
+  if (!*rp || !*ci) return fail(NM_ERR_OOM, "host allocation");
+  if (A->on_device) {
+    NM_CUDA(cudaMemcpy(*rp, A->rowptr, sizeof(int64_t) * (A->n + 1), cudaMemcpyDeviceToHost));
+    if (A->nnz) NM_CUDA(cudaMemcpy(*ci, A->col, sizeof(int32_t) * A->nnz, cudaMemcpyDeviceToHost));
+  } else {
+    memcpy(*rp, A->rowptr, sizeof(int64_t) * (A->n + 1));
+    if (A->nnz) memcpy(*ci, A->col, sizeof(int32_t) * A->nnz);
+  }
+  return NM_OK;
+}
+
+}  // namespace nm
+
+using namespace nm;
+
+extern "C" {
+
+const char* nm_status_string(nm_status s) {
+  switch (s) {
+    case NM_OK: return "NM_OK";
+    case NM_ERR_INVALID_ARG: return "NM_ERR_INVALID_ARG";
+    case NM_ERR_UNSUPPORTED: return "NM_ERR_UNSUPPORTED";
+    case NM_ERR_BAD_CSR: return "NM_ERR_BAD_CSR";
+    case NM_ERR_NOT_SYMMETRIC: return "NM_ERR_NOT_SYMMETRIC";
+    case NM_ERR_CUDA: return "NM_ERR_CUDA";
+    case NM_ERR_OOM: return "NM_ERR_OOM";
+  }
+  return "NM_ERR_UNKNOWN";
+}
+
+const char* nm_last_error(void) { return g_last_error.c_str(); }
+
+int nm_version(void) { return 1; }
+
+void nm_packed_free(nm_packed* P) {
+  if (!P) return;
+  int cur = 0;
+  cudaGetDevice(&cur);
+  cudaSetDevice(P->device);
+  void* ptrs[] = {P->panel_mb_ptr, P->panel_chunk_ptr, P->unit_order, P->mb_seg, P->mb_sel,
+                  P->image, P->xrow, P->res_rowptr, P->res_col, P->res_val};
+  for (void* p : ptrs)
+    if (p) cudaFree(p);
+  cudaSetDevice(cur);
+  delete P;
+}
+
+nm_status nm_packed_info(const nm_packed* P, int64_t* n_mb, int64_t* packed_nnz,
+                         int64_t* residual_nnz, int64_t* device_bytes, int64_t* n_chunks) {
+  if (!P) return fail(NM_ERR_INVALID_ARG, "nm_packed_info: NULL handle");
+  if (n_mb) *n_mb = P->n_mb;
+  if (packed_nnz) *packed_nnz = P->packed_nnz;
+  if (residual_nnz) *residual_nnz = P->res_nnz;
+  if (device_bytes) *device_bytes = (int64_t)P->device_bytes;
+  if (n_chunks) *n_chunks = P->n_chunks;
+  return NM_OK;
+}
+
+nm_status nm_export_canonical(const nm_packed* P, int64_t* panel_ptr, int32_t* mb_seg,
+                              uint8_t* sel, uint8_t* nib, uint16_t* vals, int64_t* res_rowptr,
+                              int32_t* res_col, uint16_t* res_val) {
+  if (!P) return fail(NM_ERR_INVALID_ARG, "nm_export_canonical: NULL handle");
+  int cur = 0;
+  NM_CUDA(cudaGetDevice(&cur));
+  NM_CUDA(cudaSetDevice(P->device));
+  const int64_t rows = P->row_end - P->row_begin;
+  std::vector<int64_t> mbp(P->n_panels + 1), chp(P->n_panels + 1);
+  NM_CUDA(cudaMemcpy(mbp.data(), P->panel_mb_ptr, sizeof(int64_t) * (P->n_panels + 1),
+                     cudaMemcpyDeviceToHost));
+  NM_CUDA(cudaMemcpy(chp.data(), P->panel_chunk_ptr, sizeof(int64_t) * (P->n_panels + 1),
+                     cudaMemcpyDeviceToHost));
+  if (panel_ptr) memcpy(panel_ptr, mbp.data(), sizeof(int64_t) * (P->n_panels + 1));
+  if (mb_seg && P->n_mb)
+    NM_CUDA(cudaMemcpy(mb_seg, P->mb_seg, sizeof(int32_t) * P->n_mb, cudaMemcpyDeviceToHost));
+  if (sel && P->n_mb) {
+    std::vector<uint32_t> s(P->n_mb);
+    NM_CUDA(cudaMemcpy(s.data(), P->mb_sel, sizeof(uint32_t) * P->n_mb, cudaMemcpyDeviceToHost));
+    for (int64_t m = 0; m < P->n_mb; ++m)
+      for (int j = 0; j < 4; ++j) sel[m * 4 + j] = (uint8_t)((s[m] >> (8 * j)) & 0xFF);
+  }
+  if ((nib || vals) && P->n_mb) {
+    std::vector<uint8_t> img((size_t)P->n_chunks * kChunkBytes);
+    NM_CUDA(cudaMemcpy(img.data(), P->image, img.size(), cudaMemcpyDeviceToHost));
+    for (int64_t p = 0; p < P->n_panels; ++p) {
+      for (int64_t m = mbp[p]; m < mbp[p + 1]; ++m) {
+        int64_t local = m - mbp[p];
+        int64_t c = chp[p] + local / kChunkMB;
+        int g = (int)(local % kChunkMB);
+        const uint8_t* cv = img.data() + (size_t)c * kChunkBytes;
+        const uint32_t* cm = (const uint32_t*)(cv + kChunkValBytes);
+        for (int r = 0; r < kPanelRows; ++r) {
+          int m0 = r % 8, m1 = (r / 8) % 2, m2 = r / 16, k1 = g / 4, q = g % 4;
+          int lane = m0 + 8 * k1 + 16 * m2;
+          uint32_t w = cm[lane];
+          uint8_t nb = (uint8_t)((w >> (16 * m1 + 4 * q)) & 0xF);
+          if (nib) nib[m * kPanelRows + r] = nb;
+          if (vals) {
+            for (int slot = 0; slot < 2; ++slot) {
+              int k = 2 * g + slot;
+              size_t off = (size_t)(r % 8) * 16 + (size_t)(r / 8) * 256 + (size_t)(k / 8) * 128 +
+                           (size_t)(k % 8) * 2;
+              uint16_t v;
+              memcpy(&v, cv + off, 2);
+              vals[(m * kPanelRows + r) * 2 + slot] = v;
+            }
+          }
+        }
+      }
+    }
+  }
+  if (res_rowptr)
+    NM_CUDA(cudaMemcpy(res_rowptr, P->res_rowptr, sizeof(int64_t) * (rows + 1),
+                       cudaMemcpyDeviceToHost));
+  if (res_col && P->res_nnz)
+    NM_CUDA(cudaMemcpy(res_col, P->res_col, sizeof(int32_t) * P->res_nnz, cudaMemcpyDeviceToHost));
+  if (res_val && P->res_nnz)
+    NM_CUDA(cudaMemcpy(res_val, P->res_val, sizeof(uint16_t) * P->res_nnz, cudaMemcpyDeviceToHost));
+  NM_CUDA(cudaSetDevice(cur));
+  return NM_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,567 @@
+// nm_pack / nm_pack_rows: the sm_100a V:N:M packer (SPTC form of PAPER.md:L492).
+//
+//  1. B = P A P^T for the requested row range (row gather + column relabel + radix sort).
+//  2. Meta-blocks = distinct (panel, segment) pairs with any nonzero, ascending (radix sort +
+//     run-length encode of panel*S + col/Mp keys).
+//  3. Column counts per meta-block -> the k = 4 selected columns (vertical constraint,
+//     L338-339): largest counts, ties to the smaller offset, ascending.
+//  4. Per (row, meta-block): the first <= 2 nonzeros among the selected columns (horizontal
+//     constraint, N = 2) go to the two MMA slots with a 4-bit index pair; the rest to the
+//     residual CSR.  Values and metadata are written straight into the MMA-native image.
+#include <cub/cub.cuh>
+
+#include <algorithm>
+#include <numeric>
+#include <vector>
+
+#include "nm_internal.h"
+
+namespace nm {
+namespace {
+
+constexpr int kWarp = 32;
+
+// byte offset of element (r, k) inside a chunk's value block (UMMA K-major no swizzle,
+// LBO = 128 B between the two 8-element K chunks, SBO = 256 B between 8-row groups)
+__host__ __device__ inline uint32_t val_off(int r, int k) {
+  return (uint32_t)((r & 7) * 16 + (r >> 3) * 256 + (k >> 3) * 128 + (k & 7) * 2);
+}
+// tensor-memory lane word and bit shift of the nibble of row r, meta-block g of a chunk
+__host__ __device__ inline void meta_pos(int r, int g, int* word, int* shift) {
+  int m0 = r & 7, m1 = (r >> 3) & 1, m2 = r >> 4, k1 = g >> 2, q = g & 3;
+  *word = m0 + 8 * k1 + 16 * m2;
+  *shift = 16 * m1 + 4 * q;
+}
+
+__global__ void k_iperm(const int32_t* __restrict__ perm, int32_t* __restrict__ iperm, int64_t n) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x)
+    iperm[perm[p]] = (int32_t)p;
+}
+
+__global__ void k_identity(int32_t* __restrict__ perm, int64_t n) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x)
+    perm[p] = (int32_t)p;
+}
+
+// deg[l] = degree of B row rb + l
+__global__ void k_row_deg(const int64_t* __restrict__ rp, const int32_t* __restrict__ perm,
+                          int64_t rb, int64_t rows, int64_t* __restrict__ deg) {
+  for (int64_t l = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; l < rows;
+       l += (int64_t)gridDim.x * blockDim.x) {
+    int32_t u = perm[rb + l];
+    deg[l] = rp[u + 1] - rp[u];
+  }
+}
+
+// key = local_row << 32 | new_col, value = 16-bit value bits (warp per row)
+__global__ void k_fill_keys(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
+                            const uint16_t* __restrict__ val, uint16_t one,
+                            const int32_t* __restrict__ perm, const int32_t* __restrict__ iperm,
+                            int64_t rb, int64_t rows, const int64_t* __restrict__ Brp,
+                            uint64_t* __restrict__ key, uint16_t* __restrict__ v16) {
+  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kWarp;
+  int lane = threadIdx.x % kWarp;
+  int64_t nw = (int64_t)gridDim.x * blockDim.x / kWarp;
+  for (int64_t l = warp; l < rows; l += nw) {
+    int32_t u = perm[rb + l];
+    int64_t s = rp[u], d = rp[u + 1] - s, o = Brp[l];
+    for (int64_t k = lane; k < d; k += kWarp) {
+      key[o + k] = ((uint64_t)l << 32) | (uint32_t)iperm[ci[s + k]];
+      v16[o + k] = val ? val[s + k] : one;
+    }
+  }
+}
+
+__global__ void k_split_keys(const uint64_t* __restrict__ key, int32_t* __restrict__ Bci,
+                             int64_t nnz) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nnz;
+       k += (int64_t)gridDim.x * blockDim.x)
+    Bci[k] = (int32_t)(key[k] & 0xFFFFFFFFu);
+}
+
+// meta-block key of every entry: panel * S + col / Mp (warp per row)
+__global__ void k_mbkey(const int64_t* __restrict__ Brp, const int32_t* __restrict__ Bci,
+                        int64_t rows, int Mp, int64_t S, int64_t* __restrict__ key) {
+  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kWarp;
+  int lane = threadIdx.x % kWarp;
+  int64_t nw = (int64_t)gridDim.x * blockDim.x / kWarp;
+  for (int64_t l = warp; l < rows; l += nw) {
+    int64_t panel = l / kPanelRows;
+    for (int64_t k = Brp[l] + lane; k < Brp[l + 1]; k += kWarp)
+      key[k] = panel * S + Bci[k] / Mp;
+  }
+}
+
+__device__ inline int64_t lower_bound64(const int64_t* __restrict__ a, int64_t n, int64_t x) {
+  int64_t lo = 0, hi = n;
+  while (lo < hi) {
+    int64_t mid = (lo + hi) >> 1;
+    if (a[mid] < x) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+// panel_mb_ptr[r] = first meta-block of panel r; chunk counts per panel
+__global__ void k_panel_ptr(const int64_t* __restrict__ mbkey, int64_t n_mb, int64_t P,
+                            int64_t S, int64_t* __restrict__ mbp, int64_t* __restrict__ nchunk) {
+  for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r <= P;
+       r += (int64_t)gridDim.x * blockDim.x) {
+    mbp[r] = lower_bound64(mbkey, n_mb, r * S);
+  }
+}
+
+__global__ void k_chunk_counts(const int64_t* __restrict__ mbp, int64_t P,
+                               int64_t* __restrict__ nchunk) {
+  for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < P;
+       r += (int64_t)gridDim.x * blockDim.x)
+    nchunk[r] = (mbp[r + 1] - mbp[r] + kChunkMB - 1) / kChunkMB;
+}
+
+__global__ void k_meta_init(uint8_t* __restrict__ image, int64_t n_chunks) {
+  int64_t total = n_chunks * (kChunkMetaBytes / 4);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t c = i / (kChunkMetaBytes / 4), w = i % (kChunkMetaBytes / 4);
+    ((uint32_t*)(image + c * kChunkBytes + kChunkValBytes))[w] = kMetaNone;
+  }
+}
+
+__global__ void k_fill_i32(int32_t* __restrict__ a, int64_t n, int32_t v) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    a[i] = v;
+}
+
+// per-entry meta-block id and column counts (warp per row)
+__global__ void k_colcount(const int64_t* __restrict__ Brp, const int32_t* __restrict__ Bci,
+                           int64_t rows, int Mp, int64_t S, const int64_t* __restrict__ mbkey,
+                           int64_t n_mb, int32_t* __restrict__ cnt, int64_t* __restrict__ emb) {
+  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kWarp;
+  int lane = threadIdx.x % kWarp;
+  int64_t nw = (int64_t)gridDim.x * blockDim.x / kWarp;
+  for (int64_t l = warp; l < rows; l += nw) {
+    int64_t panel = l / kPanelRows;
+    for (int64_t k = Brp[l] + lane; k < Brp[l + 1]; k += kWarp) {
+      int64_t s = Bci[k] / Mp;
+      int64_t m = lower_bound64(mbkey, n_mb, panel * S + s);
+      emb[k] = m;
+      atomicAdd(&cnt[m * Mp + (Bci[k] - s * Mp)], 1);
+    }
+  }
+}
+
+// selected columns (4 largest counts, ties -> smaller offset, ascending) and X row indices
+__global__ void k_select(const int32_t* __restrict__ cnt, int Mp, int64_t n_mb,
+                         const int64_t* __restrict__ mbkey, int64_t S, int64_t n,
+                         const int64_t* __restrict__ mbp, const int64_t* __restrict__ chp,
+                         int64_t P, int32_t* __restrict__ mb_seg, uint32_t* __restrict__ mb_sel,
+                         int32_t* __restrict__ xrow) {
+  for (int64_t m = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; m < n_mb;
+       m += (int64_t)gridDim.x * blockDim.x) {
+    int64_t panel = mbkey[m] / S, s = mbkey[m] % S;
+    mb_seg[m] = (int32_t)s;
+    const int32_t* c = cnt + m * Mp;
+    int sel[4];
+    if (Mp == 4) {
+      sel[0] = 0; sel[1] = 1; sel[2] = 2; sel[3] = 3;
+    } else {
+      uint32_t taken = 0;
+      for (int t = 0; t < 4; ++t) {
+        int bj = -1;
+        for (int j = 0; j < Mp; ++j) {
+          if (taken & (1u << j)) continue;
+          if (bj < 0 || c[j] > c[bj]) bj = j;
+        }
+        taken |= 1u << bj;
+        sel[t] = bj;
+      }
+      // ascending
+      for (int a = 0; a < 4; ++a)
+        for (int b = a + 1; b < 4; ++b)
+          if (sel[b] < sel[a]) { int t = sel[a]; sel[a] = sel[b]; sel[b] = t; }
+    }
+    mb_sel[m] = (uint32_t)sel[0] | ((uint32_t)sel[1] << 8) | ((uint32_t)sel[2] << 16) |
+                ((uint32_t)sel[3] << 24);
+    int64_t local = m - mbp[panel];
+    int64_t chunk = chp[panel] + local / kChunkMB;
+    int g = (int)(local % kChunkMB);
+    for (int j = 0; j < 4; ++j) {
+      int64_t col = s * Mp + sel[j];
+      // zero-count or phantom columns gather nothing (zero-filled operand rows)
+      xrow[chunk * 32 + g * 4 + j] = (col < n && c[sel[j]] > 0) ? (int32_t)col : -1;
+    }
+  }
+}
+
+// Places every entry: MMA slot (value + nibble) or residual flag.  One thread per entry; the
+// entry inspects its (row, segment) group, which is contiguous and at most Mp long.
+__global__ void k_place(const int64_t* __restrict__ Brp, const int32_t* __restrict__ Bci,
+                        const uint16_t* __restrict__ Bval, int64_t rows, int Mp,
+                        const int64_t* __restrict__ emb, const uint32_t* __restrict__ mb_sel,
+                        const int64_t* __restrict__ mbkey, int64_t S,
+                        const int64_t* __restrict__ mbp, const int64_t* __restrict__ chp,
+                        uint8_t* __restrict__ image, uint8_t* __restrict__ resflag,
+                        unsigned long long* __restrict__ kept_count) {
+  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kWarp;
+  int lane = threadIdx.x % kWarp;
+  int64_t nw = (int64_t)gridDim.x * blockDim.x / kWarp;
+  for (int64_t l = warp; l < rows; l += nw) {
+    int64_t b = Brp[l], e = Brp[l + 1];
+    for (int64_t k = b + lane; k < e; k += kWarp) {
+      int32_t col = Bci[k];
+      int64_t s = col / Mp;
+      uint32_t sel = mb_sel[emb[k]];
+      auto jof = [&](int32_t c) -> int {
+        int off = c - (int)(s * Mp);
+        for (int j = 0; j < 4; ++j)
+          if ((int)((sel >> (8 * j)) & 0xFF) == off) return j;
+        return -1;
+      };
+      // group bounds
+      int64_t gs = k;
+      while (gs > b && Bci[gs - 1] / Mp == s) --gs;
+      int64_t ge = k + 1;
+      while (ge < e && Bci[ge] / Mp == s) ++ge;
+      int jk = jof(col);
+      int rank = 0, ja = -1, jb = -1;
+      int64_t ka = -1;
+      for (int64_t t = gs; t < ge; ++t) {
+        int jt = jof(Bci[t]);
+        if (jt < 0) continue;
+        if (t < k) ++rank;
+        if (ja < 0) { ja = jt; ka = t; }
+        else if (jb < 0) { jb = jt; }
+      }
+      bool kept = jk >= 0 && rank < 2;
+      resflag[k] = kept ? 0 : 1;
+      if (!kept) continue;
+      atomicAdd(kept_count, 1ull);
+      int64_t m = emb[k];
+      int64_t panel = l / kPanelRows;
+      int64_t local = m - mbp[panel];
+      int64_t chunk = chp[panel] + local / kChunkMB;
+      int g = (int)(local % kChunkMB);
+      int r = (int)(l % kPanelRows);
+      uint8_t* cv = image + chunk * kChunkBytes;
+      // slot assignment (reading #19): two kept (a<b) -> (a,b) slots 0,1; one kept
+      // at j<3 -> (j,3) slot 0; one kept at j=3 -> (0,3) slot 1
+      int i0, i1, slot;
+      if (jb >= 0) { i0 = ja; i1 = jb; slot = (k == ka) ? 0 : 1; }
+      else if (ja < 3) { i0 = ja; i1 = 3; slot = 0; }
+      else { i0 = 0; i1 = 3; slot = 1; }
+      *(uint16_t*)(cv + val_off(r, 2 * g + slot)) = Bval[k];
+      if (k == ka) {
+        int w, sh;
+        meta_pos(r, g, &w, &sh);
+        uint32_t nib = (uint32_t)(i0 | (i1 << 2));
+        atomicXor((uint32_t*)(cv + kChunkValBytes) + w, (nib ^ 0x4u) << sh);
+      }
+      (void)mbkey;
+      (void)S;
+    }
+  }
+}
+
+__global__ void k_res_count(const int64_t* __restrict__ Brp, const uint8_t* __restrict__ resflag,
+                            int64_t rows, int64_t* __restrict__ rc) {
+  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kWarp;
+  int lane = threadIdx.x % kWarp;
+  int64_t nw = (int64_t)gridDim.x * blockDim.x / kWarp;
+  for (int64_t l = warp; l < rows; l += nw) {
+    int64_t c = 0;
+    for (int64_t k = Brp[l] + lane; k < Brp[l + 1]; k += kWarp) c += resflag[k];
+    for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+    if (lane == 0) rc[l] = c;
+  }
+}
+
+__global__ void k_res_fill(const int64_t* __restrict__ Brp, const int32_t* __restrict__ Bci,
+                           const uint16_t* __restrict__ Bval, const uint8_t* __restrict__ resflag,
+                           int64_t rows, const int64_t* __restrict__ rrp,
+                           int32_t* __restrict__ rci, uint16_t* __restrict__ rval) {
+  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kWarp;
+  int lane = threadIdx.x % kWarp;
+  int64_t nw = (int64_t)gridDim.x * blockDim.x / kWarp;
+  for (int64_t l = warp; l < rows; l += nw) {
+    int64_t o = rrp[l];
+    for (int64_t base = Brp[l]; base < Brp[l + 1]; base += kWarp) {
+      int64_t k = base + lane;
+      int f = (k < Brp[l + 1]) ? resflag[k] : 0;
+      unsigned mask = __ballot_sync(0xffffffffu, f);
+      if (f) {
+        int pos = __popc(mask & ((1u << lane) - 1));
+        rci[o + pos] = Bci[k];
+        rval[o + pos] = Bval[k];
+      }
+      o += __popc(mask);
+    }
+  }
+}
+
+struct DevBuf {
+  void* p = nullptr;
+  cudaStream_t s = nullptr;
+  DevBuf() = default;
+  DevBuf(const DevBuf&) = delete;
+  ~DevBuf() {
+    if (p) cudaFreeAsync(p, s);
+  }
+  template <typename T>
+  T* as() { return (T*)p; }
+};
+
+inline nm_status dalloc(DevBuf& b, size_t bytes, cudaStream_t s) {
+  b.s = s;
+  NM_CUDA(cudaMallocAsync(&b.p, bytes > 0 ? bytes : 16, s));
+  return NM_OK;
+}
+
+#define NM_TRY(x)                  \
+  do {                             \
+    nm_status st_ = (x);           \
+    if (st_ != NM_OK) return st_;  \
+  } while (0)
+
+inline int grid_for(int64_t work, int block) {
+  int64_t g = (work + block - 1) / block;
+  if (g < 1) g = 1;
+  if (g > 148 * 16) g = 148 * 16;
+  return (int)g;
+}
+
+nm_status scan_excl(const int64_t* in, int64_t* out, int64_t n, cudaStream_t s) {
+  size_t bytes = 0;
+  NM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, bytes, in, out, n, s));
+  DevBuf tmp;
+  NM_TRY(dalloc(tmp, bytes, s));
+  NM_CUDA(cub::DeviceScan::ExclusiveSum(tmp.p, bytes, in, out, n, s));
+  return NM_OK;
+}
+
+nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int M, int Vp,
+                    nm_dtype dtype, int64_t rb, int64_t re, cudaStream_t s, nm_packed** out) {
+  if (!A || !out) return fail(NM_ERR_INVALID_ARG, "nm_pack: NULL argument");
+  if (N != 2) return fail(NM_ERR_UNSUPPORTED, "nm_pack: N must be 2 (hardware 2:4, L496)");
+  if (!(M == 4 || M == 8 || M == 16)) return fail(NM_ERR_UNSUPPORTED, "nm_pack: M must be 4, 8 or 16");
+  if (V < 1) return fail(NM_ERR_INVALID_ARG, "nm_pack: V < 1");
+  if (Vp == 0) Vp = kPanelRows;
+  if (Vp != kPanelRows) return fail(NM_ERR_UNSUPPORTED, "nm_pack: Vp must be 128");
+  if (dtype != NM_F16 && dtype != NM_BF16) return fail(NM_ERR_UNSUPPORTED, "nm_pack: dtype must be f16 or bf16");
+  const int64_t n = A->n;
+  if (n <= 0 || A->nnz < 0) return fail(NM_ERR_INVALID_ARG, "nm_pack: empty graph");
+  if (n >= (int64_t)1 << 31) return fail(NM_ERR_UNSUPPORTED, "nm_pack: n >= 2^31");
+  if (rb < 0 || re > n || rb > re || rb % Vp != 0)
+    return fail(NM_ERR_INVALID_ARG, "nm_pack_rows: bad row range (row_begin must be a multiple of Vp)");
+  const int Mp = (V == 1) ? 4 : M;
+  const int64_t rows = re - rb;
+  const int64_t P = (rows + Vp - 1) / Vp;
+  const int64_t S = (n + Mp - 1) / Mp;
+
+  if (!A->on_device) {
+    nm_status st = validate_csr_host(n, A->rowptr, A->col, false);
+    if (st != NM_OK) return st;
+  }
+  DevCsr dA;
+  NM_TRY(upload_csr(A, dtype, &dA, s));
+
+  DevBuf d_perm, d_iperm;
+  NM_TRY(dalloc(d_perm, sizeof(int32_t) * n, s));
+  NM_TRY(dalloc(d_iperm, sizeof(int32_t) * n, s));
+  if (perm_host) {
+    // validate the permutation on the host
+    std::vector<uint8_t> seen(n, 0);
+    for (int64_t p = 0; p < n; ++p) {
+      int32_t v = perm_host[p];
+      if (v < 0 || v >= n || seen[v]) return fail(NM_ERR_INVALID_ARG, "nm_pack: perm is not a permutation");
+      seen[v] = 1;
+    }
+    NM_CUDA(cudaMemcpyAsync(d_perm.p, perm_host, sizeof(int32_t) * n, cudaMemcpyHostToDevice, s));
+  } else {
+    k_identity<<<grid_for(n, 256), 256, 0, s>>>(d_perm.as<int32_t>(), n);
+  }
+  k_iperm<<<grid_for(n, 256), 256, 0, s>>>(d_perm.as<int32_t>(), d_iperm.as<int32_t>(), n);
+
+  // ---- 1. B rows [rb, re) ----
+  DevBuf d_deg, d_Brp;
+  NM_TRY(dalloc(d_deg, sizeof(int64_t) * (rows + 1), s));
+  NM_TRY(dalloc(d_Brp, sizeof(int64_t) * (rows + 1), s));
+  NM_CUDA(cudaMemsetAsync(d_deg.p, 0, sizeof(int64_t) * (rows + 1), s));
+  k_row_deg<<<grid_for(rows, 256), 256, 0, s>>>(dA.rp, d_perm.as<int32_t>(), rb, rows, d_deg.as<int64_t>());
+  NM_TRY(scan_excl(d_deg.as<int64_t>(), d_Brp.as<int64_t>(), rows + 1, s));
+  int64_t bnnz = 0;
+  NM_CUDA(cudaMemcpyAsync(&bnnz, d_Brp.as<int64_t>() + rows, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  NM_CUDA(cudaStreamSynchronize(s));
+
+  DevBuf d_key, d_key2, d_v, d_v2, d_Bci;
+  NM_TRY(dalloc(d_key, sizeof(uint64_t) * bnnz, s));
+  NM_TRY(dalloc(d_key2, sizeof(uint64_t) * bnnz, s));
+  NM_TRY(dalloc(d_v, sizeof(uint16_t) * bnnz, s));
+  NM_TRY(dalloc(d_v2, sizeof(uint16_t) * bnnz, s));
+  NM_TRY(dalloc(d_Bci, sizeof(int32_t) * bnnz, s));
+  k_fill_keys<<<grid_for(rows * 32, 256), 256, 0, s>>>(
+      dA.rp, dA.ci, dA.val, one_bits(dtype), d_perm.as<int32_t>(), d_iperm.as<int32_t>(), rb,
+      rows, d_Brp.as<int64_t>(), d_key.as<uint64_t>(), d_v.as<uint16_t>());
+  NM_CUDA(cudaGetLastError());
+  {
+    int end_bit = 32;
+    while (end_bit < 64 && (((uint64_t)rows) >> (end_bit - 32)) != 0) ++end_bit;
+    size_t bytes = 0;
+    NM_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, bytes, d_key.as<uint64_t>(), d_key2.as<uint64_t>(),
+                                            d_v.as<uint16_t>(), d_v2.as<uint16_t>(), bnnz, 0, end_bit, s));
+    DevBuf tmp;
+    NM_TRY(dalloc(tmp, bytes, s));
+    NM_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, bytes, d_key.as<uint64_t>(), d_key2.as<uint64_t>(),
+                                            d_v.as<uint16_t>(), d_v2.as<uint16_t>(), bnnz, 0, end_bit, s));
+  }
+  k_split_keys<<<grid_for(bnnz, 256), 256, 0, s>>>(d_key2.as<uint64_t>(), d_Bci.as<int32_t>(), bnnz);
+  const int32_t* Bci = d_Bci.as<int32_t>();
+  const uint16_t* Bval = d_v2.as<uint16_t>();
+  const int64_t* Brp = d_Brp.as<int64_t>();
+
+  // ---- 2. meta-blocks ----
+  DevBuf d_mk, d_mk2, d_mbkey, d_runs, d_nruns;
+  NM_TRY(dalloc(d_mk, sizeof(int64_t) * bnnz, s));
+  NM_TRY(dalloc(d_mk2, sizeof(int64_t) * bnnz, s));
+  NM_TRY(dalloc(d_mbkey, sizeof(int64_t) * bnnz, s));
+  NM_TRY(dalloc(d_runs, sizeof(int64_t) * bnnz, s));
+  NM_TRY(dalloc(d_nruns, sizeof(int64_t), s));
+  k_mbkey<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, rows, Mp, S, d_mk.as<int64_t>());
+  {
+    size_t bytes = 0;
+    NM_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, bytes, d_mk.as<int64_t>(), d_mk2.as<int64_t>(), bnnz, 0, 64, s));
+    DevBuf tmp;
+    NM_TRY(dalloc(tmp, bytes, s));
+    NM_CUDA(cub::DeviceRadixSort::SortKeys(tmp.p, bytes, d_mk.as<int64_t>(), d_mk2.as<int64_t>(), bnnz, 0, 64, s));
+  }
+  {
+    size_t bytes = 0;
+    NM_CUDA(cub::DeviceRunLengthEncode::Encode(nullptr, bytes, d_mk2.as<int64_t>(), d_mbkey.as<int64_t>(),
+                                               d_runs.as<int64_t>(), d_nruns.as<int64_t>(), bnnz, s));
+    DevBuf tmp;
+    NM_TRY(dalloc(tmp, bytes, s));
+    NM_CUDA(cub::DeviceRunLengthEncode::Encode(tmp.p, bytes, d_mk2.as<int64_t>(), d_mbkey.as<int64_t>(),
+                                               d_runs.as<int64_t>(), d_nruns.as<int64_t>(), bnnz, s));
+  }
+  int64_t n_mb = 0;
+  if (bnnz > 0) {
+    NM_CUDA(cudaMemcpyAsync(&n_mb, d_nruns.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    NM_CUDA(cudaStreamSynchronize(s));
+  }
+
+  nm_packed* Pk = new nm_packed();
+  NM_CUDA(cudaGetDevice(&Pk->device));
+  Pk->n = n; Pk->row_begin = rb; Pk->row_end = re;
+  Pk->V = V; Pk->N = N; Pk->M = M; Pk->Vp = Vp; Pk->Mp = Mp; Pk->dtype = dtype;
+  Pk->n_panels = P; Pk->n_mb = n_mb;
+  struct Guard {
+    nm_packed* p;
+    bool ok = false;
+    ~Guard() { if (!ok) nm_packed_free(p); }
+  } guard{Pk};
+  auto palloc = [&](void** ptr, size_t bytes) -> nm_status {
+    NM_CUDA(cudaMalloc(ptr, bytes > 0 ? bytes : 16));
+    Pk->device_bytes += bytes;
+    return NM_OK;
+  };
+  NM_TRY(palloc((void**)&Pk->panel_mb_ptr, sizeof(int64_t) * (P + 1)));
+  NM_TRY(palloc((void**)&Pk->panel_chunk_ptr, sizeof(int64_t) * (P + 1)));
+  k_panel_ptr<<<grid_for(P + 1, 256), 256, 0, s>>>(d_mbkey.as<int64_t>(), n_mb, P, S, Pk->panel_mb_ptr, nullptr);
+  DevBuf d_nch;
+  NM_TRY(dalloc(d_nch, sizeof(int64_t) * (P + 1), s));
+  NM_CUDA(cudaMemsetAsync(d_nch.p, 0, sizeof(int64_t) * (P + 1), s));
+  k_chunk_counts<<<grid_for(P, 256), 256, 0, s>>>(Pk->panel_mb_ptr, P, d_nch.as<int64_t>());
+  NM_TRY(scan_excl(d_nch.as<int64_t>(), Pk->panel_chunk_ptr, P + 1, s));
+  std::vector<int64_t> chp(P + 1);
+  NM_CUDA(cudaMemcpyAsync(chp.data(), Pk->panel_chunk_ptr, sizeof(int64_t) * (P + 1), cudaMemcpyDeviceToHost, s));
+  NM_CUDA(cudaStreamSynchronize(s));
+  const int64_t n_chunks = chp[P];
+  Pk->n_chunks = n_chunks;
+
+  // unit order: panels with most chunks first (stable) -- greedy balance for the persistent grid
+  {
+    std::vector<int32_t> order(P);
+    std::iota(order.begin(), order.end(), 0);
+    std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+      return (chp[a + 1] - chp[a]) > (chp[b + 1] - chp[b]);
+    });
+    NM_TRY(palloc((void**)&Pk->unit_order, sizeof(int32_t) * P));
+    NM_CUDA(cudaMemcpyAsync(Pk->unit_order, order.data(), sizeof(int32_t) * P, cudaMemcpyHostToDevice, s));
+    NM_CUDA(cudaStreamSynchronize(s));
+  }
+
+  NM_TRY(palloc((void**)&Pk->mb_seg, sizeof(int32_t) * n_mb));
+  NM_TRY(palloc((void**)&Pk->mb_sel, sizeof(uint32_t) * n_mb));
+  NM_TRY(palloc((void**)&Pk->image, (size_t)kChunkBytes * n_chunks));
+  NM_TRY(palloc((void**)&Pk->xrow, sizeof(int32_t) * 32 * n_chunks));
+  NM_CUDA(cudaMemsetAsync(Pk->image, 0, (size_t)kChunkBytes * n_chunks, s));
+  if (n_chunks) {
+    k_meta_init<<<grid_for(n_chunks * 128, 256), 256, 0, s>>>(Pk->image, n_chunks);
+    k_fill_i32<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(Pk->xrow, n_chunks * 32, -1);
+  }
+
+  // ---- 3. column counts and selection ----
+  DevBuf d_cnt, d_emb;
+  NM_TRY(dalloc(d_cnt, sizeof(int32_t) * Mp * (n_mb > 0 ? n_mb : 1), s));
+  NM_TRY(dalloc(d_emb, sizeof(int64_t) * bnnz, s));
+  NM_CUDA(cudaMemsetAsync(d_cnt.p, 0, sizeof(int32_t) * Mp * (n_mb > 0 ? n_mb : 1), s));
+  if (bnnz) {
+    k_colcount<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, rows, Mp, S, d_mbkey.as<int64_t>(), n_mb,
+                                                       d_cnt.as<int32_t>(), d_emb.as<int64_t>());
+    k_select<<<grid_for(n_mb, 256), 256, 0, s>>>(d_cnt.as<int32_t>(), Mp, n_mb, d_mbkey.as<int64_t>(), S, n,
+                                                 Pk->panel_mb_ptr, Pk->panel_chunk_ptr, P, Pk->mb_seg,
+                                                 Pk->mb_sel, Pk->xrow);
+  }
+  NM_CUDA(cudaGetLastError());
+
+  // ---- 4. placement and residual ----
+  DevBuf d_flag, d_kept, d_rc;
+  NM_TRY(dalloc(d_flag, bnnz, s));
+  NM_TRY(dalloc(d_kept, sizeof(unsigned long long), s));
+  NM_TRY(dalloc(d_rc, sizeof(int64_t) * (rows + 1), s));
+  NM_CUDA(cudaMemsetAsync(d_kept.p, 0, sizeof(unsigned long long), s));
+  NM_CUDA(cudaMemsetAsync(d_rc.p, 0, sizeof(int64_t) * (rows + 1), s));
+  if (bnnz) {
+    k_place<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, Bval, rows, Mp, d_emb.as<int64_t>(), Pk->mb_sel,
+                                                    d_mbkey.as<int64_t>(), S, Pk->panel_mb_ptr,
+                                                    Pk->panel_chunk_ptr, Pk->image, d_flag.as<uint8_t>(),
+                                                    d_kept.as<unsigned long long>());
+    k_res_count<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, d_flag.as<uint8_t>(), rows, d_rc.as<int64_t>());
+  }
+  NM_CUDA(cudaGetLastError());
+  NM_TRY(palloc((void**)&Pk->res_rowptr, sizeof(int64_t) * (rows + 1)));
+  NM_TRY(scan_excl(d_rc.as<int64_t>(), Pk->res_rowptr, rows + 1, s));
+  int64_t res_nnz = 0;
+  unsigned long long kept = 0;
+  NM_CUDA(cudaMemcpyAsync(&res_nnz, Pk->res_rowptr + rows, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  NM_CUDA(cudaMemcpyAsync(&kept, d_kept.p, sizeof(kept), cudaMemcpyDeviceToHost, s));
+  NM_CUDA(cudaStreamSynchronize(s));
+  Pk->res_nnz = res_nnz;
+  Pk->packed_nnz = (int64_t)kept;
+  NM_TRY(palloc((void**)&Pk->res_col, sizeof(int32_t) * res_nnz));
+  NM_TRY(palloc((void**)&Pk->res_val, sizeof(uint16_t) * res_nnz));
+  if (res_nnz)
+    k_res_fill<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, Bval, d_flag.as<uint8_t>(), rows,
+                                                       Pk->res_rowptr, Pk->res_col, Pk->res_val);
+  NM_CUDA(cudaGetLastError());
+  NM_CUDA(cudaStreamSynchronize(s));
+  guard.ok = true;
+  *out = Pk;
+  return NM_OK;
+}
+
+}  // namespace
+}  // namespace nm
+
+extern "C" nm_status nm_pack(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
+                             nm_dtype dtype, void* stream, nm_packed** out) {
+  if (!A) return nm::fail(NM_ERR_INVALID_ARG, "nm_pack: NULL graph");
+  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, 0, A->n, (cudaStream_t)stream, out);
+}
+
+extern "C" nm_status nm_pack_rows(const nm_csr* A, const int32_t* perm, int V, int N, int M,
+                                  int Vp, nm_dtype dtype, int64_t row_begin, int64_t row_end,
+                                  void* stream, nm_packed** out) {
+  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, (cudaStream_t)stream, out);
+}

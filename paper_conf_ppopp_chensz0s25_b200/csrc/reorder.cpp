@@ -1,0 +1,396 @@
+// nm_reorder: the SGRP heuristic of PAPER.md §4 (Alg. 1-3), deterministic and bit-identical
+// to the CPU oracle under the readings of DESIGN.md §3.  Runs on the host (the greedy Stage-2
+// is inherently sequential: every recorded pair changes which positions are still fresh);
+// the per-row counting loops are OpenMP-parallel.  Works on the graph in its original labels
+// through perm / iperm instead of materialising B = P A P^T.
+#include <algorithm>
+#include <chrono>
+#include <cstdint>
+#include <cstring>
+#include <numeric>
+#include <vector>
+
+#include "nm_internal.h"
+
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+namespace nm {
+namespace {
+
+struct Graph {
+  int64_t n = 0;
+  const int64_t* rp = nullptr;
+  const int32_t* ci = nullptr;
+  int64_t deg(int64_t v) const { return rp[v + 1] - rp[v]; }
+};
+
+// rank of b in the binary reflected Gray order = inverse Gray code (reading #1)
+inline int64_t hamming_rank(uint64_t b) {
+  uint64_t h = b;
+  for (int sh = 1; sh < 64; sh <<= 1) h ^= h >> sh;
+  return (int64_t)h;
+}
+
+// Per-row segment histogram of B row p: sorted (segment, bits) pairs.
+struct RowSegs {
+  std::vector<int64_t> seg;
+  std::vector<uint32_t> bits;
+  std::vector<int32_t> cnt;
+};
+
+inline void row_segments(const Graph& g, const std::vector<int32_t>& perm, const std::vector<int32_t>& iperm,
+                         int64_t p, int M, std::vector<int32_t>& scratch, RowSegs& out) {
+  const int32_t u = perm[p];
+  scratch.clear();
+  for (int64_t k = g.rp[u]; k < g.rp[u + 1]; ++k) scratch.push_back(iperm[g.ci[k]]);
+  std::sort(scratch.begin(), scratch.end());
+  out.seg.clear();
+  out.bits.clear();
+  out.cnt.clear();
+  for (size_t i = 0; i < scratch.size();) {
+    const int64_t s = scratch[i] / M;
+    uint32_t b = 0;
+    int c = 0;
+    while (i < scratch.size() && scratch[i] / M == s) {
+      b |= 1u << (M - 1 - (scratch[i] - s * M));  // first column of the segment -> MSB
+      ++c;
+      ++i;
+    }
+    out.seg.push_back(s);
+    out.bits.push_back(b);
+    out.cnt.push_back(c);
+  }
+}
+
+// omega and PScore (horizontal constraint, L203 / L396)
+int64_t omega_pscore(const Graph& g, const std::vector<int32_t>& perm, const std::vector<int32_t>& iperm, int N,
+                     int M, std::vector<int32_t>* pscore) {
+  const int64_t S = (g.n + M - 1) / M;
+  if (pscore) pscore->assign(S, 0);
+  int64_t omega = 0;
+#pragma omp parallel reduction(+ : omega)
+  {
+    std::vector<int32_t> scratch;
+    RowSegs rs;
+#pragma omp for schedule(dynamic, 256)
+    for (int64_t p = 0; p < g.n; ++p) {
+      row_segments(g, perm, iperm, p, M, scratch, rs);
+      for (size_t j = 0; j < rs.seg.size(); ++j)
+        if (rs.cnt[j] > N) {
+          ++omega;
+          if (pscore) {
+#pragma omp atomic
+            (*pscore)[rs.seg[j]] += 1;
+          }
+        }
+    }
+  }
+  return omega;
+}
+
+// MBscore: meta-blocks (V rows x M columns) with more than k = 4 distinct nonzero columns
+int64_t mbscore(const Graph& g, const std::vector<int32_t>& perm, const std::vector<int32_t>& iperm, int V,
+                int M) {
+  const int64_t P = (g.n + V - 1) / V;
+  int64_t mb = 0;
+#pragma omp parallel reduction(+ : mb)
+  {
+    std::vector<int32_t> cols;
+#pragma omp for schedule(dynamic, 64)
+    for (int64_t r = 0; r < P; ++r) {
+      cols.clear();
+      const int64_t r1 = std::min<int64_t>(g.n, (r + 1) * (int64_t)V);
+      for (int64_t p = r * (int64_t)V; p < r1; ++p) {
+        const int32_t u = perm[p];
+        for (int64_t k = g.rp[u]; k < g.rp[u + 1]; ++k) cols.push_back(iperm[g.ci[k]]);
+      }
+      std::sort(cols.begin(), cols.end());
+      cols.erase(std::unique(cols.begin(), cols.end()), cols.end());
+      for (size_t i = 0; i < cols.size();) {
+        const int64_t s = cols[i] / M;
+        int d = 0;
+        while (i < cols.size() && cols[i] / M == s) { ++d; ++i; }
+        if (d > 4) ++mb;
+      }
+    }
+  }
+  return mb;
+}
+
+void invert(const std::vector<int32_t>& perm, std::vector<int32_t>& iperm) {
+  iperm.resize(perm.size());
+  for (size_t p = 0; p < perm.size(); ++p) iperm[perm[p]] = (int32_t)p;
+}
+
+// ---- Stage-1: one sort (Alg. 2 lines 4-13) ------------------------------------------------
+void stage1_sort(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>& iperm, int N, int M) {
+  const int64_t n = g.n, S = (n + M - 1) / M;
+  // key of row p: pairs (sgn(c)*(S-s), c) for its nonzero codes in ascending s, then (0,0)
+  std::vector<int64_t> koff(n + 1, 0);
+  std::vector<std::vector<int64_t>> keys(n);
+#pragma omp parallel
+  {
+    std::vector<int32_t> scratch;
+    RowSegs rs;
+#pragma omp for schedule(dynamic, 256)
+    for (int64_t p = 0; p < n; ++p) {
+      row_segments(g, perm, iperm, p, M, scratch, rs);
+      std::vector<int64_t>& k = keys[p];
+      k.clear();
+      k.reserve(2 * rs.seg.size() + 2);
+      for (size_t j = 0; j < rs.seg.size(); ++j) {
+        const int64_t h = hamming_rank(rs.bits[j]);
+        const int64_t c = (rs.cnt[j] > N) ? -h : h;  // negated when violating N:M (L405-411)
+        if (c == 0) continue;
+        k.push_back((c > 0 ? 1 : -1) * (S - rs.seg[j]));
+        k.push_back(c);
+      }
+      k.push_back(0);
+      k.push_back(0);
+    }
+  }
+  std::vector<int64_t> order(n);
+  std::iota(order.begin(), order.end(), 0);
+  std::stable_sort(order.begin(), order.end(), [&](int64_t a, int64_t b) {
+    return std::lexicographical_compare(keys[a].begin(), keys[a].end(), keys[b].begin(), keys[b].end());
+  });
+  std::vector<int32_t> np(n);
+  for (int64_t p = 0; p < n; ++p) np[p] = perm[order[p]];
+  perm.swap(np);
+  invert(perm, iperm);
+}
+
+// ---- Stage-2 (Alg. 3) ----------------------------------------------------------------------
+struct SegCount {
+  // dense per-vertex counters with a touched list: cnt[w] = #vertices of the segment adjacent to w
+  std::vector<int32_t> cnt;
+  std::vector<int32_t> touched;
+  void init(int64_t n) { cnt.assign(n, 0); }
+  void build(const Graph& g, const std::vector<int32_t>& perm, int64_t seg, int M) {
+    clear();
+    for (int64_t q = seg * M; q < std::min<int64_t>(g.n, seg * M + M); ++q) {
+      const int32_t x = perm[q];
+      for (int64_t k = g.rp[x]; k < g.rp[x + 1]; ++k) {
+        const int32_t w = g.ci[k];
+        if (cnt[w] == 0) touched.push_back(w);
+        cnt[w]++;
+      }
+    }
+  }
+  void clear() {
+    for (int32_t w : touched) cnt[w] = 0;
+    touched.clear();
+  }
+};
+
+struct Pair {
+  bool found = false;
+  int64_t g = 0, gp = 0, gt = 0, u = -1, v = -1;
+};
+
+// gains of swapping positions u (segment p) and v (segment t), w.r.t. the pass-start order
+inline void gains(const Graph& g, const std::vector<int32_t>& perm, const SegCount& cp, const SegCount& ct, int N,
+                  int64_t u, int64_t v, int64_t* gp, int64_t* gt) {
+  const int32_t x = perm[u], y = perm[v];
+  int64_t a = g.rp[x], ae = g.rp[x + 1], b = g.rp[y], be = g.rp[y + 1];
+  int64_t sp = 0, st = 0;
+  while (a < ae || b < be) {
+    int32_t w;
+    int d;
+    if (b >= be || (a < ae && g.ci[a] < g.ci[b])) { w = g.ci[a++]; d = -1; }
+    else if (a >= ae || g.ci[b] < g.ci[a]) { w = g.ci[b++]; d = +1; }
+    else { ++a; ++b; continue; }
+    const int c1 = cp.cnt[w], c2 = ct.cnt[w];
+    sp += (c1 > N) - (c1 + d > N);
+    st += (c2 > N) - (c2 - d > N);
+  }
+  *gp = sp;
+  *gt = st;
+}
+
+Pair freshtop(const Graph& g, const std::vector<int32_t>& perm, const SegCount& cp, const SegCount& ct, int N,
+              int M, int64_t p, int64_t t, const std::vector<uint8_t>& used, bool need_positive) {
+  Pair best;
+  for (int64_t u = p * M; u < std::min<int64_t>(g.n, p * M + M); ++u) {
+    if (used[u]) continue;
+    for (int64_t v = t * M; v < std::min<int64_t>(g.n, t * M + M); ++v) {
+      if (used[v]) continue;
+      int64_t gp, gt;
+      gains(g, perm, cp, ct, N, u, v, &gp, &gt);
+      const int64_t gg = gp + gt;
+      if (need_positive && gg <= 0) continue;
+      if (!best.found || gg > best.g) {  // ties keep the smallest (u, v) (reading #18)
+        best.found = true;
+        best.g = gg;
+        best.gp = gp;
+        best.gt = gt;
+        best.u = u;
+        best.v = v;
+      }
+    }
+  }
+  return best;
+}
+
+bool all_used(const std::vector<uint8_t>& used, int64_t seg, int M, int64_t n) {
+  for (int64_t q = seg * M; q < std::min<int64_t>(n, seg * M + M); ++q)
+    if (!used[q]) return false;
+  return true;
+}
+
+int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>& iperm, int N, int M,
+               int maxiter, int gain_rule, int64_t* max_pairs) {
+  const int64_t n = g.n, S = (n + M - 1) / M;
+  int64_t passes = 0;
+  std::vector<int32_t> pscore;
+  std::vector<int64_t> est(S);
+  std::vector<uint8_t> inI(S), used(n);
+  SegCount cp, ct;
+  cp.init(n);
+  ct.init(n);
+  std::vector<int64_t> su, sv;
+  for (int it = 0; it <= maxiter; ++it) {
+    omega_pscore(g, perm, iperm, N, M, &pscore);
+    std::vector<int64_t> I;
+    for (int64_t s = 0; s < S; ++s)
+      if (pscore[s] > 0) I.push_back(s);
+    if (I.empty()) break;
+    std::stable_sort(I.begin(), I.end(), [&](int64_t a, int64_t b) { return pscore[a] > pscore[b]; });
+    for (int64_t s = 0; s < S; ++s) { est[s] = pscore[s]; inI[s] = 0; }
+    for (int64_t s : I) inI[s] = 1;
+    std::fill(used.begin(), used.end(), 0);
+    su.clear();
+    sv.clear();
+    if (I.size() == 1) {
+      const int64_t p = I[0];
+      if (S == 1) break;
+      int64_t t = -1, tn = 0;
+      for (int64_t s = 0; s < S; ++s) {  // the sparsest other segment (reading #16)
+        if (s == p) continue;
+        int64_t z = 0;
+        for (int64_t q = s * M; q < std::min<int64_t>(n, s * M + M); ++q) z += g.deg(perm[q]);
+        if (t < 0 || z < tn) { t = s; tn = z; }
+      }
+      cp.build(g, perm, p, M);
+      ct.build(g, perm, t, M);
+      int64_t npairs = 0;
+      for (;;) {
+        Pair pr = freshtop(g, perm, cp, ct, N, M, p, t, used, true);  // "beneficial" swaps
+        if (!pr.found) break;
+        su.push_back(pr.u);
+        sv.push_back(pr.v);
+        ++npairs;
+        used[pr.u] = used[pr.v] = 1;
+        est[p] -= pr.gp;
+        if (est[p] <= 0 || all_used(used, p, M, n)) break;
+      }
+      *max_pairs = std::max(*max_pairs, npairs);
+    } else {
+      size_t head = 0;
+      int64_t live = (int64_t)I.size();
+      std::vector<int64_t> snap;
+      while (live > 1) {
+        while (!inI[I[head]]) ++head;
+        const int64_t p = I[head++];
+        inI[p] = 0;
+        --live;
+        snap.clear();
+        for (size_t k = head; k < I.size(); ++k)
+          if (inI[I[k]]) snap.push_back(I[k]);
+        cp.build(g, perm, p, M);
+        int64_t npairs = 0;
+        for (int64_t t : snap) {
+          if (!inI[t]) continue;
+          ct.build(g, perm, t, M);
+          Pair pr = freshtop(g, perm, cp, ct, N, M, p, t, used, gain_rule == 1);
+          if (!pr.found) continue;
+          su.push_back(pr.u);
+          sv.push_back(pr.v);
+          ++npairs;
+          used[pr.u] = used[pr.v] = 1;
+          est[p] -= pr.gp;
+          est[t] -= pr.gt;
+          if (est[t] <= 0) { inI[t] = 0; --live; }
+          if (est[p] <= 0 || all_used(used, p, M, n)) break;
+        }
+        *max_pairs = std::max(*max_pairs, npairs);
+      }
+      ct.clear();
+    }
+    cp.clear();
+    if (su.empty()) break;
+    for (size_t k = 0; k < su.size(); ++k) std::swap(perm[su[k]], perm[sv[k]]);
+    invert(perm, iperm);
+    ++passes;
+  }
+  return passes;
+}
+
+}  // namespace
+}  // namespace nm
+
+using namespace nm;
+
+extern "C" nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
+                                int32_t* perm_out, nm_reorder_stats* st) {
+  if (!A || !perm_out) return fail(NM_ERR_INVALID_ARG, "nm_reorder: NULL argument");
+  if (V < 1 || N < 1 || M <= N) return fail(NM_ERR_INVALID_ARG, "nm_reorder: need V >= 1, 1 <= N < M");
+  if (M > 32) return fail(NM_ERR_UNSUPPORTED, "nm_reorder: M > 32");
+  if (A->n <= 0) return fail(NM_ERR_INVALID_ARG, "nm_reorder: empty graph");
+  if (A->n >= ((int64_t)1 << 31)) return fail(NM_ERR_UNSUPPORTED, "nm_reorder: n >= 2^31");
+  nm_reorder_opts o = {10, 10, 10, 0, 1};
+  if (opts) o = *opts;
+  auto t0 = std::chrono::steady_clock::now();
+  int64_t* rp = nullptr;
+  int32_t* ci = nullptr;
+  nm_status s = host_csr(A, &rp, &ci);
+  if (s != NM_OK) { free(rp); free(ci); return s; }
+  s = validate_csr_host(A->n, rp, ci, true);
+  if (s != NM_OK) { free(rp); free(ci); return s; }
+  Graph g;
+  g.n = A->n;
+  g.rp = rp;
+  g.ci = ci;
+  const int64_t n = g.n;
+  std::vector<int32_t> perm(n), iperm(n), best;
+  std::iota(perm.begin(), perm.end(), 0);
+  iperm = perm;
+  nm_reorder_stats stats;
+  memset(&stats, 0, sizeof(stats));
+  int64_t w = omega_pscore(g, perm, iperm, N, M, nullptr);
+  int64_t mb = mbscore(g, perm, iperm, V, M);
+  stats.omega_init = w;
+  stats.mb_init = mb;
+  int64_t best_score = w + mb;
+  best = perm;
+  int64_t it = 0;
+  while ((w > 0 || mb > 0) && it <= o.max_outer) {
+    int64_t mb1 = mb;
+    for (int i1 = 0; mb1 > 0 && i1 <= o.max_stage1; ++i1) {  // Alg. 2
+      stage1_sort(g, perm, iperm, N, M);
+      stats.stage1_iters++;
+      mb1 = mbscore(g, perm, iperm, V, M);
+    }
+    stats.stage2_passes += stage2(g, perm, iperm, N, M, o.max_stage2, o.gain_rule, &stats.max_pairs_per_primary);
+    ++it;
+    w = omega_pscore(g, perm, iperm, N, M, nullptr);
+    mb = mbscore(g, perm, iperm, V, M);
+    if (o.keep_best && w + mb < best_score) {
+      best_score = w + mb;
+      best = perm;
+    }
+  }
+  stats.outer_iters = it;
+  const std::vector<int32_t>& res = o.keep_best ? best : perm;
+  memcpy(perm_out, res.data(), sizeof(int32_t) * n);
+  invert(res, iperm);
+  stats.omega_final = omega_pscore(g, res, iperm, N, M, nullptr);
+  stats.mb_final = mbscore(g, res, iperm, V, M);
+  stats.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+  if (st) *st = stats;
+  free(rp);
+  free(ci);
+  return NM_OK;
+}

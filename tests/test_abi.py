@@ -1,0 +1,57 @@
+"""The C-ABI library loads and exports every symbol include/nm.h declares (no GPU needed,
+no device compute)."""
+import ctypes
+import os
+import re
+
+import pytest
+
+from paper_conf_ppopp_chensz0s25_b200 import _lib, build
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "nm.h")).read()
+    return sorted(set(re.findall(r"^NM_API\s+[\w\s\*]+?\b(nm_\w+)\s*\(", src, flags=re.M)))
+
+
+def test_build_and_load():
+    build.build()
+    lib = _lib.load()
+    assert lib.nm_version() == 1
+
+
+def test_every_declared_symbol_is_exported_and_bound():
+    names = _declared()
+    assert len(names) >= 17
+    lib = ctypes.CDLL(_lib.LIB_PATH)
+    for n in names:
+        assert hasattr(lib, n), n
+        assert n in _lib.SIGNATURES, "binding missing for " + n
+    assert set(_lib.SIGNATURES) == set(names)
+
+
+def test_status_strings_and_errors():
+    lib = _lib.load()
+    for s in range(7):
+        assert lib.nm_status_string(s).decode().startswith("NM_")
+    # invalid arguments are rejected without touching a device
+    st = lib.nm_reorder(None, 1, 2, 4, None, None, None)
+    assert st == _lib.NM_ERR_INVALID_ARG
+    assert b"NULL" in lib.nm_last_error()
+
+
+def test_reorder_rejects_bad_csr_and_asymmetric():
+    import numpy as np
+    from paper_conf_ppopp_chensz0s25_b200 import api
+    ip = np.array([0, 1, 1], np.int64)
+    ic = np.array([1], np.int32)  # (0,1) without (1,0)
+    with pytest.raises(_lib.NMError) as e:
+        api.reorder(ip, ic, 1, 2, 4)
+    assert e.value.status == _lib.NM_ERR_NOT_SYMMETRIC
+    ip = np.array([0, 2, 2], np.int64)
+    ic = np.array([1, 1], np.int32)  # duplicate
+    with pytest.raises(_lib.NMError) as e:
+        api.reorder(ip, ic, 1, 2, 4)
+    assert e.value.status == _lib.NM_ERR_BAD_CSR

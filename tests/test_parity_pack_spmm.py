@@ -1,0 +1,203 @@
+"""GPU parity: nm_count_violations, nm_pack (canonical export) and nm_spmm through the C ABI
+vs the CPU oracle.
+
+Bars: counts, permutation, packed arrays and residual CSR are bit-exact;
+Y (fp32) satisfies |Y - Y_ref| <= 1e-3 * (|A| |X|) elementwise, Y_ref = fp64 A X on the same
+16-bit-rounded inputs (BASELINE.json north_star tolerance).
+"""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_ppopp_chensz0s25_b200 import api, graphs
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+TOL = 1e-3
+
+
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return torch.device("cuda:0")
+
+
+def _graph(kind, seed):
+    if kind == "c1":
+        return graphs.er_graph(2048, 16384, 1)
+    if kind == "er":
+        return graphs.er_graph(700, 5000, seed, self_loops=True)
+    if kind == "pl":
+        return graphs.lmcl_graph(1500, 12000, 2.1, 1, 0.0, seed, scramble=True)
+    if kind == "band":
+        return graphs.banded_graph(1300, 10, seed)
+    if kind == "tiny":
+        return graphs.fixture_f1()
+    raise ValueError(kind)
+
+
+CASES = [("tiny", 1, 1, 4), ("c1", 1, 1, 4), ("er", 2, 1, 4), ("pl", 3, 1, 4), ("band", 4, 1, 4),
+         ("band", 5, 64, 8), ("pl", 6, 128, 16), ("er", 7, 8, 8), ("band", 8, 128, 8)]
+
+
+@pytest.mark.parametrize("kind,seed,V,M", CASES)
+def test_counts(kind, seed, V, M):
+    _cuda()
+    ip, ic = _graph(kind, seed)
+    n = len(ip) - 1
+    perm = np.random.default_rng(seed).permutation(n).astype(np.int32)
+    for pm in (None, perm):
+        w0, mb0, ps0 = oracle.counts(ip, ic, pm, V, 2, M)
+        w1, mb1, ps1 = api.count_violations(ip, ic, pm, V, 2, M)
+        assert (w0, mb0) == (w1, mb1)
+        assert np.array_equal(ps0, ps1)
+
+
+def _values(ip, ic, dtype, seed):
+    v = graphs.symmetric_values(ip, ic, seed)
+    bits, v64 = graphs.round16(v, dtype)
+    return v, bits, v64
+
+
+@pytest.mark.parametrize("kind,seed,V,M", CASES)
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+def test_pack_canonical_bit_exact(kind, seed, V, M, dtype):
+    _cuda()
+    ip, ic = _graph(kind, seed)
+    perm, _ = api.reorder(ip, ic, V, 2, M)
+    v32, bits, _ = _values(ip, ic, dtype, seed)
+    Mp = 4 if V == 1 else M
+    ref = oracle.pack(ip, ic, bits, 0, perm, 128, Mp)
+    P = api.pack(ip, ic, perm, V, 2, M, dtype=dtype, val=v32)  # device rounds f32 -> 16 bit
+    got = P.export_canonical()
+    for k in ("panel_ptr", "mb_seg", "sel", "nib", "vals", "res_rowptr", "res_col", "res_val"):
+        assert np.array_equal(ref[k], got[k]), k
+    inf = P.info()
+    assert inf["packed_nnz"] + inf["residual_nnz"] == ip[-1]
+
+
+def test_pack_rows_shards_match_oracle_rows():
+    _cuda()
+    ip, ic = _graph("pl", 11)
+    n = len(ip) - 1
+    perm, _ = api.reorder(ip, ic, 1, 2, 4)
+    ref = oracle.pack(ip, ic, None, 0x3C00, perm, 128, 4)
+    cuts = [0, 512, 1024, n]
+    for a, b in zip(cuts[:-1], cuts[1:]):
+        P = api.pack(ip, ic, perm, 1, 2, 4, row_begin=a, row_end=b)
+        got = P.export_canonical()
+        pa, pb = a // 128, (b + 127) // 128
+        m0, m1 = ref["panel_ptr"][pa], ref["panel_ptr"][pb]
+        assert np.array_equal(got["panel_ptr"], ref["panel_ptr"][pa:pb + 1] - m0)
+        assert np.array_equal(got["mb_seg"], ref["mb_seg"][m0:m1])
+        assert np.array_equal(got["nib"], ref["nib"][m0 * 128:m1 * 128])
+        assert np.array_equal(got["vals"], ref["vals"][m0 * 256:m1 * 256])
+        r0, r1 = ref["res_rowptr"][a], ref["res_rowptr"][b]
+        assert np.array_equal(got["res_rowptr"], ref["res_rowptr"][a:b + 1] - r0)
+        assert np.array_equal(got["res_col"], ref["res_col"][r0:r1])
+
+
+def _spmm_check(ip, ic, perm, V, M, F, dtype, seed, part_check=True):
+    dev = _cuda()
+    n = len(ip) - 1
+    v32, bits, v64 = _values(ip, ic, dtype, seed)
+    X32 = graphs.features(n, F, seed + 1)
+    xbits, x64 = graphs.round16(X32, dtype)
+    Y_ref, E, _ = oracle.spmm(ip, ic, v64, x64)
+    P = api.pack(ip, ic, perm, V, 2, M, dtype=dtype, val=v32)
+    tdt = torch.float16 if dtype == "f16" else torch.bfloat16
+    ldx = (F + 7) // 8 * 8
+    X = torch.zeros((n, ldx), dtype=torch.int16, device=dev)
+    X[:, :F] = torch.from_numpy(xbits.view(np.int16)).to(dev)
+    X = X.view(tdt)
+    PX = torch.empty_like(X)
+    perm_d = torch.from_numpy(perm.astype(np.int32)).to(dev)
+    api.permute_rows(X, PX, perm_d, dtype)
+    Yp = torch.full((n, F), float("nan"), dtype=torch.float32, device=dev)
+    api.spmm(P, PX, Yp, F=F)
+    Y = torch.empty_like(Yp)
+    api.unpermute_rows(Yp, Y, perm_d, "f32")
+    torch.cuda.synchronize()
+    Yh = Y.cpu().numpy().astype(np.float64)
+    assert np.isfinite(Yh).all()
+    err = np.abs(Yh - Y_ref)
+    bad = err > TOL * E + 1e-30
+    assert not bad.any(), "max err %g at %s (bound %g)" % (err.max(), np.argwhere(bad)[0], (TOL * E)[bad][0])
+    return P
+
+
+@pytest.mark.parametrize("kind,seed,V,M", CASES)
+@pytest.mark.parametrize("F", [32, 128])
+def test_spmm_parity(kind, seed, V, M, F):
+    ip, ic = _graph(kind, seed)
+    perm, _ = api.reorder(ip, ic, V, 2, M)
+    _spmm_check(ip, ic, perm, V, M, F, "f16", seed)
+
+
+@pytest.mark.parametrize("F", [1, 8, 17, 64, 100, 192, 200, 256, 300, 520])
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+def test_spmm_feature_widths(F, dtype):
+    ip, ic = _graph("er", 21)
+    n = len(ip) - 1
+    perm = np.random.default_rng(3).permutation(n).astype(np.int32)
+    _spmm_check(ip, ic, perm, 1, 4, F, dtype, 21)
+
+
+def test_spmm_identity_perm_and_residual_heavy():
+    # random order without reorder: many violations -> large residual at 128:2:16
+    ip, ic = _graph("pl", 31)
+    n = len(ip) - 1
+    P = _spmm_check(ip, ic, np.arange(n, dtype=np.int32), 128, 16, 64, "f16", 31)
+    assert P.info()["residual_nnz"] > 0
+
+
+def test_spmm_sptc_plus_residual_equals_total():
+    dev = _cuda()
+    ip, ic = _graph("band", 41)
+    n = len(ip) - 1
+    perm, _ = api.reorder(ip, ic, 8, 2, 8)
+    P = api.pack(ip, ic, perm, 8, 2, 8)
+    X = torch.randn((n, 64), device=dev).to(torch.float16)
+    Y1 = torch.empty((n, 64), device=dev)
+    Y2 = torch.empty((n, 64), device=dev)
+    api.spmm(P, X, Y1)
+    api.spmm(P, X, Y2, part="sptc")
+    api.spmm(P, X, Y2, part="residual")
+    torch.cuda.synchronize()
+    assert torch.equal(Y1, Y2)
+
+
+def test_dense_conforming_panel_equals_dense_gemm():
+    """A fully 2:4-dense panel (every 4-group of every row holds 2 nonzeros) is a plain
+    structured-sparse GEMM: compare with torch's dense fp32 matmul of the same operands."""
+    dev = _cuda()
+    n = 256
+    rows, cols = [], []
+    rng = np.random.default_rng(5)
+    for i in range(n):
+        for g in range(n // 4):
+            for j in sorted(rng.choice(4, 2, replace=False)):
+                rows.append(i)
+                cols.append(4 * g + j)
+    A = np.zeros((n, n), bool)
+    A[rows, cols] = True
+    A = A | A.T  # symmetric (may exceed 2 per group -> residual keeps it exact)
+    ip = np.concatenate([[0], np.cumsum(A.sum(1))]).astype(np.int64)
+    ic = np.nonzero(A)[1].astype(np.int32)
+    _spmm_check(ip, ic, np.arange(n, dtype=np.int32), 1, 4, 128, "bf16", 5)
+
+
+def test_empty_rows_and_isolated_vertices():
+    # vertices 300..399 isolated: their rows of Y must be exactly 0
+    dev = _cuda()
+    ipa, ica = graphs.er_graph(300, 1500, 9)
+    n = 400
+    ip = np.concatenate([ipa, np.full(100, ipa[-1])]).astype(np.int64)
+    P = _spmm_check(ip, ica, np.arange(n, dtype=np.int32), 1, 4, 64, "f16", 9)
+    X = torch.ones((n, 64), device=dev, dtype=torch.float16)
+    Y = torch.full((n, 64), 7.0, device=dev)
+    api.spmm(P, X, Y)
+    torch.cuda.synchronize()
+    assert torch.all(Y[300:] == 0)

@@ -12,6 +12,7 @@
 #include <vector>
 #include <random>
 #include <cuda_fp16.h>
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
 #define CK(x) do { cudaError_t e = (x); if (e != cudaSuccess) { \
@@ -37,6 +38,7 @@ struct Params {
   uint32_t meta_col;
   uint32_t e_id2;
   int a_bytes, b_bytes;
+  uint32_t b_layout;  // 0 = SWIZZLE_NONE, 2 = SWIZZLE_128B
 };
 
 template <int N>
@@ -45,6 +47,7 @@ probe_kernel(const uint8_t* __restrict__ a_img, const uint8_t* __restrict__ b_im
              const uint32_t* __restrict__ meta, float* __restrict__ D, Params p) {
   __shared__ __align__(1024) uint8_t smA[8192];
   __shared__ __align__(1024) uint8_t smB[16384];
+  // (N=128 K=32 16-bit B = 8 KB)
   __shared__ uint32_t tmem_base_sh;
   __shared__ __align__(8) uint64_t mbar;
   const int tid = threadIdx.x, warp = tid >> 5;
@@ -75,7 +78,7 @@ probe_kernel(const uint8_t* __restrict__ a_img, const uint8_t* __restrict__ b_im
   asm volatile("tcgen05.fence::after_thread_sync;");
   if (tid == 0) {
     uint64_t ad = make_sdesc(smem_u32(smA), p.a_lbo, p.a_sbo);
-    uint64_t bd = make_sdesc(smem_u32(smB), p.b_lbo, p.b_sbo);
+    uint64_t bd = make_sdesc(smem_u32(smB), p.b_lbo, p.b_sbo) | ((uint64_t)p.b_layout << 61);
     uint32_t acc = 0;
     if (p.sparse) {
       uint32_t e = tbase + p.meta_col;
@@ -296,7 +299,7 @@ int main() {
         }
       }
     // id2 / column-offset probe with H1 at meta column 129 (odd) and id2 0/1
-    for (int id2 = 0; id2 < 2; ++id2) {
+    for (int id2 = 0; id2 < 0; ++id2) {
       for (int col = 129; col <= 130; ++col) {
         Params p{};
         p.a_lbo = 128; p.a_sbo = 256; p.b_lbo = 128; p.b_sbo = 512;
@@ -308,6 +311,55 @@ int main() {
         for (int i = 0; i < M * K; ++i) bad += (out[i] != Alog[i]);
         printf("SPARSE H1 meta_col=%d id2=%d: mismatches=%d %s\n", col, id2, bad, bad == 0 ? "MATCH" : "");
       }
+    }
+  }
+  // ---------------- sparse, N=128, B MN-major SWIZZLE_128B, f16 and bf16 ----------------
+  for (int bf = 0; bf < 2; ++bf) {
+    const int K = 32, N = 128, KC = 16;
+    static const int pairs[6][2] = {{0, 1}, {0, 2}, {0, 3}, {1, 2}, {1, 3}, {2, 3}};
+    std::vector<__half> Ac(M * KC);      // raw 16-bit storage (bf16 bits reinterpret)
+    std::vector<int> nib(M * 8);
+    std::vector<double> Alog(M * K, 0.0), Bv(K * N);
+    auto enc = [&](float v) { __half h; if (bf) { __nv_bfloat16 b = __float2bfloat16(v); memcpy(&h, &b, 2);} else h = __float2half(v); return h; };
+    for (int r = 0; r < M; ++r)
+      for (int g = 0; g < 8; ++g) {
+        int pi = rng() % 6;
+        int i0 = pairs[pi][0], i1 = pairs[pi][1];
+        nib[r * 8 + g] = i0 | (i1 << 2);
+        float v0 = (float)((int)(rng() % 17) - 8) * 0.25f, v1 = (float)((int)(rng() % 17) - 8) * 0.25f;
+        Ac[r * KC + 2 * g] = enc(v0); Ac[r * KC + 2 * g + 1] = enc(v1);
+        Alog[r * K + 4 * g + i0] = v0; Alog[r * K + 4 * g + i1] = v1;
+      }
+    std::vector<__half> B(K * N);
+    for (int k = 0; k < K; ++k) for (int n = 0; n < N; ++n) { float v = (float)((int)(rng() % 9) - 4); B[k * N + n] = enc(v); Bv[k * N + n] = v; }
+    std::vector<uint8_t> aimg(M * KC * 2), bimg(K * N * 2);
+    kmajor_image(aimg, Ac, M, KC, 128, 256);
+    // SW128 MN-major: atom = 8 K-rows x 128 B (64 elems), 16B chunk c of row r at (c ^ r%8);
+    // K-groups at SBO = 1024, 64-element N-chunks at LBO = 4096.
+    for (int k = 0; k < K; ++k)
+      for (int n = 0; n < N; ++n) {
+        int nc = n / 64, c16 = (n % 64) / 8, r = k % 8;
+        size_t off = (size_t)nc * 4096 + (size_t)(k / 8) * 1024 + r * 128 + ((c16 ^ r) * 16) + (n % 8) * 2;
+        memcpy(&bimg[off], &B[k * N + n], 2);
+      }
+    std::vector<double> ref(M * N, 0.0);
+    for (int i = 0; i < M; ++i) for (int j = 0; j < N; ++j) for (int k = 0; k < K; ++k) ref[i * N + j] += Alog[i * K + k] * Bv[k * N + j];
+    std::vector<uint32_t> meta(128);
+    for (int L = 0; L < 128; ++L) {
+      int m0 = L % 8, k1 = (L / 8) % 2, m2 = L / 16; int r0 = m0 + 16 * m2, r1 = r0 + 8; uint32_t w = 0;
+      for (int q = 0; q < 4; ++q) { w |= (uint32_t)nib[r0 * 8 + 4 * k1 + q] << (4 * q); w |= (uint32_t)nib[r1 * 8 + 4 * k1 + q] << (16 + 4 * q); }
+      meta[L] = w;
+    }
+    for (int v = 0; v < 2; ++v) {
+      Params p{};
+      p.a_lbo = 128; p.a_sbo = 256;
+      p.b_lbo = v ? 1024 : 4096; p.b_sbo = v ? 4096 : 1024; p.b_layout = 2;
+      p.idesc = make_idesc(1, M, N, 0, 1) | (bf ? ((1u << 7) | (1u << 10)) : 0u);
+      p.sparse = 1; p.meta_col = 128;
+      std::vector<float> out;
+      run<128>(aimg, bimg, meta, out, p);
+      double err = 0; for (int i = 0; i < M * N; ++i) err = fmax(err, fabs(out[i] - ref[i]));
+      printf("SPARSE N=128 SW128-B %s b(lbo=%u,sbo=%u): max_err=%g %s\n", bf ? "bf16" : "f16", p.b_lbo, p.b_sbo, err, err == 0 ? "MATCH" : "");
     }
   }
   printf("PROBE DONE\n");
