@@ -1,0 +1,415 @@
+#!/usr/bin/env python
+"""bench.py -- V:N:M SpMM on B200 sparse tensor cores (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NAME] [--impl ours|reference]
+
+One step = one pass of the hot path over the workload: the X-row permutation, the
+tcgen05.mma.sp SpMM, the residual CSR SpMM and the Y-row unpermutation (SURVEY §8(a)
+a5-a8), with the permutations folded into the SpMM's gather/scatter indices
+(NM_PACK_ORIGINAL_ORDER): Y = A X in the original vertex order.  Reordering (a1-a2) and
+packing (a4) are offline preprocessing -- run and reported, not timed.
+
+Multi-GPU (torchrun, N > 1): the rows of B = P A P^T are split into contiguous,
+panel-aligned blocks, one per rank, X replicated; the SpMM needs no exchange
+(the GCN driver in paper_conf_ppopp_chensz0s25_b200/dist.py all-gathers).  Total work is
+fixed: "scaling": "strong".  Time = max over ranks of the device-timed region.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    # configs[1] (SuiteSparse-shaped sweep) headline point: banded n = 2^20, avg degree 16
+    "c2-banded-n1m-d16-f128-1:2:4": dict(kind="band", n=1 << 20, d=16, F=128, V=1, M=4, dtype="f16"),
+    "c2-banded-n1m-d32-f128-1:2:4": dict(kind="band", n=1 << 20, d=32, F=128, V=1, M=4, dtype="f16"),
+    "c2-banded-n262k-d16-f128-64:2:8": dict(kind="band", n=1 << 18, d=16, F=128, V=64, M=8, dtype="f16"),
+    "c2-powerlaw-n262k-d16-f128-1:2:4": dict(kind="pl", n=1 << 18, d=16, F=128, V=1, M=4, dtype="f16"),
+    "c2-powerlaw-n262k-d16-f128-128:2:16": dict(kind="pl", n=1 << 18, d=16, F=128, V=128, M=16, dtype="f16"),
+    # configs[0]: ER n = 2048, m = 16384, F = 32, 2:4, fp16 (oracle-sized correctness case)
+    "c1-er-n2048-f32-1:2:4": dict(kind="er", n=2048, m=16384, F=32, V=1, M=4, dtype="f16"),
+}
+DEFAULT = "c2-banded-n1m-d16-f128-1:2:4"
+METRIC = "V:N:M SpMM GFLOP/s & % sparse-MMA/HBM roofline vs cuSPARSE, 1/2/4/8 B200"
+
+
+def make_graph(w):
+    from paper_conf_ppopp_chensz0s25_b200 import graphs
+    if w["kind"] == "band":
+        seed = graphs.seed_of("banded", w["n"], w["d"])
+        ip, ic = graphs.banded_graph(w["n"], w["d"], seed)
+    elif w["kind"] == "pl":
+        seed = graphs.seed_of("powerlaw", w["n"], w["d"])
+        ip, ic = graphs.lmcl_graph(w["n"], w["n"] * w["d"] // 2, 2.1, 1, 0.0, seed, scramble=True)
+    elif w["kind"] == "er":
+        seed = 1
+        ip, ic = graphs.er_graph(w["n"], w["m"], seed)
+    else:
+        raise ValueError(w["kind"])
+    vals = graphs.symmetric_values(ip, ic, seed + 1)
+    X32 = graphs.features(w["n"], w["F"], seed + 2)
+    return ip, ic, vals, X32
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d.get("hbm_gbs", 6650.0), d.get("bf16_tflops", 1590.0), "measured"
+    return 6650.0, 1590.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle sampling during the timed region (B200_PROFILING.md)."""
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + q,
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cpu_oracle_sample(ip, ic, vals, X32, dtype, budget_s=12.0):
+    """The oracle (fp64 CSR SpMM, all host cores) on a bounded row sample of the workload."""
+    import oracle
+    from paper_conf_ppopp_chensz0s25_b200 import graphs
+    n = len(ip) - 1
+    _, v64 = graphs.round16(vals, dtype)
+    _, x64 = graphs.round16(X32, dtype)
+    cores = len(os.sched_getaffinity(0))
+    # calibrate on 1/256 of the rows, then scale the sample to ~budget_s
+    rows = max(1, n // 256)
+    t0 = time.perf_counter()
+    oracle.spmm(ip[:rows + 1], ic[:ip[rows]], v64[:ip[rows]], x64, nthreads=cores)
+    dt = max(time.perf_counter() - t0, 1e-4)
+    rows = int(min(n, max(rows, rows * budget_s / dt)))
+    t0 = time.perf_counter()
+    _, _, used = oracle.spmm(ip[:rows + 1], ic[:ip[rows]], v64[:ip[rows]], x64, nthreads=cores)
+    dt = time.perf_counter() - t0
+    F = X32.shape[1]
+    gflops = 2.0 * float(ip[rows]) * F / dt / 1e9
+    return {"value": gflops, "unit": "GFLOP/s", "cores": used, "kind": "oracle",
+            "sample": "fp64 CSR SpMM over the first %d of %d rows (%d nnz), F=%d, %.1f s" %
+                      (rows, n, int(ip[rows]), F, dt)}
+
+
+def run_reference(args, w):
+    """--impl reference: the oracle as it stands, timed on the host cores (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    ip, ic, vals, X32 = make_graph(w)
+    budget = max(1.0, 120.0 / max(1, args.steps + args.warmup))
+    for _ in range(args.warmup):
+        cpu_oracle_sample(ip, ic, vals, X32, w["dtype"], budget_s=min(budget, 3.0))
+    samples = [cpu_oracle_sample(ip, ic, vals, X32, w["dtype"], budget_s=budget) for _ in range(args.steps)]
+    val = statistics.median(s["value"] for s in samples)
+    F = w["F"]
+    nnz = int(ip[-1])
+    step_ms = 2.0 * nnz * F / (val * 1e9) * 1e3
+    line = {"metric": METRIC, "value": val, "unit": "GFLOP/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": step_ms, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": args.workload, "n": w["n"], "nnz": nnz, "F": F,
+                       "pattern": "%d:2:%d" % (w["V"], w["M"]), "parallelism": "cpu"},
+            "cpu_baseline": dict(samples[-1], value=val),
+            "e2e": {"value": val, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--workload", default=DEFAULT, choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cusparse", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--order", default="original", choices=["original", "permuted"])
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    w = WORKLOADS[args.workload]
+    if args.impl == "reference":
+        return run_reference(args, w)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ppopp_chensz0s25_b200 import api, graphs
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    # ---------------- inputs (seeded, synthetic) and offline preprocessing ----------------
+    t0 = time.perf_counter()
+    ip, ic, vals, X32 = make_graph(w)
+    gen_s = time.perf_counter() - t0
+    n, F, V, M, dt = w["n"], w["F"], w["V"], w["M"], w["dtype"]
+    nnz = int(ip[-1])
+    perm, rst = api.reorder(ip, ic, V, 2, M)
+    from paper_conf_ppopp_chensz0s25_b200.dist import shard_rows
+    rb, re = shard_rows(n, world, rank)
+    t0 = time.perf_counter()
+    P = api.pack(ip, ic, perm, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order=args.order)
+    torch.cuda.synchronize()
+    pack_s = time.perf_counter() - t0
+    info = P.info()
+    xbits, _ = graphs.round16(X32, dt)
+    tdt = torch.float16 if dt == "f16" else torch.bfloat16
+    X = torch.from_numpy(xbits.view(np.int16)).to(dev).view(tdt)
+    Y = torch.empty((n, F), dtype=torch.float32, device=dev)
+    perm_d = torch.from_numpy(perm).to(dev)
+    PX = torch.empty_like(X) if args.order == "permuted" else None
+    Yp = torch.empty((re - rb, F), dtype=torch.float32, device=dev) if args.order == "permuted" else None
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+    stream = torch.cuda.current_stream()
+    has_res = info["residual_nnz"] > 0
+
+    def step(ev=None):
+        if args.order == "original":
+            if ev: ev[0].record(stream)
+            api.spmm(P, X, Y, part="sptc")
+            if ev: ev[1].record(stream)
+            if has_res:
+                api.spmm(P, X, Y, part="residual")
+            if ev: ev[2].record(stream)
+        else:
+            if ev: ev[0].record(stream)
+            api.permute_rows(X, PX, perm_d, dt)
+            api.spmm(P, PX, Yp, part="sptc")
+            if ev: ev[1].record(stream)
+            if has_res:
+                api.spmm(P, PX, Yp, part="residual")
+            api.unpermute_rows(Yp, Y, perm_d[rb:re], "f32")
+            if ev: ev[2].record(stream)
+
+    launches_per_step = 1 + int(has_res) + (2 if args.order == "permuted" else 0)
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    # ---------------- timed region (device events; L2 flushed between steps) ----------------
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for k in range(args.steps):
+            flush.zero_()
+            step(evs[k])
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    step_ms = [e[0].elapsed_time(e[2]) for e in evs]
+    sptc_ms = [e[0].elapsed_time(e[1]) for e in evs]
+    total_ms = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(total_ms, op=dist.ReduceOp.MAX)
+    total_ms = float(total_ms.item())
+    ms_per_step = total_ms / args.steps
+    useful_flop = 2.0 * nnz * F  # all ranks together (strong scaling: fixed total work)
+    value = useful_flop / (ms_per_step * 1e-3) / 1e9
+
+    # ---------------- roofline of the dominant kernel (k_spmm_sptc, this rank) ----------------
+    hbm_gbs, bf16_tf, peak_src = peaks()
+    chunks = info["n_chunks"]
+    # algorithmic bytes per launch: packed image (4608 B/chunk) + gather indices (128 B/chunk)
+    # + X read once (rows of X the shard touches, F*2 B) + Y written once (rows*F*4 B)
+    rows_b = re - rb
+    x_rows = n if world == 1 else n  # X replicated; a shard touches (almost) all rows on these graphs
+    alg_bytes = chunks * (4608 + 128) + x_rows * F * 2 + rows_b * F * 4
+    k_ms = statistics.mean(sptc_ms)
+    achieved = alg_bytes / (k_ms * 1e-3) / 1e9
+    t_mma_ms = 2.0 * chunks * 128 * max(F, 64) * 32 / (2 * bf16_tf * 1e12) * 1e3  # sparse = 2x dense rate
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_gbs, "unit": "GB/s",
+                "frac": achieved / hbm_gbs, "traffic": None, "peak_source": peak_src,
+                "kernel": "k_spmm_sptc", "kernel_ms": k_ms, "alg_bytes_per_launch": alg_bytes,
+                "t_hbm_ms": alg_bytes / (hbm_gbs * 1e9) * 1e3, "t_mma_ms": t_mma_ms}
+    prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(prof):
+        try:
+            tr = json.load(open(prof)).get(args.workload)
+            if tr:
+                roofline["traffic"] = tr["dram_bytes_per_launch"]
+                roofline["traffic_source"] = "profiles/ncu_traffic.json (%s)" % tr.get("round", "")
+        except Exception:
+            pass
+
+    # ---------------- end-to-end through the public API with host buffers ----------------
+    e2e = None
+    if world == 1:
+        Xh = torch.empty(X.shape, dtype=tdt).pin_memory()
+        Xh.copy_(X.cpu())
+        Yh = torch.empty((n, F), dtype=torch.float32).pin_memory()
+        for _ in range(2):
+            X.copy_(Xh, non_blocking=True)
+            step()
+            Yh.copy_(Y, non_blocking=True)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ks = max(3, args.steps // 2)
+        e0.record(stream)
+        for _ in range(ks):
+            X.copy_(Xh, non_blocking=True)
+            step()
+            Yh.copy_(Y, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        e2e_ms = e0.elapsed_time(e1) / ks
+        e2e = {"value": useful_flop / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s", "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": int(Xh.numel() * Xh.element_size()),
+               "d2h_bytes_per_step": int(Yh.numel() * Yh.element_size())}
+
+    # ---------------- cuSPARSE on the same box (original order, same rounded inputs) ----------
+    cus = None
+    if not args.no_cusparse and world == 1:
+        try:
+            cus = cusparse_baseline(ip, ic, vals, X, dt, F, dev, args.steps, flush)
+        except Exception as ex:  # report, never fake
+            cus = {"error": str(ex)[:200]}
+
+    # ---------------- CPU oracle baseline (rank 0, N = 1) ----------------
+    cpu = None
+    if world == 1 and not args.no_cpu:
+        cpu = cpu_oracle_sample(ip, ic, vals, X32, dt)
+
+    clocks = clk.summary()
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": dt, "data": "synthetic",
+                "config": {"workload": args.workload, "graph": w["kind"], "n": n, "nnz": nnz, "F": F,
+                           "pattern": "%d:2:%d" % (V, M), "order": args.order,
+                           "parallelism": "row-shard x%d" % world,
+                           "l2": "flushed between steps (256 MiB write outside the event-timed intervals)"},
+                "gpu_launches": launches_per_step * args.steps,
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "cusparse": cus,
+                "preprocess": {"gen_s": gen_s, "reorder_s": rst["seconds"], "pack_s": pack_s,
+                               "omega_init": rst["omega_init"], "omega_final": rst["omega_final"],
+                               "mb_init": rst["mb_init"], "mb_final": rst["mb_final"],
+                               "violation_removal": (None if rst["omega_init"] == 0 else
+                                                     1.0 - rst["omega_final"] / rst["omega_init"]),
+                               "n_mb": info["n_mb"], "n_chunks": chunks,
+                               "slots_per_nnz": chunks * 8 * 128 * 2 / max(1, nnz),
+                               "residual_nnz": info["residual_nnz"],
+                               "packed_bytes": info["device_bytes"]},
+                "step_ms_median": statistics.median(step_ms), "sptc_ms_median": statistics.median(sptc_ms)}
+        if cus and "ms" in cus:
+            line["speedup_vs_cusparse"] = cus["ms"] / ms_per_step
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def cusparse_baseline(ip, ic, vals, X, dt, F, dev, steps, flush):
+    import ctypes
+
+    import torch
+    from paper_conf_ppopp_chensz0s25_b200 import build, graphs
+    lib = ctypes.CDLL(build.build_baseline())
+    lib.cs_create.restype = ctypes.c_int
+    n = len(ip) - 1
+    rp = torch.from_numpy(ip.astype(np.int32)).to(dev)
+    ci = torch.from_numpy(ic).to(dev)
+    vb, _ = graphs.round16(vals, dt)
+    va = torch.from_numpy(vb.view(np.int16)).to(dev)
+    Yc = torch.empty((n, F), dtype=torch.float32, device=dev)
+    res = {}
+    for name, alg in (("csr_alg2", 2), ("default", 0)):
+        h = ctypes.c_void_p()
+        yf = ctypes.c_int()
+        rc = lib.cs_create(ctypes.c_int64(n), ctypes.c_int64(len(ic)), ctypes.c_void_p(rp.data_ptr()),
+                           ctypes.c_void_p(ci.data_ptr()), ctypes.c_void_p(va.data_ptr()), int(dt == "bf16"),
+                           F, ctypes.c_void_p(X.data_ptr()), ctypes.c_int64(X.stride(0)),
+                           ctypes.c_void_p(Yc.data_ptr()), ctypes.c_int64(F), alg, ctypes.byref(h),
+                           ctypes.byref(yf))
+        if rc != 0:
+            res[name] = {"error": "cs_create rc=%d" % rc}
+            continue
+        s = ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+        for _ in range(3):
+            lib.cs_run(h, s)
+        ts = []
+        for _ in range(steps):
+            flush.zero_()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            rc = lib.cs_run(h, s)
+            b.record()
+            ts.append((a, b))
+        torch.cuda.synchronize()
+        ms = statistics.mean(a.elapsed_time(b) for a, b in ts)
+        res[name] = {"ms": ms, "gflops": 2.0 * len(ic) * F / (ms * 1e-3) / 1e9, "y_fp32": bool(yf.value),
+                     "rc": rc}
+        lib.cs_destroy(h)
+    best = min((v for v in res.values() if "ms" in v), key=lambda v: v["ms"], default=None)
+    if best:
+        res["ms"] = best["ms"]
+        res["gflops"] = best["gflops"]
+    res["note"] = "cusparseSpMM CSR, original vertex order, 16-bit A/X, fp32 compute"
+    return res
+
+
+if __name__ == "__main__":
+    main()

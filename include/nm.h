@@ -131,6 +131,21 @@ NM_API nm_status nm_pack_rows(const nm_csr* A, const int32_t* perm, int V, int N
                        nm_dtype dtype, int64_t row_begin, int64_t row_end, void* stream,
                        nm_packed** out);
 
+/* General form.  flags:
+ *   0                      -- operands in permuted order: nm_spmm reads PX = P X (n rows) and
+ *                             writes Yp rows 0..(row_end-row_begin) (rows of B).
+ *   NM_PACK_ORIGINAL_ORDER -- the permutation is folded into the operand indices: nm_spmm
+ *                             reads X in the ORIGINAL vertex order (gathering row perm[q] for
+ *                             column q of B) and writes Y in the original order, row
+ *                             perm[p] for each packed row p of B, into an n-row buffer.
+ *                             Y = A X for those rows without separate permute/unpermute
+ *                             passes (Fig. 1 caption L38 realised inside the SpMM).
+ * The canonical export is identical in both modes. */
+#define NM_PACK_ORIGINAL_ORDER 1
+NM_API nm_status nm_pack_ex(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
+                            nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags,
+                            void* stream, nm_packed** out);
+
 /* Sizes: #meta-blocks, #values kept in MMA slots, #residual nonzeros, device bytes held,
  * #K=32 chunks (8 meta-blocks each, padded per panel).  Any pointer may be NULL. */
 NM_API nm_status nm_packed_info(const nm_packed* P, int64_t* n_mb, int64_t* packed_nnz,

@@ -16,6 +16,7 @@ NM_OK, NM_ERR_INVALID_ARG, NM_ERR_UNSUPPORTED, NM_ERR_BAD_CSR, NM_ERR_NOT_SYMMET
     NM_ERR_CUDA, NM_ERR_OOM = range(7)
 NM_F16, NM_BF16, NM_F32 = 0, 1, 2
 NM_RELU = 1
+NM_PACK_ORIGINAL_ORDER = 1
 
 P64 = ctypes.POINTER(ctypes.c_int64)
 P32 = ctypes.POINTER(ctypes.c_int32)
@@ -55,6 +56,9 @@ SIGNATURES = {
     "nm_pack_rows": (ctypes.c_int, [ctypes.POINTER(nm_csr), P32, ctypes.c_int, ctypes.c_int,
                                     ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int64,
                                     ctypes.c_int64, VP, ctypes.POINTER(VP)]),
+    "nm_pack_ex": (ctypes.c_int, [ctypes.POINTER(nm_csr), P32, ctypes.c_int, ctypes.c_int,
+                                  ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int64,
+                                  ctypes.c_int64, ctypes.c_int, VP, ctypes.POINTER(VP)]),
     "nm_packed_info": (ctypes.c_int, [VP, P64, P64, P64, P64, P64]),
     "nm_export_canonical": (ctypes.c_int, [VP, P64, P32, PU8, PU8, PU16, P64, P32, PU16]),
     "nm_packed_free": (None, [VP]),

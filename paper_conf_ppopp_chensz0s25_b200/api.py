@@ -132,9 +132,10 @@ class Packed:
 
 
 def pack(indptr, indices, perm, V: int, N: int, M: int, dtype="f16", val=None, val_dtype=None,
-         row_begin=None, row_end=None, stream=None):
-    """nm_pack / nm_pack_rows of B = P A P^T.  val: values per CSR entry (numpy, dtype
-    val_dtype in {'f16','bf16' (uint16 bits),'f32'}) or None for a binary adjacency."""
+         row_begin=None, row_end=None, stream=None, order="permuted"):
+    """nm_pack / nm_pack_rows / nm_pack_ex of B = P A P^T.  val: values per CSR entry (numpy,
+    dtype val_dtype in {'f16','bf16' (uint16 bits),'f32'}) or None for a binary adjacency.
+    order='original' folds the permutation into the SpMM (NM_PACK_ORIGINAL_ORDER)."""
     if val is not None and val_dtype is None:
         val_dtype = "f32" if val.dtype == np.float32 else ("f16" if val.dtype == np.float16 else "bf16")
     c, keep = _csr_struct(indptr, indices, val, val_dtype or "f16")
@@ -142,6 +143,14 @@ def pack(indptr, indices, perm, V: int, N: int, M: int, dtype="f16", val=None, v
     h = ctypes.c_void_p()
     pp = None if pm is None else pm.ctypes.data_as(L.P32)
     sp = _stream_ptr(stream)
+    if order == "original":
+        rb = 0 if row_begin is None else int(row_begin)
+        re = c.n if row_end is None else int(row_end)
+        L.check(L.load().nm_pack_ex(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], rb, re,
+                                    L.NM_PACK_ORIGINAL_ORDER, sp, ctypes.byref(h)), "nm_pack_ex")
+        P = Packed(h, c.n, rb, re, dtype)
+        P.order = "original"
+        return P
     if row_begin is None:
         L.check(L.load().nm_pack(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], sp, ctypes.byref(h)),
                 "nm_pack")

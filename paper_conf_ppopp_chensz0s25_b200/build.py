@@ -63,5 +63,25 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+BASELINE_SRC = os.path.join(ROOT, "bench_support", "cusparse_shim.cu")
+BASELINE_LIB = os.path.join(ROOT, "bench_support", "libcusparse_shim.so")
+
+
+def build_baseline(force: bool = False) -> str:
+    """cuSPARSE comparison shim used by bench.py (baseline, not part of libnm)."""
+    if not force and os.path.exists(BASELINE_LIB) and \
+            os.path.getmtime(BASELINE_LIB) >= os.path.getmtime(BASELINE_SRC):
+        return BASELINE_LIB
+    tmp = BASELINE_LIB + ".tmp%d" % os.getpid()
+    cmd = [NVCC] + ARCH + ["-O3", "-std=c++17", "-Xcompiler", "-fPIC", "-shared", BASELINE_SRC,
+                           "-o", tmp, "-lcusparse"]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError("baseline shim build failed:\n%s" % r.stderr)
+    os.replace(tmp, BASELINE_LIB)
+    return BASELINE_LIB
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    print(build_baseline(force="--force" in sys.argv))

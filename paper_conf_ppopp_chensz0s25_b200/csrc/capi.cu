@@ -168,7 +168,8 @@ void nm_packed_free(nm_packed* P) {
   cudaGetDevice(&cur);
   cudaSetDevice(P->device);
   void* ptrs[] = {P->panel_mb_ptr, P->panel_chunk_ptr, P->unit_order, P->mb_seg, P->mb_sel,
-                  P->image, P->xrow, P->res_rowptr, P->res_col, P->res_val};
+                  P->image, P->res_rowptr, P->res_col, P->res_val, P->row_map,
+                  P->res_gather};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   cudaSetDevice(cur);

@@ -22,9 +22,15 @@ namespace nm {
 //            tools/probes/probe_umma_sp.b200.txt).
 constexpr int kPanelRows = 128;   // Vp = MMA M
 constexpr int kChunkMB = 8;       // meta-blocks per chunk (K = 32 logical / 4)
+//   xrow   : 32 x int32, the row of X gathered for each logical k (meta-block g, selected
+//            column j -> k = 4g + j); -1 = zero row (phantom or zero-count column: the TMA
+//            gather fills it with zeros without reading memory).
+// The record (4736 B) is moved by one cp.async.bulk per chunk.
 constexpr int kChunkValBytes = 4096;
 constexpr int kChunkMetaBytes = 512;
-constexpr int kChunkBytes = kChunkValBytes + kChunkMetaBytes;
+constexpr int kChunkXrowBytes = 128;
+constexpr int kChunkBytes = kChunkValBytes + kChunkMetaBytes + kChunkXrowBytes;
+constexpr int kChunkXrowOff = kChunkValBytes + kChunkMetaBytes;
 constexpr uint32_t kMetaNone = 0x44444444u;  // every nibble = (0,1): legal code, zero values
 
 }  // namespace nm
@@ -42,11 +48,14 @@ struct nm_packed {
   int32_t* unit_order = nullptr;       // [n_panels] panels, most chunks first
   int32_t* mb_seg = nullptr;           // [n_mb]
   uint32_t* mb_sel = nullptr;          // [n_mb] byte j = sel[j]
-  uint8_t* image = nullptr;            // [n_chunks * kChunkBytes]
-  int32_t* xrow = nullptr;             // [n_chunks * 32] row of PX per logical k, -1 = zero row
+  uint8_t* image = nullptr;            // [n_chunks * kChunkBytes] chunk records
   int64_t* res_rowptr = nullptr;       // [rows+1]
-  int32_t* res_col = nullptr;          // [res_nnz]
+  int32_t* res_col = nullptr;          // [res_nnz] canonical (permuted) column
   uint16_t* res_val = nullptr;         // [res_nnz]
+  // NM_PACK_ORIGINAL_ORDER: xrow holds original vertex ids, plus
+  int flags = 0;
+  int32_t* row_map = nullptr;          // [rows] output row of Y = perm[row_begin + l]
+  int32_t* res_gather = nullptr;       // [res_nnz] X row to gather = perm[res_col]
   size_t device_bytes = 0;
 };
 

@@ -20,6 +20,7 @@ __device__ __forceinline__ float h2f(uint16_t b, int bf) {
 template <int BF>
 __global__ void __launch_bounds__(256) k_residual(const int64_t* __restrict__ rp, const int32_t* __restrict__ rc,
                                                   const uint16_t* __restrict__ rv, int64_t rows,
+                                                  const int32_t* __restrict__ row_map,
                                                   const uint16_t* __restrict__ X, int64_t ldx,
                                                   float* __restrict__ Y, int64_t ldy, int F) {
   const int lane = threadIdx.x & 31;
@@ -45,7 +46,7 @@ __global__ void __launch_bounds__(256) k_residual(const int64_t* __restrict__ rp
           if (f + 2 < F) a2 += v * h2f(x[2], BF);
         }
       }
-      float* y = Y + l * ldy + f;
+      float* y = Y + (row_map ? (int64_t)row_map[l] : l) * ldy + f;
       if (f < F) y[0] += a0;
       if (f + 1 < F) y[1] += a1;
       if (f + 2 < F) y[2] += a2;
@@ -116,11 +117,12 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
                                cudaStream_t s) {
   const int64_t rows = P->row_end - P->row_begin;
   if (P->res_nnz == 0 || rows == 0) return NM_OK;
+  const int32_t* rcol = P->res_gather ? P->res_gather : P->res_col;
   if (P->dtype == NM_BF16)
-    k_residual<1><<<grid_rows(rows, 8), 256, 0, s>>>(P->res_rowptr, P->res_col, P->res_val, rows,
+    k_residual<1><<<grid_rows(rows, 8), 256, 0, s>>>(P->res_rowptr, rcol, P->res_val, rows, P->row_map,
                                                      (const uint16_t*)PX, ldx, Yp, ldy, F);
   else
-    k_residual<0><<<grid_rows(rows, 8), 256, 0, s>>>(P->res_rowptr, P->res_col, P->res_val, rows,
+    k_residual<0><<<grid_rows(rows, 8), 256, 0, s>>>(P->res_rowptr, rcol, P->res_val, rows, P->row_map,
                                                      (const uint16_t*)PX, ldx, Yp, ldy, F);
   NM_CUDA(cudaGetLastError());
   return NM_OK;

@@ -128,10 +128,14 @@ __global__ void k_meta_init(uint8_t* __restrict__ image, int64_t n_chunks) {
   }
 }
 
-__global__ void k_fill_i32(int32_t* __restrict__ a, int64_t n, int32_t v) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
-       i += (int64_t)gridDim.x * blockDim.x)
-    a[i] = v;
+// perm == nullptr: initialise every record's xrow to -1; else map xrow entries through perm
+__global__ void k_xrow_map(const int32_t* __restrict__ perm, uint8_t* __restrict__ image, int64_t n_chunks) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_chunks * 32;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t* x = (int32_t*)(image + (i >> 5) * kChunkBytes + kChunkXrowOff) + (i & 31);
+    if (!perm) *x = -1;
+    else if (*x >= 0) *x = perm[*x];
+  }
 }
 
 // per-entry meta-block id and column counts (warp per row)
@@ -157,7 +161,7 @@ __global__ void k_select(const int32_t* __restrict__ cnt, int Mp, int64_t n_mb,
                          const int64_t* __restrict__ mbkey, int64_t S, int64_t n,
                          const int64_t* __restrict__ mbp, const int64_t* __restrict__ chp,
                          int64_t P, int32_t* __restrict__ mb_seg, uint32_t* __restrict__ mb_sel,
-                         int32_t* __restrict__ xrow) {
+                         uint8_t* __restrict__ image) {
   for (int64_t m = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; m < n_mb;
        m += (int64_t)gridDim.x * blockDim.x) {
     int64_t panel = mbkey[m] / S, s = mbkey[m] % S;
@@ -187,10 +191,11 @@ __global__ void k_select(const int32_t* __restrict__ cnt, int Mp, int64_t n_mb,
     int64_t local = m - mbp[panel];
     int64_t chunk = chp[panel] + local / kChunkMB;
     int g = (int)(local % kChunkMB);
+    int32_t* xrow = (int32_t*)(image + chunk * kChunkBytes + kChunkXrowOff);
     for (int j = 0; j < 4; ++j) {
       int64_t col = s * Mp + sel[j];
       // zero-count or phantom columns gather nothing (zero-filled operand rows)
-      xrow[chunk * 32 + g * 4 + j] = (col < n && c[sel[j]] > 0) ? (int32_t)col : -1;
+      xrow[g * 4 + j] = (col < n && c[sel[j]] > 0) ? (int32_t)col : -1;
     }
   }
 }
@@ -340,8 +345,16 @@ nm_status scan_excl(const int64_t* in, int64_t* out, int64_t n, cudaStream_t s) 
   return NM_OK;
 }
 
+// identity == 1: a[i] = perm[i] (perm already offset); else a[i] = a[i] >= 0 ? perm[a[i]] : -1
+__global__ void k_map(const int32_t* __restrict__ perm, int32_t* __restrict__ a, int64_t m, int identity) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
+    if (identity) a[i] = perm[i];
+    else a[i] = a[i] >= 0 ? perm[a[i]] : -1;
+  }
+}
+
 nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int M, int Vp,
-                    nm_dtype dtype, int64_t rb, int64_t re, cudaStream_t s, nm_packed** out) {
+                    nm_dtype dtype, int64_t rb, int64_t re, int flags, cudaStream_t s, nm_packed** out) {
   if (!A || !out) return fail(NM_ERR_INVALID_ARG, "nm_pack: NULL argument");
   if (N != 2) return fail(NM_ERR_UNSUPPORTED, "nm_pack: N must be 2 (hardware 2:4, L496)");
   if (!(M == 4 || M == 8 || M == 16)) return fail(NM_ERR_UNSUPPORTED, "nm_pack: M must be 4, 8 or 16");
@@ -494,11 +507,10 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   NM_TRY(palloc((void**)&Pk->mb_seg, sizeof(int32_t) * n_mb));
   NM_TRY(palloc((void**)&Pk->mb_sel, sizeof(uint32_t) * n_mb));
   NM_TRY(palloc((void**)&Pk->image, (size_t)kChunkBytes * n_chunks));
-  NM_TRY(palloc((void**)&Pk->xrow, sizeof(int32_t) * 32 * n_chunks));
   NM_CUDA(cudaMemsetAsync(Pk->image, 0, (size_t)kChunkBytes * n_chunks, s));
   if (n_chunks) {
     k_meta_init<<<grid_for(n_chunks * 128, 256), 256, 0, s>>>(Pk->image, n_chunks);
-    k_fill_i32<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(Pk->xrow, n_chunks * 32, -1);
+    k_xrow_map<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(nullptr, Pk->image, n_chunks);
   }
 
   // ---- 3. column counts and selection ----
@@ -511,7 +523,7 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
                                                        d_cnt.as<int32_t>(), d_emb.as<int64_t>());
     k_select<<<grid_for(n_mb, 256), 256, 0, s>>>(d_cnt.as<int32_t>(), Mp, n_mb, d_mbkey.as<int64_t>(), S, n,
                                                  Pk->panel_mb_ptr, Pk->panel_chunk_ptr, P, Pk->mb_seg,
-                                                 Pk->mb_sel, Pk->xrow);
+                                                 Pk->mb_sel, Pk->image);
   }
   NM_CUDA(cudaGetLastError());
 
@@ -545,6 +557,20 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     k_res_fill<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, Bval, d_flag.as<uint8_t>(), rows,
                                                        Pk->res_rowptr, Pk->res_col, Pk->res_val);
   NM_CUDA(cudaGetLastError());
+  if (flags & NM_PACK_ORIGINAL_ORDER) {
+    // fold P into the operand indices: gather X[perm[q]], write Y[perm[p]]
+    Pk->flags = flags;
+    NM_TRY(palloc((void**)&Pk->row_map, sizeof(int32_t) * rows));
+    NM_TRY(palloc((void**)&Pk->res_gather, sizeof(int32_t) * res_nnz));
+    const int32_t* pm = d_perm.as<int32_t>();
+    k_map<<<grid_for(rows, 256), 256, 0, s>>>(pm + rb, Pk->row_map, rows, 1);
+    if (n_chunks) k_xrow_map<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(pm, Pk->image, n_chunks);
+    if (res_nnz) {
+      NM_CUDA(cudaMemcpyAsync(Pk->res_gather, Pk->res_col, sizeof(int32_t) * res_nnz, cudaMemcpyDeviceToDevice, s));
+      k_map<<<grid_for(res_nnz, 256), 256, 0, s>>>(pm, Pk->res_gather, res_nnz, 0);
+    }
+    NM_CUDA(cudaGetLastError());
+  }
   NM_CUDA(cudaStreamSynchronize(s));
   guard.ok = true;
   *out = Pk;
@@ -557,11 +583,18 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
 extern "C" nm_status nm_pack(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
                              nm_dtype dtype, void* stream, nm_packed** out) {
   if (!A) return nm::fail(NM_ERR_INVALID_ARG, "nm_pack: NULL graph");
-  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, 0, A->n, (cudaStream_t)stream, out);
+  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, 0, A->n, 0, (cudaStream_t)stream, out);
 }
 
 extern "C" nm_status nm_pack_rows(const nm_csr* A, const int32_t* perm, int V, int N, int M,
                                   int Vp, nm_dtype dtype, int64_t row_begin, int64_t row_end,
                                   void* stream, nm_packed** out) {
-  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, (cudaStream_t)stream, out);
+  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, 0, (cudaStream_t)stream, out);
+}
+
+extern "C" nm_status nm_pack_ex(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
+                                nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags, void* stream,
+                                nm_packed** out) {
+  if (flags & ~NM_PACK_ORIGINAL_ORDER) return nm::fail(NM_ERR_INVALID_ARG, "nm_pack_ex: unknown flags");
+  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, flags, (cudaStream_t)stream, out);
 }

@@ -23,9 +23,9 @@ import numpy as np
 
 def _csr_from_pairs(n: int, u: np.ndarray, v: np.ndarray):
     """Directed pairs (already both directions, unique) -> CSR with sorted columns."""
-    order = np.lexsort((v, u))
-    u = u[order]
-    v = v[order]
+    key = np.sort(u.astype(np.int64) * n + v.astype(np.int64))
+    u = key // n
+    v = key - u * n
     indptr = np.zeros(n + 1, np.int64)
     np.cumsum(np.bincount(u, minlength=n), out=indptr[1:])
     return indptr, v.astype(np.int32)
@@ -175,16 +175,18 @@ def symmetric_values(indptr, indices, seed: int, lo: float = 0.25, hi: float = 1
     """One value per undirected edge, |v| in [lo, hi) with a random sign (never +-0), stored
     on both (i,j) and (j,i) -- A stays symmetric in value, not only in pattern."""
     n = len(indptr) - 1
-    rows = np.repeat(np.arange(n, dtype=np.int64), np.diff(indptr))
-    cols = indices.astype(np.int64)
-    a = np.minimum(rows, cols)
-    b = np.maximum(rows, cols)
-    key = a * n + b
-    uniq, inv = np.unique(key, return_inverse=True)
-    rng = np.random.default_rng(seed)
-    mag = lo + (hi - lo) * rng.random(uniq.size)
-    sgn = np.where(rng.random(uniq.size) < 0.5, -1.0, 1.0)
-    return (mag * sgn)[inv].astype(np.float32)
+    rows = np.repeat(np.arange(n, dtype=np.uint64), np.diff(indptr))
+    cols = indices.astype(np.uint64)
+    key = np.minimum(rows, cols) * np.uint64(n) + np.maximum(rows, cols)
+    # counter-based: splitmix64(seed, edge key) -> 53-bit uniform + sign bit
+    with np.errstate(over="ignore"):
+        z = key + np.uint64(seed) * np.uint64(0x9E3779B97F4A7C15) + np.uint64(0x632BE59BD9B4E019)
+        z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+        z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+        z = z ^ (z >> np.uint64(31))
+    u = (z >> np.uint64(11)).astype(np.float64) * (1.0 / (1 << 53))
+    sgn = np.where((z & np.uint64(1)) == 1, -1.0, 1.0)
+    return ((lo + (hi - lo) * u) * sgn).astype(np.float32)
 
 
 def uniform_values(nnz: int, seed: int):

@@ -201,3 +201,39 @@ def test_empty_rows_and_isolated_vertices():
     api.spmm(P, X, Y)
     torch.cuda.synchronize()
     assert torch.all(Y[300:] == 0)
+
+
+@pytest.mark.parametrize("kind,seed,V,M", [("c1", 1, 1, 4), ("pl", 3, 1, 4), ("band", 5, 64, 8),
+                                           ("pl", 6, 128, 16)])
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+def test_spmm_original_order_fused(kind, seed, V, M, dtype):
+    """NM_PACK_ORIGINAL_ORDER: X in original order in, Y = A X in original order out, same
+    canonical pack; also row shards writing disjoint rows of one Y."""
+    dev = _cuda()
+    ip, ic = _graph(kind, seed)
+    n = len(ip) - 1
+    F = 96
+    perm, _ = api.reorder(ip, ic, V, 2, M)
+    v32, bits, v64 = _values(ip, ic, dtype, seed)
+    xbits, x64 = graphs.round16(graphs.features(n, F, seed + 2), dtype)
+    Y_ref, E, _ = oracle.spmm(ip, ic, v64, x64)
+    tdt = torch.float16 if dtype == "f16" else torch.bfloat16
+    X = torch.from_numpy(xbits.view(np.int16)).to(dev).view(tdt)
+    P = api.pack(ip, ic, perm, V, 2, M, dtype=dtype, val=v32, order="original")
+    ref = oracle.pack(ip, ic, bits, 0, perm, 128, 4 if V == 1 else M)
+    got = P.export_canonical()
+    for k in ("panel_ptr", "mb_seg", "nib", "vals", "res_rowptr", "res_col", "res_val"):
+        assert np.array_equal(ref[k], got[k]), k
+    Y = torch.full((n, F), float("nan"), device=dev)
+    api.spmm(P, X, Y)
+    torch.cuda.synchronize()
+    err = np.abs(Y.cpu().numpy().astype(np.float64) - Y_ref)
+    assert (err <= TOL * E).all(), err.max()
+    # two row shards into one buffer
+    Y2 = torch.full((n, F), float("nan"), device=dev)
+    cut = ((n // 2) // 128) * 128
+    for a, b in ((0, cut), (cut, n)):
+        Ps = api.pack(ip, ic, perm, V, 2, M, dtype=dtype, val=v32, order="original", row_begin=a, row_end=b)
+        api.spmm(Ps, X, Y2)
+    torch.cuda.synchronize()
+    assert torch.equal(Y, Y2)

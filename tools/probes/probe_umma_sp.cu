@@ -81,7 +81,7 @@ probe_kernel(const uint8_t* __restrict__ a_img, const uint8_t* __restrict__ b_im
     uint64_t bd = make_sdesc(smem_u32(smB), p.b_lbo, p.b_sbo) | ((uint64_t)p.b_layout << 61);
     uint32_t acc = 0;
     if (p.sparse) {
-      uint32_t e = tbase + p.meta_col;
+      uint32_t e = tbase + (p.meta_col & ~1u);  // odd column: even address + sparse_id2 = 1
       uint32_t idesc = p.idesc | (p.e_id2 & 3u);
       asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %5, 0;\n\t"
                    "tcgen05.mma.sp.cta_group::1.kind::f16 [%0], %1, %2, [%3], %4, q;\n\t}"
@@ -299,12 +299,12 @@ int main() {
         }
       }
     // id2 / column-offset probe with H1 at meta column 129 (odd) and id2 0/1
-    for (int id2 = 0; id2 < 0; ++id2) {
-      for (int col = 129; col <= 130; ++col) {
+    for (int id2 = 0; id2 < 1; ++id2) {
+      for (int col = 129; col <= 135; ++col) {
         Params p{};
         p.a_lbo = 128; p.a_sbo = 256; p.b_lbo = 128; p.b_sbo = 512;
         p.idesc = make_idesc(1, M, N, 0, 1);
-        p.sparse = 1; p.meta_col = col; p.e_id2 = id2;
+        p.sparse = 1; p.meta_col = col; p.e_id2 = col & 1;
         std::vector<float> out;
         run<32>(aimg, bimg, h1, out, p);
         int bad = 0;
