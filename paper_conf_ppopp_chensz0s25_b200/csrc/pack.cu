@@ -11,6 +11,8 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
+#include <cstdlib>
+#include <string>
 #include <numeric>
 #include <vector>
 
@@ -496,9 +498,11 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   {
     std::vector<int32_t> order(P);
     std::iota(order.begin(), order.end(), 0);
-    std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
-      return (chp[a + 1] - chp[a]) > (chp[b + 1] - chp[b]);
-    });
+    const char* ord = getenv("NM_UNIT_ORDER");
+    if (ord && std::string(ord) == "heavy")
+      std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+        return (chp[a + 1] - chp[a]) > (chp[b + 1] - chp[b]);
+      });
     NM_TRY(palloc((void**)&Pk->unit_order, sizeof(int32_t) * P));
     NM_CUDA(cudaMemcpyAsync(Pk->unit_order, order.data(), sizeof(int32_t) * P, cudaMemcpyHostToDevice, s));
     NM_CUDA(cudaStreamSynchronize(s));

@@ -4,34 +4,39 @@
 // panel is its list of non-empty meta-blocks; 8 meta-blocks (4 selected columns each) form
 // one K = 32 chunk, i.e. one tcgen05.mma.sp.cta_group::1.kind::f16 with M = 128, N = BN:
 //   record (A values, 2:4 metadata, 32 gather rows; 4736 B) <- one cp.async.bulk (HBM stream)
-//   B (32 gathered rows of X x BN, SWIZZLE_128B MN-major)  <- TMA tile::gather4, 4 rows each
+//   B (32 gathered rows of X x BN, SWIZZLE_128B MN-major)  <- cp.async 16-byte gathers
 //   E (metadata, 128 lanes x 32 b)                          <- tcgen05.st from shared memory
 //   D (fp32, 128 x BN)                                      in tensor memory (tcgen05.ld out)
-// Warp roles (persistent, one CTA per SM, 11 warps):
-//   w0 record TMA | w1 gather4 TMA | w2-5 metadata -> TMEM | w6 MMA issuer (+TMEM alloc)
-//   | w7-10 epilogue (TMEM -> registers -> Y).  All hand-offs are mbarriers; the pipeline
-//   runs across work units, so consecutive panels overlap.  Layouts measured on B200:
-//   tools/probes/probe_umma_sp.b200.txt, tools/probes/probe_gather4.b200.txt.
-#include <cuda.h>
-#include <cudaTypedefs.h>
+// Warp roles (persistent, one CTA per SM, 10 warps):
+//   w0 record TMA | w1-4 loaders: X gathers + metadata -> TMEM | w5 MMA issuer (+TMEM alloc)
+//   | w6-9 epilogue (TMEM -> registers -> smem transpose -> coalesced Y rows).
+// All hand-offs are mbarriers; the pipeline runs across work units, so consecutive panels
+// overlap.  The X gathers use cp.async rather than TMA tile::gather4: measured on B200 the
+// TMA unit spends ~57 cycles per gather4 instruction (4 rows x 128 B), which capped the
+// kernel at ~0.9 chunks/us/SM.  Layouts measured on B200:
+// tools/probes/probe_umma_sp.b200.txt, tools/probes/probe_gather4.b200.txt.
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 
-#include <mutex>
+#include <cstdlib>
 
 #include "nm_internal.h"
 
 namespace nm {
 namespace {
 
-constexpr int kThreads = 352;
-constexpr int kWarpRec = 0, kWarpGather = 1, kWarpMeta0 = 2, kWarpMma = 6;
+constexpr int kThreads = 320;
+constexpr int kWarpRec = 0, kWarpLoad0 = 1, kWarpMma = 5, kWarpEpi0 = 6;
+constexpr int kLoaders = 128;
+constexpr int kEpiTileFloats = 32 * 33;  // per epilogue warp: 32 rows x 32 cols (+1 pad)
 
 struct SpmmParams {
   const uint8_t* image;
   const int64_t* panel_chunk_ptr;
   const int32_t* unit_order;
   const int32_t* row_map;  // nullable: output row of Y for packed row l
+  const uint16_t* X;
+  int64_t ldx;
   float* Y;
   int64_t ldy;
   int F;
@@ -39,6 +44,7 @@ struct SpmmParams {
   int64_t n_units;
   int n_ftiles;
   uint32_t idesc;
+  int debug;  // profiling switches (NM_SPMM_DEBUG): 1 = no gathers, 2 = no Y stores, 8 = no metadata
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -72,13 +78,8 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t
       : "memory");
 }
 
-__device__ __forceinline__ void gather4(uint32_t dst, const CUtensorMap* tm, int col, int r0, int r1, int r2, int r3,
-                                        uint32_t mbar) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
-      "l"(tm), "r"(col), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(mbar)
-      : "memory");
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
 }
 
 __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t sbo, uint32_t layout) {
@@ -96,31 +97,34 @@ struct Cfg {
   static constexpr int kRecBytes = kChunkBytes;                 // 4736
   static constexpr int kBBytes = 32 * BN * 2;                   // 32 K-rows x BN halves
   static constexpr int kStageBytes = kRecBytes + kBBytes;
-  static constexpr int kStagesRaw = (216 * 1024) / kStageBytes;
+  static constexpr int kEpiBytes = 4 * kEpiTileFloats * 4;      // 16.5 KB
+  static constexpr int kStagesRaw = (214 * 1024 - kEpiBytes) / kStageBytes;
   static constexpr int kStages = kStagesRaw > 16 ? 16 : kStagesRaw;
+  static constexpr int kLag = kStages - 4 < 10 ? kStages - 4 : 10;  // chunks in flight per loader
   static constexpr int kNAcc = (2 * BN + kStages <= 512) ? 2 : 1;
   static constexpr int kMeta0 = kNAcc * BN;                     // metadata column of stage s: kMeta0 + s
   static constexpr int kRecRegion = ((kStages * kRecBytes + 1023) / 1024) * 1024;
-  static constexpr int kSmem = 1024 + kRecRegion + kStages * kBBytes + 1024;
+  static constexpr int kSmem = 1024 + kRecRegion + kStages * kBBytes + kEpiBytes + 1024;
   static_assert(kMeta0 + kStages <= 512, "TMEM budget");
   static_assert(BN % 64 == 0 && BN >= 64 && BN <= 256, "BN");
   static_assert(kSmem <= 227 * 1024, "smem");
+  static_assert(kLag >= 2, "pipeline depth");
 };
 
 template <int BN>
-__global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, const __grid_constant__ CUtensorMap tmX) {
+__global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
   using C = Cfg<BN>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  uint8_t* sRec = smem;                       // kStages records (16-byte aligned)
-  uint8_t* sB = smem + C::kRecRegion;         // kStages B tiles (1024-aligned)
-  uint64_t* bars = (uint64_t*)(sB + C::kStages * C::kBBytes);
-  uint64_t* full_a = bars;                    // record landed (tx)
-  uint64_t* full_b = bars + C::kStages;       // gathers landed (tx)
-  uint64_t* meta_ok = bars + 2 * C::kStages;  // metadata in TMEM (128 arrivals)
-  uint64_t* empty = bars + 3 * C::kStages;    // MMA done with the stage (tcgen05.commit)
-  uint64_t* tfull = bars + 4 * C::kStages;    // accumulator ready (2)
-  uint64_t* tempty = tfull + 2;               // accumulator drained (2)
+  uint8_t* sRec = smem;                                     // kStages records (16-byte aligned)
+  uint8_t* sB = smem + C::kRecRegion;                       // kStages B tiles (1024-aligned)
+  float* sEpi = (float*)(sB + C::kStages * C::kBBytes);     // epilogue transpose tiles
+  uint64_t* bars = (uint64_t*)((uint8_t*)sEpi + C::kEpiBytes);
+  uint64_t* full_a = bars;                  // record landed (tx)
+  uint64_t* full_b = bars + C::kStages;     // gathers + metadata ready (128 loader arrivals)
+  uint64_t* empty = bars + 2 * C::kStages;  // MMA done with the stage (tcgen05.commit)
+  uint64_t* tfull = bars + 3 * C::kStages;  // accumulator ready (2)
+  uint64_t* tempty = tfull + 2;             // accumulator drained (2)
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
 
   const int warp = threadIdx.x >> 5;
@@ -129,8 +133,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
   if (threadIdx.x == 0) {
     for (int s = 0; s < C::kStages; ++s) {
       mbar_init(smem_u32(&full_a[s]), 1);
-      mbar_init(smem_u32(&full_b[s]), 1);
-      mbar_init(smem_u32(&meta_ok[s]), 128);
+      mbar_init(smem_u32(&full_b[s]), 2 * kLoaders);  // cp.async completions + metadata stores
       mbar_init(smem_u32(&empty[s]), 1);
     }
     for (int a = 0; a < 2; ++a) {
@@ -139,7 +142,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == kWarpGather && lane == 0) asm volatile("prefetch.tensormap [%0];" ::"l"(&tmX) : "memory");
   if (warp == kWarpMma) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(tmem_slot)));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -165,8 +167,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
         }
       }
     }
-  } else if (warp == kWarpGather) {
-    // ------------------------------------------------------------ X gathers (TMA gather4)
+  } else if (warp >= kWarpLoad0 && warp < kWarpLoad0 + 4) {
+    // ------------------------------------------------------------ loaders: X gathers + metadata
+    const int quarter = warp & 3;                 // TMEM lane quarter of this warp
+    const int t = threadIdx.x - kWarpLoad0 * 32;  // 0..127
+    const int L = quarter * 32 + lane;            // TMEM lane this thread writes
+    constexpr int kRowPieces = BN / 8;            // 16-byte pieces per gathered row
+    constexpr int kPer = 32 * kRowPieces / kLoaders;
     int64_t i = 0;
     for (int64_t u = blockIdx.x; u < p.n_units; u += gridDim.x) {
       const int32_t panel = p.unit_order[u / p.n_ftiles];
@@ -176,41 +183,36 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
         const int s = (int)(i % C::kStages);
         const uint32_t ph = (uint32_t)((i / C::kStages) & 1);
         mbar_wait(smem_u32(&full_a[s]), ph);
-        const int32_t xr = *(const int32_t*)(sRec + s * C::kRecBytes + kChunkXrowOff + 4 * lane);
-        const int g = lane & 7;
-        const int r0 = __shfl_sync(0xffffffffu, xr, 4 * g + 0);
-        const int r1 = __shfl_sync(0xffffffffu, xr, 4 * g + 1);
-        const int r2 = __shfl_sync(0xffffffffu, xr, 4 * g + 2);
-        const int r3 = __shfl_sync(0xffffffffu, xr, 4 * g + 3);
-        if (lane == 0) mbar_arrive_tx(smem_u32(&full_b[s]), C::kBBytes);
-        __syncwarp();
-        if (lane < 8) {
-          const uint32_t dst = smem_u32(sB + s * C::kBBytes) + (g >> 1) * 1024 + (g & 1) * 512;
+        const uint8_t* rec = sRec + s * C::kRecBytes;
+        const uint32_t bst = smem_u32(sB + s * C::kBBytes);
 #pragma unroll
-          for (int nc = 0; nc < BN / 64; ++nc)
-            gather4(dst + nc * 4096, &tmX, ft * BN + nc * 64, r0, r1, r2, r3, smem_u32(&full_b[s]));
+        for (int q = 0; q < kPer; ++q) {
+          const int idx = t + kLoaders * q;
+          const int k = idx / kRowPieces, c16 = idx % kRowPieces;
+          int32_t xr = *(const int32_t*)(rec + kChunkXrowOff + 4 * k);
+          if (p.debug & 1) xr = -1;
+          const int col0 = ft * BN + c16 * 8;
+          uint32_t bytes = 0;
+          const uint16_t* src = p.X;
+          if (xr >= 0 && col0 < p.F) {
+            const int rem = p.F - col0;
+            bytes = rem >= 8 ? 16u : (uint32_t)(rem * 2);
+            src = p.X + (int64_t)xr * p.ldx + col0;
+          }
+          const uint32_t dst = bst + (c16 >> 3) * 4096 + (k >> 3) * 1024 + (k & 7) * 128 +
+                               ((((uint32_t)c16 & 7u) ^ ((uint32_t)k & 7u)) << 4);
+          cp_async16(dst, src, bytes);
         }
-        __syncwarp();
-      }
-    }
-  } else if (warp >= kWarpMeta0 && warp < kWarpMeta0 + 4) {
-    // ------------------------------------------------------------ 2:4 metadata -> TMEM
-    const int quarter = warp & 3;
-    const int L = quarter * 32 + lane;
-    int64_t i = 0;
-    for (int64_t u = blockIdx.x; u < p.n_units; u += gridDim.x) {
-      const int32_t panel = p.unit_order[u / p.n_ftiles];
-      const int64_t c0 = p.panel_chunk_ptr[panel], c1 = p.panel_chunk_ptr[panel + 1];
-      for (int64_t c = c0; c < c1; ++c, ++i) {
-        const int s = (int)(i % C::kStages);
-        const uint32_t ph = (uint32_t)((i / C::kStages) & 1);
-        mbar_wait(smem_u32(&full_a[s]), ph);
-        const uint32_t w = *(const uint32_t*)(sRec + s * C::kRecBytes + kChunkValBytes + 4 * L);
-        const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + s;
-        asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(w) : "memory");
-        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        // the barrier tracks this thread's gathers asynchronously (arrival when they land)
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&full_b[s])) : "memory");
+        if (!(p.debug & 8)) {
+          const uint32_t w = *(const uint32_t*)(rec + kChunkValBytes + 4 * L);
+          const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + s;
+          asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(w) : "memory");
+          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        }
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-        mbar_arrive(smem_u32(&meta_ok[s]));
+        mbar_arrive(smem_u32(&full_b[s]));
       }
     }
   } else if (warp == kWarpMma) {
@@ -230,7 +232,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
         const int s = (int)(i % C::kStages);
         const uint32_t ph = (uint32_t)((i / C::kStages) & 1);
         mbar_wait(smem_u32(&full_b[s]), ph);
-        mbar_wait(smem_u32(&meta_ok[s]), ph);
+        // gathers were written through the generic proxy (cp.async); order them before the
+        // tensor core's async-proxy reads of the stage
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         if (lane == 0) {
           const uint64_t ad = adesc0 + (uint64_t)((s * C::kRecBytes) >> 4);
@@ -264,20 +268,21 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
   } else {
     // ------------------------------------------------------------ epilogue
     const int quarter = warp & 3;  // TMEM lane quarter this warp may access
-    const int r = quarter * 32 + lane;
+    float* tile = sEpi + (warp - kWarpEpi0) * kEpiTileFloats;
     int acc = 0;
     uint32_t aphase = 0;
     const bool vec_ok = ((p.ldy & 3) == 0) && ((((uintptr_t)p.Y) & 15) == 0);
+    const int rsub = lane >> 3;       // row within a 4-row store group
+    const int cq = (lane & 7) * 4;    // column quad within the 32-column slice
     for (int64_t u = blockIdx.x; u < p.n_units; u += gridDim.x) {
       const int32_t panel = p.unit_order[u / p.n_ftiles];
       const int ft = (int)(u % p.n_ftiles);
       const int64_t c0 = p.panel_chunk_ptr[panel], c1 = p.panel_chunk_ptr[panel + 1];
+      // this lane's row (as the TMEM lane owner) and its output row in Y
+      const int64_t myrow = (int64_t)panel * kPanelRows + quarter * 32 + lane;
+      const int64_t myout = myrow < p.rows ? (p.row_map ? (int64_t)p.row_map[myrow] : myrow) : -1;
       mbar_wait(smem_u32(&tfull[acc]), aphase);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-      const int64_t grow = (int64_t)panel * kPanelRows + r;
-      const bool row_ok = grow < p.rows;
-      const int64_t orow = (row_ok && p.row_map) ? (int64_t)p.row_map[grow] : grow;
-      float* yrow = p.Y + orow * p.ldy;
 #pragma unroll 1
       for (int cc = 0; cc < BN; cc += 32) {
         uint32_t v[32];
@@ -298,20 +303,27 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
           for (int j = 0; j < 32; ++j) v[j] = 0u;
         }
         const int col = ft * BN + cc;
-        if (row_ok && col < p.F) {
-          if (vec_ok && col + 32 <= p.F) {
+        if (col >= p.F || (p.debug & 2)) continue;  // warp-uniform
+        // transpose through shared memory: lane = row -> lanes = 4 rows x 8 column quads
 #pragma unroll
-            for (int j = 0; j < 32; j += 4) {
-              float4 f = make_float4(__uint_as_float(v[j]), __uint_as_float(v[j + 1]), __uint_as_float(v[j + 2]),
-                                     __uint_as_float(v[j + 3]));
-              __stcs((float4*)(yrow + col + j), f);
+        for (int j = 0; j < 32; ++j) tile[lane * 33 + j] = __uint_as_float(v[j]);
+        __syncwarp();
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+          const int rr = g * 4 + rsub;
+          const int64_t orow = __shfl_sync(0xffffffffu, myout, rr);
+          const float* tr = tile + rr * 33 + cq;
+          if (orow >= 0) {
+            float* dst = p.Y + orow * p.ldy + col + cq;
+            if (vec_ok && col + cq + 4 <= p.F) {
+              __stcs((float4*)dst, make_float4(tr[0], tr[1], tr[2], tr[3]));
+            } else {
+              for (int e = 0; e < 4; ++e)
+                if (col + cq + e < p.F) dst[e] = tr[e];
             }
-          } else {
-#pragma unroll
-            for (int j = 0; j < 32; ++j)
-              if (col + j < p.F) yrow[col + j] = __uint_as_float(v[j]);
           }
         }
+        __syncwarp();
       }
       asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
       mbar_arrive(smem_u32(&tempty[acc]));
@@ -338,35 +350,6 @@ uint32_t make_idesc(nm_dtype dt, int BN) {
   return d;
 }
 
-PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
-  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
-  static std::once_flag once;
-  std::call_once(once, [] {
-    cudaDriverEntryPointQueryResult q;
-    void* f = nullptr;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
-        q == cudaDriverEntryPointSuccess)
-      fn = (PFN_cuTensorMapEncodeTiled_v12000)f;
-  });
-  return fn;
-}
-
-// X as a 2-D tensor [n rows x F columns], row pitch ldx; box = 64 columns x 1 row, 128-byte
-// swizzle (the UMMA SW128 MN-major atom); rows and columns outside the tensor read as zero.
-nm_status make_x_map(CUtensorMap* tm, const void* X, int64_t n, int F, int64_t ldx, nm_dtype dt) {
-  auto enc = tensor_map_encoder();
-  if (!enc) return fail(NM_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
-  cuuint64_t dims[2] = {(cuuint64_t)F, (cuuint64_t)n};
-  cuuint64_t strides[1] = {(cuuint64_t)ldx * 2};
-  cuuint32_t box[2] = {64, 1};
-  cuuint32_t es[2] = {1, 1};
-  CUresult r = enc(tm, dt == NM_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2,
-                   const_cast<void*>(X), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) return fail(NM_ERR_CUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)r));
-  return NM_OK;
-}
-
 template <int BN>
 nm_status launch_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F, cudaStream_t s) {
   using C = Cfg<BN>;
@@ -379,14 +362,13 @@ nm_status launch_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, 
   }
   int sms = 148;
   NM_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-  CUtensorMap tm;
-  nm_status st = make_x_map(&tm, PX, P->n, F, ldx, P->dtype);
-  if (st != NM_OK) return st;
   SpmmParams prm;
   prm.image = P->image;
   prm.panel_chunk_ptr = P->panel_chunk_ptr;
   prm.unit_order = P->unit_order;
   prm.row_map = P->row_map;
+  prm.X = (const uint16_t*)PX;
+  prm.ldx = ldx;
   prm.Y = Yp;
   prm.ldy = ldy;
   prm.F = F;
@@ -394,9 +376,11 @@ nm_status launch_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, 
   prm.n_ftiles = (F + BN - 1) / BN;
   prm.n_units = P->n_panels * prm.n_ftiles;
   prm.idesc = make_idesc(P->dtype, BN);
+  const char* dbg = getenv("NM_SPMM_DEBUG");
+  prm.debug = dbg ? atoi(dbg) : 0;
   int64_t grid = prm.n_units < sms ? prm.n_units : sms;
   if (grid < 1) return NM_OK;
-  k_spmm_sptc<BN><<<(unsigned)grid, kThreads, C::kSmem, s>>>(prm, tm);
+  k_spmm_sptc<BN><<<(unsigned)grid, kThreads, C::kSmem, s>>>(prm);
   NM_CUDA(cudaGetLastError());
   return NM_OK;
 }
