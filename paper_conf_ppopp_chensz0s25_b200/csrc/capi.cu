@@ -167,7 +167,7 @@ void nm_packed_free(nm_packed* P) {
   int cur = 0;
   cudaGetDevice(&cur);
   cudaSetDevice(P->device);
-  void* ptrs[] = {P->panel_mb_ptr, P->panel_chunk_ptr, P->unit_order, P->mb_seg, P->mb_sel,
+  void* ptrs[] = {P->panel_mb_ptr, P->panel_chunk_ptr, P->unit_info, P->mb_seg, P->mb_sel,
                   P->image, P->res_rowptr, P->res_col, P->res_val, P->row_map,
                   P->res_gather};
   for (void* p : ptrs)

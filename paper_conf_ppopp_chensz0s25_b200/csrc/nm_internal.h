@@ -45,7 +45,7 @@ struct nm_packed {
   // device arrays
   int64_t* panel_mb_ptr = nullptr;     // [n_panels+1]
   int64_t* panel_chunk_ptr = nullptr;  // [n_panels+1]
-  int32_t* unit_order = nullptr;       // [n_panels] panels, most chunks first
+  int4* unit_info = nullptr;           // [n_panels] schedule: {panel, #chunks, first chunk lo, hi}
   int32_t* mb_seg = nullptr;           // [n_mb]
   uint32_t* mb_sel = nullptr;          // [n_mb] byte j = sel[j]
   uint8_t* image = nullptr;            // [n_chunks * kChunkBytes] chunk records

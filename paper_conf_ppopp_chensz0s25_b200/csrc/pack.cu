@@ -494,7 +494,9 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   const int64_t n_chunks = chp[P];
   Pk->n_chunks = n_chunks;
 
-  // unit order: panels with most chunks first (stable) -- greedy balance for the persistent grid
+  // unit schedule: natural panel order (consecutive panels run concurrently on the persistent
+  // grid, so their X neighbourhoods are shared in L2); NM_UNIT_ORDER=heavy sorts by chunk
+  // count instead.  One 16-byte descriptor per panel: {panel, #chunks, first chunk}.
   {
     std::vector<int32_t> order(P);
     std::iota(order.begin(), order.end(), 0);
@@ -503,8 +505,14 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
       std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
         return (chp[a + 1] - chp[a]) > (chp[b + 1] - chp[b]);
       });
-    NM_TRY(palloc((void**)&Pk->unit_order, sizeof(int32_t) * P));
-    NM_CUDA(cudaMemcpyAsync(Pk->unit_order, order.data(), sizeof(int32_t) * P, cudaMemcpyHostToDevice, s));
+    std::vector<int4> info(P);
+    for (int64_t j = 0; j < P; ++j) {
+      const int32_t r = order[j];
+      const int64_t c0 = chp[r];
+      info[j] = make_int4(r, (int32_t)(chp[r + 1] - c0), (int32_t)(c0 & 0xFFFFFFFF), (int32_t)(c0 >> 32));
+    }
+    NM_TRY(palloc((void**)&Pk->unit_info, sizeof(int4) * P));
+    NM_CUDA(cudaMemcpyAsync(Pk->unit_info, info.data(), sizeof(int4) * P, cudaMemcpyHostToDevice, s));
     NM_CUDA(cudaStreamSynchronize(s));
   }
 

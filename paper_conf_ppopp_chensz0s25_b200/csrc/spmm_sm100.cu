@@ -7,17 +7,21 @@
 //   B (32 gathered rows of X x BN, SWIZZLE_128B MN-major)  <- cp.async 16-byte gathers
 //   E (metadata, 128 lanes x 32 b)                          <- tcgen05.st from shared memory
 //   D (fp32, 128 x BN)                                      in tensor memory (tcgen05.ld out)
-// Warp roles (persistent, one CTA per SM, 10 warps):
-//   w0 record TMA | w1-4 loaders: X gathers + metadata -> TMEM | w5 MMA issuer (+TMEM alloc)
-//   | w6-9 epilogue (TMEM -> registers -> smem transpose -> coalesced Y rows).
+// Warp roles (persistent, one CTA per SM, 18 warps):
+//   w0 record TMA + L2 prefetch of the next units' records
+//   w1-8 loaders, two groups of 4 warps taking alternate chunks: X gathers + metadata
+//   w9 MMA issuer (+ TMEM allocation)
+//   w10-17 epilogue, two warps per TMEM lane quarter: tcgen05.ld 16x256b -> 32-byte
+//   sector-aligned stores of Y rows (no shared-memory staging).
 // All hand-offs are mbarriers; the pipeline runs across work units, so consecutive panels
-// overlap.  The X gathers use cp.async rather than TMA tile::gather4: measured on B200 the
-// TMA unit spends ~57 cycles per gather4 instruction (4 rows x 128 B), which capped the
-// kernel at ~0.9 chunks/us/SM.  Layouts measured on B200:
-// tools/probes/probe_umma_sp.b200.txt, tools/probes/probe_gather4.b200.txt.
+// overlap, and every role prefetches the next unit's 16-byte schedule entry.  Design
+// evidence: TMA tile::gather4 costs ~57 cycles per instruction on B200, so X
+// rows are gathered with cp.async; a single loader group spent ~950 cycles per chunk
+// (clock64 timeline, tools/trace_spmm.py), so two groups alternate.
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 
+#include <cstdio>
 #include <cstdlib>
 
 #include "nm_internal.h"
@@ -25,15 +29,18 @@
 namespace nm {
 namespace {
 
-constexpr int kThreads = 320;
-constexpr int kWarpRec = 0, kWarpLoad0 = 1, kWarpMma = 5, kWarpEpi0 = 6;
-constexpr int kLoaders = 128;
-constexpr int kEpiTileFloats = 32 * 33;  // per epilogue warp: 32 rows x 32 cols (+1 pad)
+#ifndef NM_LOAD_GROUPS
+#define NM_LOAD_GROUPS 3
+#endif
+constexpr int kWarpRec = 0, kWarpLoad0 = 1, kLoadGroups = NM_LOAD_GROUPS;
+constexpr int kWarpMma = kWarpLoad0 + 4 * kLoadGroups, kWarpEpi0 = kWarpMma + 1, kEpiWarps = 8;
+constexpr int kThreads = (kWarpEpi0 + kEpiWarps) * 32;  // 576
+constexpr int kGroupThreads = 128;                     // loader threads per group
+constexpr int kPrefetchUnits = 2;                      // record L2-prefetch distance (units)
 
 struct SpmmParams {
   const uint8_t* image;
-  const int64_t* panel_chunk_ptr;
-  const int32_t* unit_order;
+  const int4* unit_info;   // per scheduled panel: {panel, #chunks, first chunk lo, hi}
   const int32_t* row_map;  // nullable: output row of Y for packed row l
   const uint16_t* X;
   int64_t ldx;
@@ -44,10 +51,27 @@ struct SpmmParams {
   int64_t n_units;
   int n_ftiles;
   uint32_t idesc;
-  int debug;  // profiling switches (NM_SPMM_DEBUG): 1 = no gathers, 2 = no Y stores, 8 = no metadata
+  int debug;                  // profiling switches (NM_SPMM_DEBUG): 1 = no gather reads, 2 = no Y stores
+  unsigned long long* trace;  // NM_SPMM_TRACE: per-chunk clock64 timeline of CTA 0
 };
 
+#define NM_TRACE(slot)                                                                              \
+  do {                                                                                              \
+    if (p.trace && blockIdx.x == 0 && i < 1024) p.trace[i * 8 + (slot)] = clock64();                \
+  } while (0)
+#define NM_TRACE_U(slot)                                                                            \
+  do {                                                                                              \
+    if (p.trace && blockIdx.x == 0 && lane == 0 && (u / ustep) < 1024)                               \
+      p.trace[8192 + (u / ustep) * 4 + (slot)] = clock64();                                         \
+  } while (0)
+
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
 
 __device__ __forceinline__ void mbar_init(uint32_t a, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count));
@@ -92,23 +116,26 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t
   return d;
 }
 
+// schedule entry of unit u (prefetched one unit ahead by every role)
+__device__ __forceinline__ int4 unit_entry(const SpmmParams& p, int64_t u) {
+  return u < p.n_units ? __ldg(p.unit_info + u / p.n_ftiles) : make_int4(0, 0, 0, 0);
+}
+__device__ __forceinline__ int64_t entry_c0(int4 e) { return (int64_t)(uint32_t)e.z | ((int64_t)e.w << 32); }
+
 template <int BN>
 struct Cfg {
   static constexpr int kRecBytes = kChunkBytes;                 // 4736
   static constexpr int kBBytes = 32 * BN * 2;                   // 32 K-rows x BN halves
   static constexpr int kStageBytes = kRecBytes + kBBytes;
-  static constexpr int kEpiBytes = 4 * kEpiTileFloats * 4;      // 16.5 KB
-  static constexpr int kStagesRaw = (214 * 1024 - kEpiBytes) / kStageBytes;
+  static constexpr int kStagesRaw = (214 * 1024) / kStageBytes;
   static constexpr int kStages = kStagesRaw > 16 ? 16 : kStagesRaw;
-  static constexpr int kLag = kStages - 4 < 10 ? kStages - 4 : 10;  // chunks in flight per loader
   static constexpr int kNAcc = (2 * BN + kStages <= 512) ? 2 : 1;
   static constexpr int kMeta0 = kNAcc * BN;                     // metadata column of stage s: kMeta0 + s
   static constexpr int kRecRegion = ((kStages * kRecBytes + 1023) / 1024) * 1024;
-  static constexpr int kSmem = 1024 + kRecRegion + kStages * kBBytes + kEpiBytes + 1024;
+  static constexpr int kSmem = 1024 + kRecRegion + kStages * kBBytes + 1024;
   static_assert(kMeta0 + kStages <= 512, "TMEM budget");
   static_assert(BN % 64 == 0 && BN >= 64 && BN <= 256, "BN");
   static_assert(kSmem <= 227 * 1024, "smem");
-  static_assert(kLag >= 2, "pipeline depth");
 };
 
 template <int BN>
@@ -116,12 +143,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
   using C = Cfg<BN>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  uint8_t* sRec = smem;                                     // kStages records (16-byte aligned)
-  uint8_t* sB = smem + C::kRecRegion;                       // kStages B tiles (1024-aligned)
-  float* sEpi = (float*)(sB + C::kStages * C::kBBytes);     // epilogue transpose tiles
-  uint64_t* bars = (uint64_t*)((uint8_t*)sEpi + C::kEpiBytes);
+  const uint32_t sRec = smem_u32(smem);      // kStages records (16-byte aligned)
+  const uint32_t sB = sRec + C::kRecRegion;  // kStages B tiles (1024-aligned)
+  uint64_t* bars = (uint64_t*)(smem + C::kRecRegion + C::kStages * C::kBBytes);
   uint64_t* full_a = bars;                  // record landed (tx)
-  uint64_t* full_b = bars + C::kStages;     // gathers + metadata ready (128 loader arrivals)
+  uint64_t* full_b = bars + C::kStages;     // gathers + metadata ready
   uint64_t* empty = bars + 2 * C::kStages;  // MMA done with the stage (tcgen05.commit)
   uint64_t* tfull = bars + 3 * C::kStages;  // accumulator ready (2)
   uint64_t* tempty = tfull + 2;             // accumulator drained (2)
@@ -133,12 +159,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
   if (threadIdx.x == 0) {
     for (int s = 0; s < C::kStages; ++s) {
       mbar_init(smem_u32(&full_a[s]), 1);
-      mbar_init(smem_u32(&full_b[s]), 2 * kLoaders);  // cp.async completions + metadata stores
+      mbar_init(smem_u32(&full_b[s]), 2 * kGroupThreads);  // cp.async completions + metadata stores
       mbar_init(smem_u32(&empty[s]), 1);
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(smem_u32(&tfull[a]), 1);
-      mbar_init(smem_u32(&tempty[a]), 128);
+      mbar_init(smem_u32(&tempty[a]), kEpiWarps * 32);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -150,99 +176,126 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   const uint32_t tbase = *tmem_slot;
+  const int64_t ustep = gridDim.x;
 
   if (warp == kWarpRec) {
     // ------------------------------------------------------------ record producer (HBM stream)
     if (lane == 0) {
       int64_t i = 0;
-      for (int64_t u = blockIdx.x; u < p.n_units; u += gridDim.x) {
-        const int32_t panel = p.unit_order[u / p.n_ftiles];
-        const int64_t c0 = p.panel_chunk_ptr[panel], c1 = p.panel_chunk_ptr[panel + 1];
+      int4 nxt = unit_entry(p, blockIdx.x);
+      // the records of a panel are contiguous: stream the next units' records into L2 ahead
+      // of their bulk copies (one bulk prefetch per unit, kPrefetchUnits units ahead)
+      auto prefetch_unit = [&](int4 e) {
+        if (e.y > 0)
+          asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p.image + entry_c0(e) * kChunkBytes),
+                       "r"((uint32_t)(e.y * kChunkBytes))
+                       : "memory");
+      };
+      for (int k = 0; k < kPrefetchUnits; ++k) prefetch_unit(unit_entry(p, blockIdx.x + k * ustep));
+      int s = 0;
+      uint32_t ph = 0;
+      for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
+        const int4 cur = nxt;
+        nxt = unit_entry(p, u + ustep);
+        prefetch_unit(unit_entry(p, u + kPrefetchUnits * ustep));
+        const int64_t c0 = entry_c0(cur), c1 = c0 + cur.y;
         for (int64_t c = c0; c < c1; ++c, ++i) {
-          const int s = (int)(i % C::kStages);
-          const uint32_t ph = (uint32_t)((i / C::kStages) & 1);
           mbar_wait(smem_u32(&empty[s]), ph ^ 1);
+          NM_TRACE(0);
           mbar_arrive_tx(smem_u32(&full_a[s]), C::kRecBytes);
-          bulk_g2s(smem_u32(sRec + s * C::kRecBytes), p.image + c * kChunkBytes, C::kRecBytes, smem_u32(&full_a[s]));
+          bulk_g2s(sRec + s * C::kRecBytes, p.image + c * kChunkBytes, C::kRecBytes, smem_u32(&full_a[s]));
+          if (++s == C::kStages) { s = 0; ph ^= 1; }
         }
       }
     }
-  } else if (warp >= kWarpLoad0 && warp < kWarpLoad0 + 4) {
+  } else if (warp >= kWarpLoad0 && warp < kWarpLoad0 + 4 * kLoadGroups) {
     // ------------------------------------------------------------ loaders: X gathers + metadata
-    const int quarter = warp & 3;                 // TMEM lane quarter of this warp
-    const int t = threadIdx.x - kWarpLoad0 * 32;  // 0..127
-    const int L = quarter * 32 + lane;            // TMEM lane this thread writes
-    constexpr int kRowPieces = BN / 8;            // 16-byte pieces per gathered row
-    constexpr int kPer = 32 * kRowPieces / kLoaders;
+    const int group = (warp - kWarpLoad0) >> 2;  // takes chunks i with i % kLoadGroups == group
+    const int quarter = warp & 3;                               // TMEM lane quarter of this warp
+    const int t = threadIdx.x - (kWarpLoad0 + 4 * group) * 32;  // 0..127 within the group
+    const int L = quarter * 32 + lane;                          // TMEM lane this thread writes
+    const int k = t >> 2;                                       // gathered row (logical K index)
+    const int sub = t & 3;
+    constexpr int kRowPieces = BN / 8;  // 16-byte pieces per gathered row
+    constexpr int kPer = kRowPieces / 4;  // pieces per thread
     int64_t i = 0;
-    for (int64_t u = blockIdx.x; u < p.n_units; u += gridDim.x) {
-      const int32_t panel = p.unit_order[u / p.n_ftiles];
+    int s_next = 0, g_next = 0;
+    uint32_t ph_next = 0;
+    int4 nxt = unit_entry(p, blockIdx.x);
+    for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
+      const int4 cur = nxt;
+      nxt = unit_entry(p, u + ustep);
       const int ft = (int)(u % p.n_ftiles);
-      const int64_t c0 = p.panel_chunk_ptr[panel], c1 = p.panel_chunk_ptr[panel + 1];
+      const int64_t c0 = entry_c0(cur), c1 = c0 + cur.y;
       for (int64_t c = c0; c < c1; ++c, ++i) {
-        const int s = (int)(i % C::kStages);
-        const uint32_t ph = (uint32_t)((i / C::kStages) & 1);
+        const int s = s_next;
+        const uint32_t ph = ph_next;
+        if (++s_next == C::kStages) { s_next = 0; ph_next ^= 1; }
+        const int g = g_next;
+        if (++g_next == kLoadGroups) g_next = 0;
+        if (g != group) continue;
         mbar_wait(smem_u32(&full_a[s]), ph);
-        const uint8_t* rec = sRec + s * C::kRecBytes;
-        const uint32_t bst = smem_u32(sB + s * C::kBBytes);
+        if (t == 0) NM_TRACE(1);
+        const uint32_t rec = sRec + s * C::kRecBytes;
+        const uint32_t brow = sB + s * C::kBBytes + (k >> 3) * 1024 + (k & 7) * 128;
+        int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * k);
+        if (p.debug & 1) xr = -1;
+        const uint16_t* xsrc = p.X + (int64_t)(xr < 0 ? 0 : xr) * p.ldx;
 #pragma unroll
         for (int q = 0; q < kPer; ++q) {
-          const int idx = t + kLoaders * q;
-          const int k = idx / kRowPieces, c16 = idx % kRowPieces;
-          int32_t xr = *(const int32_t*)(rec + kChunkXrowOff + 4 * k);
-          if (p.debug & 1) xr = -1;
+          const int c16 = sub + 4 * q;
           const int col0 = ft * BN + c16 * 8;
           uint32_t bytes = 0;
-          const uint16_t* src = p.X;
           if (xr >= 0 && col0 < p.F) {
             const int rem = p.F - col0;
             bytes = rem >= 8 ? 16u : (uint32_t)(rem * 2);
-            src = p.X + (int64_t)xr * p.ldx + col0;
           }
-          const uint32_t dst = bst + (c16 >> 3) * 4096 + (k >> 3) * 1024 + (k & 7) * 128 +
-                               ((((uint32_t)c16 & 7u) ^ ((uint32_t)k & 7u)) << 4);
-          cp_async16(dst, src, bytes);
+          const uint32_t dst = brow + (c16 >> 3) * 4096 + ((((uint32_t)c16 & 7u) ^ ((uint32_t)k & 7u)) << 4);
+          cp_async16(dst, bytes ? (const void*)(xsrc + col0) : (const void*)p.X, bytes);
         }
         // the barrier tracks this thread's gathers asynchronously (arrival when they land)
         asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&full_b[s])) : "memory");
-        if (!(p.debug & 8)) {
-          const uint32_t w = *(const uint32_t*)(rec + kChunkValBytes + 4 * L);
-          const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + s;
-          asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(w) : "memory");
-          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-        }
+        const uint32_t w = lds32(rec + kChunkValBytes + 4 * L);
+        const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + s;
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(w) : "memory");
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         mbar_arrive(smem_u32(&full_b[s]));
+        if (t == 0) NM_TRACE(2);
       }
     }
   } else if (warp == kWarpMma) {
-    // ------------------------------------------------------------ MMA issuer
-    int64_t i = 0;
-    int acc = 0;
-    uint32_t aphase = 0;
-    const uint64_t adesc0 = sdesc(smem_u32(sRec), 128, 256, 0);
-    const uint64_t bdesc0 = sdesc(smem_u32(sB), 4096, 1024, 2);
-    for (int64_t u = blockIdx.x; u < p.n_units; u += gridDim.x) {
-      const int32_t panel = p.unit_order[u / p.n_ftiles];
-      const int64_t c0 = p.panel_chunk_ptr[panel], c1 = p.panel_chunk_ptr[panel + 1];
-      mbar_wait(smem_u32(&tempty[acc]), aphase ^ 1);
-      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-      const uint32_t dcol = tbase + acc * BN;
-      for (int64_t c = c0; c < c1; ++c, ++i) {
-        const int s = (int)(i % C::kStages);
-        const uint32_t ph = (uint32_t)((i / C::kStages) & 1);
-        mbar_wait(smem_u32(&full_b[s]), ph);
-        // gathers were written through the generic proxy (cp.async); order them before the
-        // tensor core's async-proxy reads of the stage
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    // ------------------------------------------------------------ MMA issuer (one thread)
+    // The cp.async gathers are published through cp.async.mbarrier.arrive on full_b; as in
+    // CUTLASS's PipelineUmmaConsumerAsync (cp.async -> UMMA) no extra proxy fence is issued.
+    if (lane == 0) {
+      int64_t i = 0;  // chunk counter (trace only)
+      int s = 0;
+      uint32_t ph = 0;
+      int acc = 0;
+      uint32_t aphase = 0;
+      const uint64_t adesc0 = sdesc(sRec, 128, 256, 0);
+      const uint64_t bdesc0 = sdesc(sB, 4096, 1024, 2);
+      int4 nxt = unit_entry(p, blockIdx.x);
+      for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
+        const int4 cur = nxt;
+        nxt = unit_entry(p, u + ustep);
+        const int nch = cur.y;
+        mbar_wait(smem_u32(&tempty[acc]), aphase ^ 1);
+        NM_TRACE_U(1);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        if (lane == 0) {
+        const uint32_t dcol = tbase + acc * BN;
+        for (int c = 0; c < nch; ++c, ++i) {
+          mbar_wait(smem_u32(&full_b[s]), ph);
+          NM_TRACE(3);
+          if (p.debug & 16) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
           const uint64_t ad = adesc0 + (uint64_t)((s * C::kRecBytes) >> 4);
           const uint64_t bd = bdesc0 + (uint64_t)((s * C::kBBytes) >> 4);
           const uint32_t mcol = C::kMeta0 + s;
           const uint32_t ecol = tbase + (mcol & ~1u);   // even column address ...
           const uint32_t idesc = p.idesc | (mcol & 1u);  // ... + sparse_id2 selects the odd one
-          const uint32_t accum = (c > c0) ? 1u : 0u;
+          const uint32_t accum = c > 0 ? 1u : 0u;
           asm volatile(
               "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %5, 0;\n\t"
               "tcgen05.mma.sp.cta_group::1.kind::f16 [%0], %1, %2, [%3], %4, q;\n\t}" ::"r"(dcol),
@@ -251,45 +304,58 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
           asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
                            smem_u32(&empty[s]))
                        : "memory");
+          if (++s == C::kStages) { s = 0; ph ^= 1; }
         }
-        __syncwarp();
-      }
-      if (lane == 0) {
-        if (c1 > c0)
+        if (nch > 0)
           asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
                            smem_u32(&tfull[acc]))
                        : "memory");
         else
           mbar_arrive(smem_u32(&tfull[acc]));
+        if (++acc == C::kNAcc) { acc = 0; aphase ^= 1; }
       }
-      __syncwarp();
-      if (++acc == C::kNAcc) { acc = 0; aphase ^= 1; }
     }
+    __syncwarp();
   } else {
     // ------------------------------------------------------------ epilogue
-    const int quarter = warp & 3;  // TMEM lane quarter this warp may access
-    float* tile = sEpi + (warp - kWarpEpi0) * kEpiTileFloats;
+    // tcgen05.ld 16x256b: thread t holds rows (t/4) and (t/4 + 8) of its 16-lane block,
+    // columns 2*(t%4) + {0,1} of every 8-column repetition -> 8-byte stores, four threads
+    // complete a 32-byte sector of a Y row.
+    const int quarter = warp & 3;                        // TMEM lane quarter this warp may access
+    const int half = (warp - kWarpEpi0) >> 2;            // which 16 lanes of the quarter
+    const int lane0 = quarter * 32 + half * 16;          // first TMEM lane of this warp's block
+    const int rlo = lane0 + (lane >> 2), rhi = rlo + 8;  // rows (within the panel) of this thread
+    const int cpair = 2 * (lane & 3);
     int acc = 0;
     uint32_t aphase = 0;
-    const bool vec_ok = ((p.ldy & 3) == 0) && ((((uintptr_t)p.Y) & 15) == 0);
-    const int rsub = lane >> 3;       // row within a 4-row store group
-    const int cq = (lane & 7) * 4;    // column quad within the 32-column slice
-    for (int64_t u = blockIdx.x; u < p.n_units; u += gridDim.x) {
-      const int32_t panel = p.unit_order[u / p.n_ftiles];
+    const bool vec_ok = ((p.ldy & 1) == 0) && ((((uintptr_t)p.Y) & 7) == 0);
+    auto out_row = [&](int4 e, int r) -> int64_t {
+      const int64_t g = (int64_t)e.x * kPanelRows + r;
+      return g < p.rows ? (p.row_map ? (int64_t)__ldg(p.row_map + g) : g) : -1;
+    };
+    int4 nxt = unit_entry(p, blockIdx.x);
+    int64_t nlo = blockIdx.x < p.n_units ? out_row(nxt, rlo) : -1;
+    int64_t nhi = blockIdx.x < p.n_units ? out_row(nxt, rhi) : -1;
+    for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
+      const int4 cur = nxt;
+      const int64_t olo = nlo, ohi = nhi;
+      nxt = unit_entry(p, u + ustep);
+      if (u + ustep < p.n_units) {
+        nlo = out_row(nxt, rlo);
+        nhi = out_row(nxt, rhi);
+      }
       const int ft = (int)(u % p.n_ftiles);
-      const int64_t c0 = p.panel_chunk_ptr[panel], c1 = p.panel_chunk_ptr[panel + 1];
-      // this lane's row (as the TMEM lane owner) and its output row in Y
-      const int64_t myrow = (int64_t)panel * kPanelRows + quarter * 32 + lane;
-      const int64_t myout = myrow < p.rows ? (p.row_map ? (int64_t)p.row_map[myrow] : myrow) : -1;
+      const bool has = cur.y > 0;
       mbar_wait(smem_u32(&tfull[acc]), aphase);
+      NM_TRACE_U(2);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 #pragma unroll 1
-      for (int cc = 0; cc < BN; cc += 32) {
+      for (int cc = 0; cc < BN; cc += 64) {
         uint32_t v[32];
-        if (c1 > c0) {
-          const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + acc * BN + cc;
+        if (has) {
+          const uint32_t taddr = tbase + ((uint32_t)lane0 << 16) + acc * BN + cc;
           asm volatile(
-              "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+              "tcgen05.ld.sync.aligned.16x256b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
               "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
                 "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
@@ -302,31 +368,31 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
 #pragma unroll
           for (int j = 0; j < 32; ++j) v[j] = 0u;
         }
-        const int col = ft * BN + cc;
-        if (col >= p.F || (p.debug & 2)) continue;  // warp-uniform
-        // transpose through shared memory: lane = row -> lanes = 4 rows x 8 column quads
+        if (p.debug & 2) continue;
 #pragma unroll
-        for (int j = 0; j < 32; ++j) tile[lane * 33 + j] = __uint_as_float(v[j]);
-        __syncwarp();
-#pragma unroll
-        for (int g = 0; g < 8; ++g) {
-          const int rr = g * 4 + rsub;
-          const int64_t orow = __shfl_sync(0xffffffffu, myout, rr);
-          const float* tr = tile + rr * 33 + cq;
-          if (orow >= 0) {
-            float* dst = p.Y + orow * p.ldy + col + cq;
-            if (vec_ok && col + cq + 4 <= p.F) {
-              __stcs((float4*)dst, make_float4(tr[0], tr[1], tr[2], tr[3]));
-            } else {
-              for (int e = 0; e < 4; ++e)
-                if (col + cq + e < p.F) dst[e] = tr[e];
+        for (int j = 0; j < 8; ++j) {
+          const int col = ft * BN + cc + 8 * j + cpair;
+          if (col >= p.F) continue;
+          const float2 lo = make_float2(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]));
+          const float2 hi = make_float2(__uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3]));
+          if (vec_ok && col + 2 <= p.F) {
+            if (olo >= 0) __stcs((float2*)(p.Y + olo * p.ldy + col), lo);
+            if (ohi >= 0) __stcs((float2*)(p.Y + ohi * p.ldy + col), hi);
+          } else {
+            if (olo >= 0) {
+              p.Y[olo * p.ldy + col] = lo.x;
+              if (col + 1 < p.F) p.Y[olo * p.ldy + col + 1] = lo.y;
+            }
+            if (ohi >= 0) {
+              p.Y[ohi * p.ldy + col] = hi.x;
+              if (col + 1 < p.F) p.Y[ohi * p.ldy + col + 1] = hi.y;
             }
           }
         }
-        __syncwarp();
       }
       asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
       mbar_arrive(smem_u32(&tempty[acc]));
+      NM_TRACE_U(3);
       if (++acc == C::kNAcc) { acc = 0; aphase ^= 1; }
     }
   }
@@ -364,8 +430,7 @@ nm_status launch_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, 
   NM_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
   SpmmParams prm;
   prm.image = P->image;
-  prm.panel_chunk_ptr = P->panel_chunk_ptr;
-  prm.unit_order = P->unit_order;
+  prm.unit_info = P->unit_info;
   prm.row_map = P->row_map;
   prm.X = (const uint16_t*)PX;
   prm.ldx = ldx;
@@ -378,10 +443,27 @@ nm_status launch_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, 
   prm.idesc = make_idesc(P->dtype, BN);
   const char* dbg = getenv("NM_SPMM_DEBUG");
   prm.debug = dbg ? atoi(dbg) : 0;
+  prm.trace = nullptr;
+  const char* tr = getenv("NM_SPMM_TRACE");
+  if (tr) {
+    NM_CUDA(cudaMalloc(&prm.trace, 16384 * 8));
+    NM_CUDA(cudaMemset(prm.trace, 0, 16384 * 8));
+  }
   int64_t grid = prm.n_units < sms ? prm.n_units : sms;
   if (grid < 1) return NM_OK;
   k_spmm_sptc<BN><<<(unsigned)grid, kThreads, C::kSmem, s>>>(prm);
   NM_CUDA(cudaGetLastError());
+  if (prm.trace) {  // profiling aid only: synchronous dump of CTA 0's timeline
+    NM_CUDA(cudaStreamSynchronize(s));
+    static unsigned long long h[16384];
+    NM_CUDA(cudaMemcpy(h, prm.trace, sizeof(h), cudaMemcpyDeviceToHost));
+    FILE* f = fopen(tr, "wb");
+    if (f) {
+      fwrite(h, sizeof(h), 1, f);
+      fclose(f);
+    }
+    cudaFree(prm.trace);
+  }
   return NM_OK;
 }
 

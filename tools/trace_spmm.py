@@ -1,0 +1,68 @@
+"""Timeline of the SpMM pipeline on CTA 0 (profiling aid, not part of the product).
+
+Runs the bench workload once with NM_SPMM_TRACE set: the kernel records clock64() at the
+hand-off points of its first 1024 chunks / units and this script prints per-chunk latencies:
+  rec   : record producer passes the empty-barrier (stage free) and issues the bulk copy
+  ld    : loader thread 0 sees the record landed (full_a)
+  ldone : loader thread 0 finished issuing gathers + metadata
+  mma   : MMA warp sees the stage ready (full_b)
+"""
+import os
+import sys
+
+import numpy as np
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+
+def main():
+    import torch
+
+    import bench
+    from paper_conf_ppopp_chensz0s25_b200 import api, graphs
+    wl = sys.argv[1] if len(sys.argv) > 1 else bench.DEFAULT
+    w = bench.WORKLOADS[wl]
+    ip, ic, vals, X32 = bench.make_graph(w)
+    perm, _ = api.reorder(ip, ic, w["V"], 2, w["M"])
+    P = api.pack(ip, ic, perm, w["V"], 2, w["M"], dtype=w["dtype"], val=vals, order="original")
+    xb, _ = graphs.round16(X32, w["dtype"])
+    X = torch.from_numpy(xb.view(np.int16)).cuda().view(torch.float16)
+    Y = torch.empty((w["n"], w["F"]), device="cuda")
+    for _ in range(3):
+        api.spmm(P, X, Y, part="sptc")
+    torch.cuda.synchronize()
+    path = "/tmp/nm_trace.bin"
+    os.environ["NM_SPMM_TRACE"] = path
+    api.spmm(P, X, Y, part="sptc")
+    torch.cuda.synchronize()
+    del os.environ["NM_SPMM_TRACE"]
+    t = np.fromfile(path, dtype=np.uint64).astype(np.int64)
+    ch = t[:8192].reshape(1024, 8)[:, :4]
+    un = t[8192:].reshape(2048, 4)
+    n = int((ch[:, 0] > 0).sum())
+    ch = ch[:n]
+    base = ch[0, 0]
+    ch = ch - base
+    print("chunks traced:", n)
+    d_rec_ld = ch[:, 1] - ch[:, 0]
+    d_ld = ch[:, 2] - ch[:, 1]
+    d_ld_mma = ch[:, 3] - ch[:, 2]
+    gap = np.diff(ch[:, 0])
+    for name, v in [("record issue -> loader sees record", d_rec_ld), ("loader issue time", d_ld),
+                    ("loader done -> MMA sees stage", d_ld_mma), ("record issue interval", gap),
+                    ("MMA interval", np.diff(ch[:, 3]))]:
+        print("%-38s median %7d  p10 %7d  p90 %7d cycles" % (name, np.median(v), np.percentile(v, 10),
+                                                             np.percentile(v, 90)))
+    nu = int((un[:, 1] > 0).sum())
+    un = un[:nu] - base
+    print("units traced:", nu)
+    print("unit: mma_start(tempty ok) epi_start(tfull) epi_end")
+    for k in range(min(8, nu)):
+        print(k, un[k, 1], un[k, 2], un[k, 3])
+    print("epilogue duration median", np.median(un[:, 3] - un[:, 2]))
+    print("first 24 chunks (rec, ld, ldone, mma):")
+    print(ch[:24])
+
+
+if __name__ == "__main__":
+    main()
