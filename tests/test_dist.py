@@ -1,0 +1,92 @@
+"""Host-side logic of the row-partitioned multi-GPU path: shard boundaries and
+the all-gather assembly of paper_conf_ppopp_chensz0s25_b200.dist.gcn_forward, run with the
+gloo backend on CPU, world_size 2 (the per-rank SpMM is stood in by the oracle here, so the
+collective/sharding logic is what is tested)."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_ppopp_chensz0s25_b200 import dist as nmdist
+from paper_conf_ppopp_chensz0s25_b200 import graphs
+
+
+@pytest.mark.parametrize("n", [1, 127, 128, 129, 1000, 2048, 5000])
+@pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
+def test_shard_rows_partition(n, world):
+    cuts = [nmdist.shard_rows(n, world, r) for r in range(world)]
+    assert cuts[0][0] == 0 and cuts[-1][1] == n
+    for (a, b), (c, d) in zip(cuts[:-1], cuts[1:]):
+        assert b == c
+    for a, b in cuts:
+        assert (a % 128 == 0 or a == n) and a <= b  # empty trailing shards start at n
+        assert b - a <= nmdist.padded_rows(n, world)
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _problem():
+    n, f0, f1, f2 = 700, 16, 12, 8
+    ip, ic = graphs.er_graph(n, 3000, 5, self_loops=True)
+    vals = graphs.symmetric_values(ip, ic, 6).astype(np.float64)
+    rng = np.random.default_rng(0)
+    H = rng.standard_normal((n, f0))
+    Ws = [rng.standard_normal((f0, f1)), rng.standard_normal((f1, f2))]
+    bs = [rng.standard_normal(f1), rng.standard_normal(f2)]
+    return ip, ic, vals, H, Ws, bs
+
+
+def _local_layer_factory(ip, ic, vals):
+    import oracle
+
+    def local_layer(l, Hf, W, b, relu, rb, re):
+        XW = Hf.numpy() @ W
+        sub_ip = ip[rb:re + 1] - ip[rb]
+        Y, _, _ = oracle.spmm(sub_ip, ic[ip[rb]:ip[re]], vals[ip[rb]:ip[re]], XW)
+        Y = Y + b
+        if relu:
+            Y = np.maximum(Y, 0.0)
+        return torch.from_numpy(Y)
+
+    return local_layer
+
+
+def _worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    ip, ic, vals, H, Ws, bs = _problem()
+    layers = [(Ws[0], bs[0], True), (Ws[1], bs[1], False)]
+    out = nmdist.gcn_forward(torch.from_numpy(H), layers, _local_layer_factory(ip, ic, vals))
+    q.put((rank, out.numpy()))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_gcn_forward_gloo_world2_matches_single_process():
+    ip, ic, vals, H, Ws, bs = _problem()
+    layers = [(Ws[0], bs[0], True), (Ws[1], bs[1], False)]
+    ref = nmdist.gcn_forward(torch.from_numpy(H), layers, _local_layer_factory(ip, ic, vals)).numpy()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    got = dict(q.get(timeout=120) for _ in range(2))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for r in range(2):
+        assert got[r].shape == ref.shape
+        np.testing.assert_allclose(got[r], ref, rtol=1e-12, atol=1e-12)

@@ -1,0 +1,67 @@
+"""GPU parity of nm_gcn_layer (Eq. 1: H' = ReLU(Ahat (H W) + b), linear first
+as GCN does, L564).  The aggregation is checked against the oracle's fp64 SpMM applied to the
+exact bf16 operand H W the GPU consumed (read back from the layer's workspace):
+|H' - relu(Ahat XW + b)| <= 1e-3 * (|Ahat| |XW|) + one bf16 rounding of the output."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_ppopp_chensz0s25_b200 import api, graphs
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+
+def _gcn_norm(ip, ic):
+    """Ahat = D^-1/2 (A + I) D^-1/2 on a graph that already contains its self-loops."""
+    n = len(ip) - 1
+    deg = np.diff(ip).astype(np.float64)
+    rows = np.repeat(np.arange(n), np.diff(ip))
+    return (1.0 / np.sqrt(deg[rows] * deg[ic])).astype(np.float32)
+
+
+@pytest.mark.parametrize("n,fin,fout,V,M", [(2048, 64, 32, 1, 4), (3000, 128, 64, 8, 8), (1500, 96, 128, 1, 4)])
+@pytest.mark.parametrize("relu", [True, False])
+def test_gcn_layer(n, fin, fout, V, M, relu):
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    dev = torch.device("cuda:0")
+    ip, ic = graphs.er_graph(n, 6 * n, 3, self_loops=True)
+    vals = _gcn_norm(ip, ic)
+    vbits, v64 = graphs.round16(vals, "bf16")
+    perm, _ = api.reorder(ip, ic, V, 2, M)
+    P = api.pack(ip, ic, perm, V, 2, M, dtype="bf16", val=vals)
+    rng = np.random.default_rng(1)
+    H32 = rng.standard_normal((n, fin)).astype(np.float32)
+    W32 = (rng.standard_normal((fin, fout)) / np.sqrt(fin)).astype(np.float32)
+    b = rng.standard_normal(fout).astype(np.float32)
+    hb, _ = graphs.round16(H32, "bf16")
+    wb, _ = graphs.round16(W32, "bf16")
+    H = torch.from_numpy(hb.view(np.int16)).to(dev).view(torch.bfloat16)
+    W = torch.from_numpy(wb.view(np.int16)).to(dev).view(torch.bfloat16)
+    pd = torch.from_numpy(perm).to(dev)
+    PH = torch.empty_like(H)
+    api.permute_rows(H, PH, pd, "bf16")
+    ws = torch.empty(api.gcn_workspace_bytes(n, fout), dtype=torch.uint8, device=dev)
+    Hout_p = torch.empty((n, fout), dtype=torch.bfloat16, device=dev)
+    bias = torch.from_numpy(b).to(dev)
+    api.gcn_layer(P, PH, W, bias, Hout_p, ws, relu=relu)
+    torch.cuda.synchronize()
+    # the bf16 XW the aggregation consumed (permuted order), from the workspace
+    xw_bits = ws[: n * fout * 2].view(torch.int16).cpu().numpy().view(np.uint16).reshape(n, fout)
+    xw_p = graphs.bf16_bits_to_f64(xw_bits)
+    # sanity: XW is H W (permuted) up to bf16 rounding of a fp32-accumulated GEMM
+    ref_xw = (graphs.bf16_bits_to_f64(hb) @ graphs.bf16_bits_to_f64(wb))[perm]
+    assert np.abs(xw_p - ref_xw).max() <= 1e-2 * np.abs(ref_xw).max()
+    xw = np.empty_like(xw_p)
+    xw[perm] = xw_p  # back to the original order
+    Y, E, _ = oracle.spmm(ip, ic, v64, xw)
+    ref = Y + b
+    if relu:
+        ref = np.maximum(ref, 0.0)
+    Hout = torch.empty_like(Hout_p)
+    api.unpermute_rows(Hout_p, Hout, pd, "bf16")
+    torch.cuda.synchronize()
+    got = graphs.bf16_bits_to_f64(Hout.view(torch.int16).cpu().numpy().view(np.uint16))
+    bound = 1e-3 * E + 2.0 ** -8 * np.abs(ref) + 1e-30
+    assert (np.abs(got - ref) <= bound).all(), np.abs(got - ref).max()
