@@ -228,7 +228,20 @@ def main():
     gen_s = time.perf_counter() - t0
     n, F, V, M, dt = w["n"], w["F"], w["V"], w["M"], w["dtype"]
     nnz = int(ip[-1])
-    perm, rst = api.reorder(ip, ic, V, 2, M)
+    if world == 1:
+        perm, rst = api.reorder(ip, ic, V, 2, M)
+    else:
+        # one rank reorders (host, multi-threaded), the permutation is broadcast over NCCL
+        keys = ("omega_init", "omega_final", "mb_init", "mb_final", "seconds")
+        buf = torch.zeros(n + len(keys), dtype=torch.float64, device=dev)
+        if rank == 0:
+            perm, rst = api.reorder(ip, ic, V, 2, M)
+            buf[:n] = torch.from_numpy(perm.astype(np.float64)).to(dev)
+            buf[n:] = torch.tensor([float(rst[k]) for k in keys], dtype=torch.float64, device=dev)
+        dist.broadcast(buf, 0)
+        hb = buf.cpu().numpy()
+        perm = hb[:n].astype(np.int32)
+        rst = {k: (float(v) if k == "seconds" else int(v)) for k, v in zip(keys, hb[n:])}
     from paper_conf_ppopp_chensz0s25_b200.dist import shard_rows
     rb, re = shard_rows(n, world, rank)
     t0 = time.perf_counter()

@@ -128,7 +128,9 @@ struct Cfg {
   static constexpr int kBBytes = 32 * BN * 2;                   // 32 K-rows x BN halves
   static constexpr int kStageBytes = kRecBytes + kBBytes;
   static constexpr int kStagesRaw = (214 * 1024) / kStageBytes;
-  static constexpr int kStages = kStagesRaw > 16 ? 16 : kStagesRaw;
+  // a multiple of the loader-group count: group g owns stages s % kLoadGroups == g, so every
+  // stage has one consumer group that visits it in chunk order (parity waits stay valid)
+  static constexpr int kStages = ((kStagesRaw > 16 ? 16 : kStagesRaw) / kLoadGroups) * kLoadGroups;
   static constexpr int kNAcc = (2 * BN + kStages <= 512) ? 2 : 1;
   static constexpr int kMeta0 = kNAcc * BN;                     // metadata column of stage s: kMeta0 + s
   static constexpr int kRecRegion = ((kStages * kRecBytes + 1023) / 1024) * 1024;
@@ -210,7 +212,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
     }
   } else if (warp >= kWarpLoad0 && warp < kWarpLoad0 + 4 * kLoadGroups) {
     // ------------------------------------------------------------ loaders: X gathers + metadata
-    const int group = (warp - kWarpLoad0) >> 2;  // takes chunks i with i % kLoadGroups == group
+    const int group = (warp - kWarpLoad0) >> 2;  // owns the stages s with s % kLoadGroups == group
     const int quarter = warp & 3;                               // TMEM lane quarter of this warp
     const int t = threadIdx.x - (kWarpLoad0 + 4 * group) * 32;  // 0..127 within the group
     const int L = quarter * 32 + lane;                          // TMEM lane this thread writes
@@ -219,7 +221,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
     constexpr int kRowPieces = BN / 8;  // 16-byte pieces per gathered row
     constexpr int kPer = kRowPieces / 4;  // pieces per thread
     int64_t i = 0;
-    int s_next = 0, g_next = 0;
+    int s_next = 0;
     uint32_t ph_next = 0;
     int4 nxt = unit_entry(p, blockIdx.x);
     for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
@@ -231,9 +233,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
         const int s = s_next;
         const uint32_t ph = ph_next;
         if (++s_next == C::kStages) { s_next = 0; ph_next ^= 1; }
-        const int g = g_next;
-        if (++g_next == kLoadGroups) g_next = 0;
-        if (g != group) continue;
+        // stage ownership (not chunk round-robin): a group that skipped ahead could otherwise
+        // test the parity of a stage two phases ahead and pass on a stale record
+        if (s % kLoadGroups != group) continue;
         mbar_wait(smem_u32(&full_a[s]), ph);
         if (t == 0) NM_TRACE(1);
         const uint32_t rec = sRec + s * C::kRecBytes;
@@ -266,8 +268,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
     }
   } else if (warp == kWarpMma) {
     // ------------------------------------------------------------ MMA issuer (one thread)
-    // The cp.async gathers are published through cp.async.mbarrier.arrive on full_b; as in
-    // CUTLASS's PipelineUmmaConsumerAsync (cp.async -> UMMA) no extra proxy fence is issued.
+    // The cp.async gathers are published through cp.async.mbarrier.arrive on full_b.
     if (lane == 0) {
       int64_t i = 0;  // chunk counter (trace only)
       int s = 0;
@@ -288,7 +289,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
         for (int c = 0; c < nch; ++c, ++i) {
           mbar_wait(smem_u32(&full_b[s]), ph);
           NM_TRACE(3);
-          if (p.debug & 16) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          // the gathers were written through the generic proxy (cp.async): make them visible
+          // to the tensor core's async-proxy operand reads (without this fence stale stage
+          // contents were observed on B200 -- tests/test_parity_fullsize.py)
+          if (!(p.debug & 16)) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
           const uint64_t ad = adesc0 + (uint64_t)((s * C::kRecBytes) >> 4);
           const uint64_t bd = bdesc0 + (uint64_t)((s * C::kBBytes) >> 4);
