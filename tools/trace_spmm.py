@@ -53,8 +53,13 @@ def main():
                     ("MMA interval", np.diff(ch[:, 3]))]:
         print("%-38s median %7d  p10 %7d  p90 %7d cycles" % (name, np.median(v), np.percentile(v, 10),
                                                              np.percentile(v, 90)))
+    mi = np.diff(ch[:, 3])
+    print("MMA interval mean %.0f; share of time in gaps > 1000 cycles: %.2f" %
+          (mi.mean(), mi[mi > 1000].sum() / mi.sum()))
     nu = int((un[:, 1] > 0).sum())
     un = un[:nu] - base
+    # unit boundary cost: MMA start of unit k+1 minus the MMA time of unit k's last chunk
+    print("epilogue start - MMA start (median): %.0f" % np.median(un[:, 2] - un[:, 1]))
     print("units traced:", nu)
     print("unit: mma_start(tempty ok) epi_start(tfull) epi_end")
     for k in range(min(8, nu)):
