@@ -101,6 +101,14 @@ typedef struct {
 NM_API nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
                      int32_t* perm_out, nm_reorder_stats* st);
 
+/* nm_select_pattern -- the paper's best-V:N:M search (§5): reorder for 1:2:M
+ * with M = 4, 8, ... (<= max_M) while the reordered graph conforms (omega = MBscore = 0),
+ * then for V:2:M with V = 2, 4, ... (<= max_V, "V going from 1 to 32 in a similar manner")
+ * while it conforms.  Returns the last conforming pattern (1:2:4 if none conforms) in
+ * *V_out / *M_out, its order in perm_out (host int32[n]) and its statistics.  Synchronous. */
+NM_API nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, const nm_reorder_opts* opts,
+                                   int32_t* perm_out, int* V_out, int* M_out, nm_reorder_stats* st);
+
 /* nm_count_violations -- omega (L203), MBscore (L382) and optionally PScore per segment
  * (L396) of B = P A P^T, computed on the GPU.  perm: host int32[n] or NULL (identity).
  * pscore: host int32[ceil(n/M)] or NULL.  Synchronous. */

@@ -147,6 +147,36 @@ def reorder(indptr, indices, V: int, N: int, M: int, max_outer: int = 10, max_st
     return perm[:n], stats
 
 
+def select_pattern(indptr, indices, max_M=32, max_V=32, **kw):
+    """Best-V:N:M search, step by step as PAPER.md:L496 (§5) describes it: try 1:2:M with M
+    initialised to 4 and doubled while the graph can be reordered to conform; then fix M and
+    try V:2:M with V doubling from 1 up to max_V in the same way.  Returns (V, M, perm, stats)
+    of the last conforming pattern (1:2:4 when even that does not conform)."""
+    def conforms(st):
+        return st["omega_final"] == 0 and st["mb_final"] == 0
+
+    perm, st = reorder(indptr, indices, 1, 2, 4, **kw)
+    best = (1, 4, perm, st)
+    if not conforms(st):
+        return best
+    M = 8
+    while M <= max_M:
+        p, s = reorder(indptr, indices, 1, 2, M, **kw)
+        if not conforms(s):
+            break
+        best = (1, M, p, s)
+        M *= 2
+    bestM = best[1]
+    V = 2
+    while V <= max_V:
+        p, s = reorder(indptr, indices, V, 2, bestM, **kw)
+        if not conforms(s):
+            break
+        best = (V, bestM, p, s)
+        V *= 2
+    return best
+
+
 def stage1_once(indptr, indices, perm, N: int, M: int):
     """One Stage-1 sort (Alg. 2 lines 4-13) starting from perm; returns the new perm."""
     rp, ci, n = _csr(indptr, indices)

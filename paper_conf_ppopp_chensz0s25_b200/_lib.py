@@ -49,6 +49,10 @@ SIGNATURES = {
     "nm_reorder": (ctypes.c_int, [ctypes.POINTER(nm_csr), ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                   ctypes.POINTER(nm_reorder_opts), P32,
                                   ctypes.POINTER(nm_reorder_stats)]),
+    "nm_select_pattern": (ctypes.c_int, [ctypes.POINTER(nm_csr), ctypes.c_int, ctypes.c_int,
+                                         ctypes.POINTER(nm_reorder_opts), P32,
+                                         ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.c_int),
+                                         ctypes.POINTER(nm_reorder_stats)]),
     "nm_count_violations": (ctypes.c_int, [ctypes.POINTER(nm_csr), P32, ctypes.c_int, ctypes.c_int,
                                            ctypes.c_int, P64, P64, P32]),
     "nm_pack": (ctypes.c_int, [ctypes.POINTER(nm_csr), P32, ctypes.c_int, ctypes.c_int, ctypes.c_int,

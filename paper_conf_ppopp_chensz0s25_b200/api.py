@@ -60,6 +60,22 @@ def reorder(indptr, indices, V: int, N: int, M: int, max_outer=10, max_stage1=10
     return perm, {f: getattr(st, f) for f, _ in L.nm_reorder_stats._fields_}
 
 
+def select_pattern(indptr, indices, max_M=32, max_V=32, max_outer=10, max_stage1=10, max_stage2=10,
+                   gain_rule=0, keep_best=1):
+    """nm_select_pattern: returns (V, M, perm, stats) of the best conforming
+    V:2:M pattern found by the paper's doubling search."""
+    c, keep = _csr_struct(indptr, indices)
+    perm = np.zeros(c.n, np.int32)
+    o = L.nm_reorder_opts(max_outer, max_stage1, max_stage2, gain_rule, keep_best)
+    st = L.nm_reorder_stats()
+    V = ctypes.c_int()
+    M = ctypes.c_int()
+    L.check(L.load().nm_select_pattern(ctypes.byref(c), max_M, max_V, ctypes.byref(o),
+                                       perm.ctypes.data_as(L.P32), ctypes.byref(V), ctypes.byref(M),
+                                       ctypes.byref(st)), "nm_select_pattern")
+    return V.value, M.value, perm, {f: getattr(st, f) for f, _ in L.nm_reorder_stats._fields_}
+
+
 def count_violations(indptr, indices, perm, V: int, N: int, M: int):
     """nm_count_violations (GPU): returns (omega, mbscore, pscore int32[ceil(n/M)])."""
     c, keep = _csr_struct(indptr, indices)

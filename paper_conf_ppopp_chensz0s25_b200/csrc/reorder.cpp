@@ -333,26 +333,13 @@ int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>&
 
 using namespace nm;
 
-extern "C" nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
-                                int32_t* perm_out, nm_reorder_stats* st) {
-  if (!A || !perm_out) return fail(NM_ERR_INVALID_ARG, "nm_reorder: NULL argument");
-  if (V < 1 || N < 1 || M <= N) return fail(NM_ERR_INVALID_ARG, "nm_reorder: need V >= 1, 1 <= N < M");
-  if (M > 32) return fail(NM_ERR_UNSUPPORTED, "nm_reorder: M > 32");
-  if (A->n <= 0) return fail(NM_ERR_INVALID_ARG, "nm_reorder: empty graph");
-  if (A->n >= ((int64_t)1 << 31)) return fail(NM_ERR_UNSUPPORTED, "nm_reorder: n >= 2^31");
-  nm_reorder_opts o = {10, 10, 10, 0, 1};
-  if (opts) o = *opts;
+namespace nm {
+namespace {
+
+// Alg. 1 on a validated host graph: perm_out receives the (keep-best) order.
+void reorder_core(const Graph& g, int V, int N, int M, const nm_reorder_opts& o, int32_t* perm_out,
+                  nm_reorder_stats* st) {
   auto t0 = std::chrono::steady_clock::now();
-  int64_t* rp = nullptr;
-  int32_t* ci = nullptr;
-  nm_status s = host_csr(A, &rp, &ci);
-  if (s != NM_OK) { free(rp); free(ci); return s; }
-  s = validate_csr_host(A->n, rp, ci, true);
-  if (s != NM_OK) { free(rp); free(ci); return s; }
-  Graph g;
-  g.n = A->n;
-  g.rp = rp;
-  g.ci = ci;
   const int64_t n = g.n;
   std::vector<int32_t> perm(n), iperm(n), best;
   std::iota(perm.begin(), perm.end(), 0);
@@ -390,7 +377,87 @@ extern "C" nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_r
   stats.mb_final = mbscore(g, res, iperm, V, M);
   stats.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
   if (st) *st = stats;
-  free(rp);
-  free(ci);
+}
+
+struct HostGraph {
+  int64_t* rp = nullptr;
+  int32_t* ci = nullptr;
+  Graph g;
+  ~HostGraph() { free(rp); free(ci); }
+  nm_status load(const nm_csr* A) {
+    nm_status s = host_csr(A, &rp, &ci);
+    if (s != NM_OK) return s;
+    s = validate_csr_host(A->n, rp, ci, true);
+    if (s != NM_OK) return s;
+    g.n = A->n;
+    g.rp = rp;
+    g.ci = ci;
+    return NM_OK;
+  }
+};
+
+nm_status check_graph_arg(const nm_csr* A) {
+  if (A->n <= 0) return fail(NM_ERR_INVALID_ARG, "empty graph");
+  if (A->n >= ((int64_t)1 << 31)) return fail(NM_ERR_UNSUPPORTED, "n >= 2^31");
+  return NM_OK;
+}
+
+}  // namespace
+}  // namespace nm
+
+extern "C" nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
+                                int32_t* perm_out, nm_reorder_stats* st) {
+  if (!A || !perm_out) return fail(NM_ERR_INVALID_ARG, "nm_reorder: NULL argument");
+  if (V < 1 || N < 1 || M <= N) return fail(NM_ERR_INVALID_ARG, "nm_reorder: need V >= 1, 1 <= N < M");
+  if (M > 32) return fail(NM_ERR_UNSUPPORTED, "nm_reorder: M > 32");
+  nm_status s = check_graph_arg(A);
+  if (s != NM_OK) return s;
+  nm_reorder_opts o = {10, 10, 10, 0, 1};
+  if (opts) o = *opts;
+  HostGraph hg;
+  s = hg.load(A);
+  if (s != NM_OK) return s;
+  reorder_core(hg.g, V, N, M, o, perm_out, st);
+  return NM_OK;
+}
+
+extern "C" nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, const nm_reorder_opts* opts,
+                                       int32_t* perm_out, int* V_out, int* M_out, nm_reorder_stats* st) {
+  if (!A || !perm_out || !V_out || !M_out) return fail(NM_ERR_INVALID_ARG, "nm_select_pattern: NULL argument");
+  if (max_M < 4 || max_M > 32 || max_V < 1) return fail(NM_ERR_INVALID_ARG, "nm_select_pattern: need 4 <= max_M <= 32, max_V >= 1");
+  nm_status s = check_graph_arg(A);
+  if (s != NM_OK) return s;
+  nm_reorder_opts o = {10, 10, 10, 0, 1};
+  if (opts) o = *opts;
+  HostGraph hg;
+  s = hg.load(A);
+  if (s != NM_OK) return s;
+  const int64_t n = hg.g.n;
+  std::vector<int32_t> cand(n);
+  nm_reorder_stats cst;
+  // 1:2:M with M = 4, 8, ... while the graph can be reordered to conform ...
+  int bestV = 1, bestM = 4;
+  nm_reorder_stats first;
+  reorder_core(hg.g, 1, 2, 4, o, perm_out, &first);
+  if (st) *st = first;
+  if (first.omega_final == 0 && first.mb_final == 0) {
+    for (int M = 8; M <= max_M; M *= 2) {
+      reorder_core(hg.g, 1, 2, M, o, cand.data(), &cst);
+      if (cst.omega_final != 0 || cst.mb_final != 0) break;
+      bestM = M;
+      memcpy(perm_out, cand.data(), sizeof(int32_t) * n);
+      if (st) *st = cst;
+    }
+    // ... then V:2:M with V = 2, 4, ..., max_V "in a similar manner" (doubling)
+    for (int V = 2; V <= max_V; V *= 2) {
+      reorder_core(hg.g, V, 2, bestM, o, cand.data(), &cst);
+      if (cst.omega_final != 0 || cst.mb_final != 0) break;
+      bestV = V;
+      memcpy(perm_out, cand.data(), sizeof(int32_t) * n);
+      if (st) *st = cst;
+    }
+  }
+  *V_out = bestV;
+  *M_out = bestM;
   return NM_OK;
 }

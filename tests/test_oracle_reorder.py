@@ -143,3 +143,27 @@ def test_banded_violations_fixed_substantially():
     perm, st = oracle.reorder(indptr, indices, 1, 2, 4, gain_rule=0)
     assert st["omega_init"] > 0
     assert st["omega_final"] < st["omega_init"]
+
+
+def test_select_pattern_closed_forms():
+    """PAPER.md:L496 search.  Self-loops only: every row has one nonzero (any M conforms) but a
+    diagonal V x M block has min(V, M) distinct columns and no permutation moves the diagonal,
+    so V stops at 4 (k = 4): expected (V, M) = (4, 32).  No edges at all: (32, 32)."""
+    n = 256
+    ip = np.arange(n + 1, dtype=np.int64)
+    ic = np.arange(n, dtype=np.int32)
+    V, M, perm, st = oracle.select_pattern(ip, ic, max_M=32, max_V=32)
+    assert (V, M) == (4, 32) and st["omega_final"] == 0 and st["mb_final"] == 0
+    ip0 = np.zeros(n + 1, dtype=np.int64)
+    V, M, perm, st = oracle.select_pattern(ip0, np.zeros(0, np.int32), max_M=32, max_V=32)
+    assert (V, M) == (32, 32)
+
+
+def test_select_pattern_returns_conforming_or_fallback():
+    for seed in range(4):
+        ip, ic = graphs.banded_graph(300, 4, 40 + seed)
+        V, M, perm, st = oracle.select_pattern(ip, ic, max_M=16, max_V=8)
+        w, mb, _ = oracle.counts(ip, ic, perm, V, 2, M)
+        assert (w, mb) == (st["omega_final"], st["mb_final"])
+        if (V, M) != (1, 4):
+            assert w == 0 and mb == 0

@@ -55,3 +55,23 @@ def test_sweep_shapes_small(kind, V, M):
 def test_literal_mode_and_caps():
     ip, ic = graphs.banded_graph(700, 12, 5)
     _check(ip, ic, 4, 2, 8, keep_best=0, max_outer=2, max_stage1=1, max_stage2=3)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_select_pattern_parity(seed):
+    if seed % 2:
+        ip, ic = graphs.banded_graph(400, 4, 60 + seed)
+    else:
+        ip, ic = graphs.er_graph(300, 500, 60 + seed)
+    Vo, Mo, po, so = oracle.select_pattern(ip, ic, max_M=16, max_V=16)
+    Vg, Mg, pg, sg = api.select_pattern(ip, ic, max_M=16, max_V=16)
+    assert (Vo, Mo) == (Vg, Mg)
+    assert np.array_equal(po, pg)
+    assert so["omega_final"] == sg["omega_final"] and so["mb_final"] == sg["mb_final"]
+
+
+def test_select_pattern_self_loops():
+    n = 256
+    ip = np.arange(n + 1, dtype=np.int64)
+    ic = np.arange(n, dtype=np.int32)
+    assert api.select_pattern(ip, ic)[:2] == (4, 32)
