@@ -203,16 +203,23 @@ NM_API nm_status nm_spmm_residual(const nm_packed* P, const void* PX, int64_t ld
                            int64_t ldy, int F, void* stream);
 
 /* ---------------------------------------------------------------------------------------
- * nm_gcn_layer -- one GCN layer (Eq. 1): Hout = act(Ahat (H W) + bias), linear first
- * (GCN "aggregates after its linear layer", L564).  Ahat: packed normalised adjacency in
- * permuted order (P Ahat P^T), H: device [rows(Ahat.n) x F_in] dtype of the pack (permuted
- * order), W: device [F_in x F_out] same dtype, row-major; bias: device fp32[F_out] or NULL;
- * Hout: device [rows x F_out] same dtype.  flags: NM_RELU.  ws: device workspace of at
- * least nm_gcn_workspace_bytes(...) bytes.  The dense H W runs on cuBLASLt (a plain
- * library GEMM); the aggregation on nm_spmm.
+ * nm_gcn_layer -- one GCN layer (Eq. 1): Hout = act(Ahat (H W) + bias).
+ *   Ahat : packed normalised adjacency in permuted order (P Ahat P^T, pack flags 0), rows
+ *          [row_begin, row_end) of it (a row shard for multi-GPU runs);
+ *   H    : device [n x F_in] (all vertices, permuted order), dtype of the pack, ld = F_in;
+ *   W    : device [F_in x F_out] same dtype, row-major;  bias: device fp32[F_out] or NULL;
+ *   Hout : device [(row_end-row_begin) x F_out] same dtype (the shard's rows).
+ *   flags: NM_RELU; order NM_LINEAR_FIRST (default, GCN "aggregates after its linear layer",
+ *          L564) / NM_AGG_FIRST / NM_ORDER_AUTO (aggregate first iff F_out > F_in).
+ *   ws   : device workspace of at least nm_gcn_workspace_bytes(n, F_in, F_out) bytes.
+ * F_in and F_out must be multiples of 8.  The dense products run on cuBLASLt (plain library
+ * GEMMs, fp32 accumulation); the aggregation on nm_spmm.  Stream-ordered.
  * ------------------------------------------------------------------------------------- */
 #define NM_RELU 1
-NM_API size_t nm_gcn_workspace_bytes(int64_t n, int F_out);
+#define NM_LINEAR_FIRST 0
+#define NM_AGG_FIRST 2
+#define NM_ORDER_AUTO 4
+NM_API size_t nm_gcn_workspace_bytes(int64_t n, int F_in, int F_out);
 NM_API nm_status nm_gcn_layer(const nm_packed* Ahat, const void* H, const void* W, const float* bias,
                        void* Hout, int F_in, int F_out, int flags, void* ws, size_t ws_bytes,
                        void* stream);

@@ -16,6 +16,7 @@ NM_OK, NM_ERR_INVALID_ARG, NM_ERR_UNSUPPORTED, NM_ERR_BAD_CSR, NM_ERR_NOT_SYMMET
     NM_ERR_CUDA, NM_ERR_OOM = range(7)
 NM_F16, NM_BF16, NM_F32 = 0, 1, 2
 NM_RELU = 1
+NM_LINEAR_FIRST, NM_AGG_FIRST, NM_ORDER_AUTO = 0, 2, 4
 NM_PACK_ORIGINAL_ORDER = 1
 
 P64 = ctypes.POINTER(ctypes.c_int64)
@@ -74,7 +75,7 @@ SIGNATURES = {
     "nm_spmm_sptc": (ctypes.c_int, [VP, VP, ctypes.c_int64, VP, ctypes.c_int64, ctypes.c_int, VP]),
     "nm_spmm_residual": (ctypes.c_int, [VP, VP, ctypes.c_int64, VP, ctypes.c_int64, ctypes.c_int,
                                         VP]),
-    "nm_gcn_workspace_bytes": (ctypes.c_size_t, [ctypes.c_int64, ctypes.c_int]),
+    "nm_gcn_workspace_bytes": (ctypes.c_size_t, [ctypes.c_int64, ctypes.c_int, ctypes.c_int]),
     "nm_gcn_layer": (ctypes.c_int, [VP, VP, VP, VP, VP, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                     VP, ctypes.c_size_t, VP]),
     "nm_status_string": (ctypes.c_char_p, [ctypes.c_int]),

@@ -197,11 +197,17 @@ def unpermute_rows(Yp, Y, perm_dev, dtype, stream=None):
             "nm_unpermute_rows")
 
 
-def gcn_workspace_bytes(n, F_out):
-    return int(L.load().nm_gcn_workspace_bytes(n, F_out))
+def gcn_workspace_bytes(n, F_in, F_out):
+    return int(L.load().nm_gcn_workspace_bytes(n, F_in, F_out))
 
 
-def gcn_layer(P: Packed, H, W, bias, Hout, ws, relu=True, stream=None):
+_ORDERS = {"linear": L.NM_LINEAR_FIRST, "aggregate": L.NM_AGG_FIRST, "auto": L.NM_ORDER_AUTO}
+
+
+def gcn_layer(P: Packed, H, W, bias, Hout, ws, relu=True, order="linear", stream=None):
+    """nm_gcn_layer: Hout (rows of P) = act(Ahat (H W) + bias); order 'linear' | 'aggregate' |
+    'auto'."""
+    flags = (L.NM_RELU if relu else 0) | _ORDERS[order]
     L.check(L.load().nm_gcn_layer(P.handle, _ptr(H), _ptr(W), _ptr(bias), _ptr(Hout), H.shape[1],
-                                  W.shape[1], L.NM_RELU if relu else 0, _ptr(ws), ws.numel(),
-                                  _stream_ptr(stream)), "nm_gcn_layer")
+                                  W.shape[1], flags, _ptr(ws), ws.numel(), _stream_ptr(stream)),
+            "nm_gcn_layer")

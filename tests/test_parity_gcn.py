@@ -42,7 +42,7 @@ def test_gcn_layer(n, fin, fout, V, M, relu):
     pd = torch.from_numpy(perm).to(dev)
     PH = torch.empty_like(H)
     api.permute_rows(H, PH, pd, "bf16")
-    ws = torch.empty(api.gcn_workspace_bytes(n, fout), dtype=torch.uint8, device=dev)
+    ws = torch.empty(api.gcn_workspace_bytes(n, fin, fout), dtype=torch.uint8, device=dev)
     Hout_p = torch.empty((n, fout), dtype=torch.bfloat16, device=dev)
     bias = torch.from_numpy(b).to(dev)
     api.gcn_layer(P, PH, W, bias, Hout_p, ws, relu=relu)
@@ -64,4 +64,46 @@ def test_gcn_layer(n, fin, fout, V, M, relu):
     torch.cuda.synchronize()
     got = graphs.bf16_bits_to_f64(Hout.view(torch.int16).cpu().numpy().view(np.uint16))
     bound = 1e-3 * E + 2.0 ** -8 * np.abs(ref) + 1e-30
+    assert (np.abs(got - ref) <= bound).all(), np.abs(got - ref).max()
+
+
+@pytest.mark.parametrize("n,fin,fout,V,M,shards", [(2048, 32, 64, 1, 4, 1), (3000, 104, 256, 128, 8, 3),
+                                                   (1500, 64, 64, 1, 4, 2)])
+def test_gcn_layer_aggregate_first_and_row_shards(n, fin, fout, V, M, shards):
+    """Aggregate-first order (ogbn-products shape, F 100(->104) -> 256, 128:2:8) and
+    panel-aligned row shards (nm_pack_rows) whose outputs tile the full result.
+    Bound: SpMM 1e-3*(|Ahat||H|)|W| + bf16 rounding of Ahat H (2^-9 relative) propagated through
+    W + bf16 rounding of the output (2^-8 relative)."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ppopp_chensz0s25_b200.dist import shard_rows
+    dev = torch.device("cuda:0")
+    ip, ic = graphs.er_graph(n, 5 * n, 4, self_loops=True)
+    vals = _gcn_norm(ip, ic)
+    _, v64 = graphs.round16(vals, "bf16")
+    perm, _ = api.reorder(ip, ic, V, 2, M)
+    rng = np.random.default_rng(2)
+    hb, h64 = graphs.round16(rng.standard_normal((n, fin)).astype(np.float32), "bf16")
+    wb, w64 = graphs.round16((rng.standard_normal((fin, fout)) / np.sqrt(fin)).astype(np.float32), "bf16")
+    b = rng.standard_normal(fout).astype(np.float32)
+    H = torch.from_numpy(hb.view(np.int16)).to(dev).view(torch.bfloat16)
+    W = torch.from_numpy(wb.view(np.int16)).to(dev).view(torch.bfloat16)
+    pd = torch.from_numpy(perm).to(dev)
+    PH = torch.empty_like(H)
+    api.permute_rows(H, PH, pd, "bf16")
+    bias = torch.from_numpy(b).to(dev)
+    ws = torch.empty(api.gcn_workspace_bytes(n, fin, fout), dtype=torch.uint8, device=dev)
+    Hout_p = torch.empty((n, fout), dtype=torch.bfloat16, device=dev)
+    for r in range(shards):
+        rb, re = shard_rows(n, shards, r)
+        P = api.pack(ip, ic, perm, V, 2, M, dtype="bf16", val=vals, row_begin=rb, row_end=re)
+        api.gcn_layer(P, PH, W, bias, Hout_p[rb:re], ws, relu=True, order="aggregate")
+        torch.cuda.synchronize()
+    Hout = torch.empty_like(Hout_p)
+    api.unpermute_rows(Hout_p, Hout, pd, "bf16")
+    torch.cuda.synchronize()
+    got = graphs.bf16_bits_to_f64(Hout.view(torch.int16).cpu().numpy().view(np.uint16))
+    Ya, Ea, _ = oracle.spmm(ip, ic, v64, h64)
+    ref = np.maximum(Ya @ w64 + b, 0.0)
+    bound = 3e-3 * (Ea @ np.abs(w64)) + 2.0 ** -8 * np.abs(ref) + 1e-30
     assert (np.abs(got - ref) <= bound).all(), np.abs(got - ref).max()
