@@ -76,10 +76,10 @@ def _lib():
                                  ctypes.POINTER(_Stats)]
         L.or_pack_count.restype = ctypes.c_int
         L.or_pack_count.argtypes = [ctypes.c_int64, P64, P32, P32, ctypes.c_int, ctypes.c_int,
-                                    P64, P64]
+                                    ctypes.c_int, P64, P64]
         L.or_pack_fill.restype = ctypes.c_int
         L.or_pack_fill.argtypes = [ctypes.c_int64, P64, P32, PU16, ctypes.c_uint16, P32,
-                                   ctypes.c_int, ctypes.c_int, P64, P64, P64, P32, PU8, PU8,
+                                   ctypes.c_int, ctypes.c_int, ctypes.c_int, P64, P64, P64, P32, PU8, PU8,
                                    PU16, P64, P32, PU16]
         L.or_spmm_f64.restype = ctypes.c_int
         L.or_spmm_f64.argtypes = [ctypes.c_int64, P64, P32, PF64, PF64, ctypes.c_int64,
@@ -186,16 +186,17 @@ def stage1_once(indptr, indices, perm, N: int, M: int):
     return out[:n]
 
 
-def pack(indptr, indices, val16, one_bits: int, perm, Vp: int, Mp: int):
+def pack(indptr, indices, val16, one_bits: int, perm, Vp: int, Mp: int, tau: int = 0):
     """Canonical V:N:M packing of B = P A P^T (reading #19).  val16: uint16 bits
-    of A's values per CSR entry (None -> one_bits)."""
+    of A's values per CSR entry (None -> one_bits).  tau: meta-blocks keeping fewer than tau
+    values go to the residual whole (hybrid split, reading #27; 0 = off)."""
     rp, ci, n = _csr(indptr, indices)
     pm = np.ascontiguousarray(perm, dtype=np.int32)
     v16 = None if val16 is None else np.ascontiguousarray(val16, dtype=np.uint16)
     nmb = ctypes.c_int64()
     rnz = ctypes.c_int64()
     L = _lib()
-    L.or_pack_count(n, _p(rp, P64), _p(ci, P32), _p(pm, P32), Vp, Mp, ctypes.byref(nmb),
+    L.or_pack_count(n, _p(rp, P64), _p(ci, P32), _p(pm, P32), Vp, Mp, tau, ctypes.byref(nmb),
                     ctypes.byref(rnz))
     P = (n + Vp - 1) // Vp
     m, r = nmb.value, rnz.value
@@ -205,7 +206,7 @@ def pack(indptr, indices, val16, one_bits: int, perm, Vp: int, Mp: int):
         vals=np.zeros(max(m, 1) * Vp * 2, np.uint16), res_rowptr=np.zeros(n + 1, np.int64),
         res_col=np.zeros(max(r, 1), np.int32), res_val=np.zeros(max(r, 1), np.uint16))
     L.or_pack_fill(n, _p(rp, P64), _p(ci, P32), _p(v16, PU16), one_bits, _p(pm, P32), Vp, Mp,
-                   ctypes.byref(nmb), ctypes.byref(rnz), _p(out["panel_ptr"], P64),
+                   tau, ctypes.byref(nmb), ctypes.byref(rnz), _p(out["panel_ptr"], P64),
                    _p(out["mb_seg"], P32), _p(out["sel"], PU8), _p(out["nib"], PU8),
                    _p(out["vals"], PU16), _p(out["res_rowptr"], P64), _p(out["res_col"], P32),
                    _p(out["res_val"], PU16))

@@ -508,15 +508,15 @@ static void select4(const int* cnt, int Mp, uint8_t* sel) {
 }
 
 int or_pack_fill(int64_t n, const int64_t* rp, const int32_t* ci, const uint16_t* val16,
-                 uint16_t one_bits, const int32_t* perm, int Vp, int Mp, int64_t* n_mb_out,
+                 uint16_t one_bits, const int32_t* perm, int Vp, int Mp, int tau, int64_t* n_mb_out,
                  int64_t* res_nnz_out, int64_t* panel_ptr, int32_t* mb_seg, uint8_t* sel_out,
                  uint8_t* nib_out, uint16_t* vals_out, int64_t* res_rp, int32_t* res_ci,
                  uint16_t* res_val);
 
 /* Counts the packed sizes: number of meta-blocks and residual nonzeros. */
 int or_pack_count(int64_t n, const int64_t* rp, const int32_t* ci, const int32_t* perm, int Vp,
-                  int Mp, int64_t* n_mb, int64_t* res_nnz) {
-  return or_pack_fill(n, rp, ci, NULL, 0, perm, Vp, Mp, n_mb, res_nnz, NULL, NULL, NULL, NULL,
+                  int Mp, int tau, int64_t* n_mb, int64_t* res_nnz) {
+  return or_pack_fill(n, rp, ci, NULL, 0, perm, Vp, Mp, tau, n_mb, res_nnz, NULL, NULL, NULL, NULL,
                       NULL, NULL, NULL, NULL);
 }
 
@@ -527,9 +527,12 @@ int or_pack_count(int64_t n, const int64_t* rp, const int32_t* ci, const int32_t
  *   nib       [n_mb*Vp]   per row of the panel: idx0 | idx1<<2
  *   vals      [n_mb*Vp*2] 16-bit value bits of the two slots
  *   res_rp [n+1], res_ci, res_val: residual CSR (new labels, ascending columns)
- * val16 holds the 16-bit bits of A's values (NULL -> one_bits for every entry). */
+ * val16 holds the 16-bit bits of A's values (NULL -> one_bits for every entry).
+ * tau (hybrid split, reading #27; not in the paper): a meta-block whose rows would
+ * keep fewer than tau values in total is not emitted -- all its entries go to the residual.
+ * tau = 0 is the plain canonical form. */
 int or_pack_fill(int64_t n, const int64_t* rp, const int32_t* ci, const uint16_t* val16,
-                 uint16_t one_bits, const int32_t* perm, int Vp, int Mp, int64_t* n_mb_out,
+                 uint16_t one_bits, const int32_t* perm, int Vp, int Mp, int tau, int64_t* n_mb_out,
                  int64_t* res_nnz_out, int64_t* panel_ptr, int32_t* mb_seg, uint8_t* sel_out,
                  uint8_t* nib_out, uint16_t* vals_out, int64_t* res_rp, int32_t* res_ci,
                  uint16_t* res_val) {
@@ -549,15 +552,30 @@ int or_pack_fill(int64_t n, const int64_t* rp, const int32_t* ci, const uint16_t
     int64_t nseg = 0;
     for (int64_t k = 0; k < cnt; ++k)
       if (k == 0 || segs[k] != segs[k - 1]) segs[nseg++] = segs[k];
-    for (int64_t z = 0; z < nseg; ++z, ++mbk) {
+    for (int64_t z = 0; z < nseg; ++z) {
       int64_t s = segs[z];
-      if (mb_seg) mb_seg[mbk] = (int32_t)s;
       int colcnt[64] = {0};
       for (int64_t i = r0; i < r1; ++i)
         for (int64_t k = B.rp[i]; k < B.rp[i + 1]; ++k)
           if (B.ci[k] / Mp == s) colcnt[B.ci[k] - s * Mp]++;
       uint8_t sel[4];
       select4(colcnt, Mp, sel);
+      if (tau > 0) {
+        /* values the block would keep: per row min(2, entries in the selected columns) */
+        int64_t kept_total = 0;
+        for (int64_t i = r0; i < r1; ++i) {
+          int nk = 0;
+          for (int j = 0; j < 4; ++j) {
+            int64_t col = s * Mp + sel[j];
+            if (col >= n) continue;
+            for (int64_t k = B.rp[i]; k < B.rp[i + 1]; ++k)
+              if (B.ci[k] == col) ++nk;
+          }
+          kept_total += nk < 2 ? nk : 2;
+        }
+        if (kept_total < tau) continue; /* whole block -> residual */
+      }
+      if (mb_seg) mb_seg[mbk] = (int32_t)s;
       if (sel_out) memcpy(sel_out + mbk * 4, sel, 4);
       for (int64_t li = 0; li < Vp; ++li) {
         int64_t i = r0 + li;
@@ -586,6 +604,7 @@ int or_pack_fill(int64_t n, const int64_t* rp, const int32_t* ci, const uint16_t
         if (nib_out) nib_out[mbk * Vp + li] = nb;
         if (vals_out) { vals_out[(mbk * Vp + li) * 2] = v0; vals_out[(mbk * Vp + li) * 2 + 1] = v1; }
       }
+      ++mbk;
     }
     if (panel_ptr) panel_ptr[r + 1] = mbk;
     free(segs);

@@ -151,3 +151,35 @@ def test_spmm_identity_and_ones():
     Y, E, _ = oracle.spmm(ip, ic, None, np.ones((n, 3)))
     deg = np.diff(ip).astype(np.float64)
     assert np.array_equal(Y[:, 0], deg) and (E >= np.abs(Y)).all()
+
+
+@pytest.mark.parametrize("ci", range(4))
+@pytest.mark.parametrize("Vp,Mp,tau", [(128, 4, 3), (128, 4, 40), (64, 8, 5), (128, 16, 2), (128, 4, 10 ** 9)])
+def test_hybrid_tau_drops_thin_blocks_whole(ci, Vp, Mp, tau):
+    """Reading #27: the tau-pack is the tau=0 pack with exactly the blocks that keep fewer than
+    tau values removed (brute-force filter of the plain pack), and stays lossless."""
+    indptr, indices = _pack_cases()[ci]
+    n = len(indptr) - 1
+    perm = np.random.default_rng(10 + ci).permutation(n).astype(np.int32)
+    val16, _ = graphs.round16(graphs.symmetric_values(indptr, indices, seed=ci), "f16")
+    full = oracle.pack(indptr, indices, val16, 0x3C00, perm, Vp, Mp)
+    pk = oracle.pack(indptr, indices, val16, 0x3C00, perm, Vp, Mp, tau=tau)
+    kept = [int(np.count_nonzero(full["vals"][m * Vp * 2:(m + 1) * Vp * 2])) for m in range(full["n_mb"])]
+    keep = [m for m in range(full["n_mb"]) if kept[m] >= tau]
+    assert pk["n_mb"] == len(keep)
+    assert list(pk["mb_seg"]) == [full["mb_seg"][m] for m in keep]
+    for i, m in enumerate(keep):
+        assert np.array_equal(pk["sel"][i * 4:i * 4 + 4], full["sel"][m * 4:m * 4 + 4])
+        assert np.array_equal(pk["nib"][i * Vp:(i + 1) * Vp], full["nib"][m * Vp:(m + 1) * Vp])
+        assert np.array_equal(pk["vals"][i * Vp * 2:(i + 1) * Vp * 2], full["vals"][m * Vp * 2:(m + 1) * Vp * 2])
+    # panel pointers count the surviving blocks of each panel
+    P = (n + Vp - 1) // Vp
+    for r in range(P):
+        exp = sum(1 for m in keep if full["panel_ptr"][r] <= m < full["panel_ptr"][r + 1])
+        assert pk["panel_ptr"][r + 1] - pk["panel_ptr"][r] == exp
+    assert pk["res_nnz"] == full["res_nnz"] + sum(kept[m] for m in range(full["n_mb"]) if kept[m] < tau)
+    Bd, present = oracle.unpack(pk, n)
+    ref, refp = dense_bits(indptr, indices, val16, perm)
+    assert np.array_equal(present, refp) and np.array_equal(Bd, ref)
+    if tau >= 10 ** 9:
+        assert pk["n_mb"] == 0 and pk["res_nnz"] == indptr[-1]
