@@ -31,16 +31,31 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 WORKLOADS = {
-    # configs[1] (SuiteSparse-shaped sweep) headline point: banded n = 2^20, avg degree 16
-    "c2-banded-n1m-d16-f128-1:2:4": dict(kind="band", n=1 << 20, d=16, F=128, V=1, M=4, dtype="f16"),
-    "c2-banded-n1m-d32-f128-1:2:4": dict(kind="band", n=1 << 20, d=32, F=128, V=1, M=4, dtype="f16"),
-    "c2-banded-n262k-d16-f128-64:2:8": dict(kind="band", n=1 << 18, d=16, F=128, V=64, M=8, dtype="f16"),
-    "c2-powerlaw-n262k-d16-f128-1:2:4": dict(kind="pl", n=1 << 18, d=16, F=128, V=1, M=4, dtype="f16"),
-    "c2-powerlaw-n262k-d16-f128-128:2:16": dict(kind="pl", n=1 << 18, d=16, F=128, V=128, M=16, dtype="f16"),
     # configs[0]: ER n = 2048, m = 16384, F = 32, 2:4, fp16 (oracle-sized correctness case)
-    "c1-er-n2048-f32-1:2:4": dict(kind="er", n=2048, m=16384, F=32, V=1, M=4, dtype="f16"),
+    "c1-er-n2048-f32-1:2:4": dict(kind="er", n=2048, m=16384, F=32, V=1, M=4, dtype="f16", tau=0),
 }
+# configs[1] (SuiteSparse-shaped sweep): any point named
+#   c2-{banded|powerlaw}-n{65k|262k|1m}-d{8|16|32|64}-f{F}-{V}:2:{M}[-tau{T}]
+# (tau omitted = the library's cost-model threshold nm_hybrid_tau(F); tau0 = plain pack).
+# The headline point: banded n = 2^20, avg degree 16, F = 128, 1:2:4.
 DEFAULT = "c2-banded-n1m-d16-f128-1:2:4"
+SWEEP = ["c2-banded-n1m-d16-f128-1:2:4", "c2-banded-n1m-d32-f128-1:2:4", "c2-banded-n262k-d16-f128-64:2:8",
+         "c2-powerlaw-n262k-d16-f128-1:2:4", "c2-powerlaw-n262k-d16-f128-128:2:16"]
+_SIZES = {"65k": 1 << 16, "262k": 1 << 18, "1m": 1 << 20}
+
+
+def parse_workload(name):
+    if name in WORKLOADS:
+        return dict(WORKLOADS[name])
+    import re
+    m = re.fullmatch(r"c2-(banded|powerlaw)-n(65k|262k|1m)-d(\d+)-f(\d+)-(\d+):2:(\d+)(?:-tau(\d+))?", name)
+    if not m:
+        raise SystemExit("unknown workload %r (see bench.py WORKLOADS / c2 grammar)" % name)
+    kind, ns, d, F, V, M, tau = m.groups()
+    return dict(kind="band" if kind == "banded" else "pl", n=_SIZES[ns], d=int(d), F=int(F), V=int(V),
+                M=int(M), dtype="f16", tau=None if tau is None else int(tau))
+
+
 METRIC = "V:N:M SpMM GFLOP/s & % sparse-MMA/HBM roofline vs cuSPARSE, 1/2/4/8 B200"
 
 
@@ -199,14 +214,14 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--workload", default=DEFAULT, choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default=DEFAULT, help="c1-er-n2048-f32-1:2:4 or a c2 sweep point (see top)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cusparse", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--order", default="original", choices=["original", "permuted"])
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
-    w = WORKLOADS[args.workload]
+    w = parse_workload(args.workload)
     if args.impl == "reference":
         return run_reference(args, w)
 
@@ -253,7 +268,8 @@ def main():
     from paper_conf_ppopp_chensz0s25_b200.dist import shard_rows
     rb, re = shard_rows(n, world, rank)
     t0 = time.perf_counter()
-    P = api.pack(ip, ic, perm, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order=args.order)
+    tau = w["tau"] if w["tau"] is not None else api.hybrid_tau(F)
+    P = api.pack(ip, ic, perm, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order=args.order, tau=tau)
     torch.cuda.synchronize()
     pack_s = time.perf_counter() - t0
     info = P.info()
@@ -314,34 +330,54 @@ def main():
     useful_flop = 2.0 * nnz * F  # all ranks together (strong scaling: fixed total work)
     value = useful_flop / (ms_per_step * 1e-3) / 1e9
 
-    # ---------------- roofline of the dominant kernel (k_spmm_sptc, this rank) ----------------
+    # ---------------- roofline of the dominant kernel (this rank) ----------------
     hbm_gbs, bf16_tf, peak_src = peaks()
     chunks = info["n_chunks"]
-    # algorithmic bytes per launch: packed image (4608 B/chunk) + gather indices (128 B/chunk)
-    # + X read once (rows of X the shard touches, F*2 B) + Y written once (rows*F*4 B)
     rows_b = re - rb
-    # X rows this shard's SpMM must read at least once (distinct neighbours of its rows)
+    # X rows each kernel must read at least once: distinct columns of B (permuted labels) with a
+    # packed entry (k_spmm_sptc gathers exactly those: zero-count selected columns are skipped)
+    # or a residual entry (k_residual); counted on the host from the shard's rows of B
+    iperm = np.empty(n, np.int64)
+    iperm[perm] = np.arange(n)
     shard_vertices = perm[rb:re].astype(np.int64)
     starts, ends = ip[shard_vertices], ip[shard_vertices + 1]
-    if world == 1:
-        x_rows = int(np.count_nonzero(np.diff(ip)))  # symmetric: columns used = non-isolated vertices
-    else:
-        lens = ends - starts
-        idx = np.repeat(starts - np.concatenate([[0], np.cumsum(lens)[:-1]]), lens) + np.arange(lens.sum())
-        x_rows = int(np.unique(ic[idx]).size)
-    alg_bytes = chunks * (4608 + 128) + x_rows * F * 2 + rows_b * F * 4
-    k_ms = statistics.mean(sptc_ms)
+    lens = ends - starts
+    idx = np.repeat(starts - np.concatenate([[0], np.cumsum(lens)[:-1]]), lens) + np.arange(lens.sum())
+    col_all = np.bincount(iperm[ic[idx]], minlength=n)
+    res = P.export_canonical(residual_only=True)
+    col_res = np.bincount(res["res_col"], minlength=n) if res["res_nnz"] else np.zeros(n, np.int64)
+    x_rows_sptc = int(np.count_nonzero(col_all > col_res))
+    x_rows_res = int(np.count_nonzero(col_res))
+    res_rows = int(np.count_nonzero(np.diff(res["res_rowptr"])))
+    x_rows = int(np.count_nonzero(col_all))
+    # algorithmic bytes per launch
+    #   k_spmm_sptc: chunk records (4736 B: values, metadata, gather rows) + X read once + Y
+    #                written once (rows * F * 4 B)
+    #   k_residual : (col, value) 6 B per residual nonzero + row pointers + X read once + the
+    #                read-modify-write of the Y rows it touches (8 F B each)
+    kern = {"k_spmm_sptc": {"alg_bytes": chunks * 4736 + x_rows_sptc * F * 2 + rows_b * F * 4,
+                            "ms": statistics.mean(sptc_ms)}}
+    if has_res:
+        kern["k_residual"] = {"alg_bytes": res["res_nnz"] * 6 + (rows_b + 1) * 8 + x_rows_res * F * 2 +
+                                           res_rows * F * 8,
+                              "ms": statistics.mean(b - a for a, b in zip(sptc_ms, step_ms))}
+    for k in kern.values():
+        k["achieved_gbs"] = k["alg_bytes"] / (k["ms"] * 1e-3) / 1e9
+        k["frac"] = k["achieved_gbs"] / hbm_gbs
+    dom = max(kern, key=lambda k: kern[k]["ms"])
+    alg_bytes, k_ms = kern[dom]["alg_bytes"], kern[dom]["ms"]
     achieved = alg_bytes / (k_ms * 1e-3) / 1e9
     t_mma_ms = 2.0 * chunks * 128 * max(F, 64) * 32 / (2 * bf16_tf * 1e12) * 1e3  # sparse = 2x dense rate
     roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_gbs, "unit": "GB/s",
                 "frac": achieved / hbm_gbs, "traffic": None, "peak_source": peak_src,
-                "kernel": "k_spmm_sptc", "kernel_ms": k_ms, "alg_bytes_per_launch": alg_bytes,
-                "t_hbm_ms": alg_bytes / (hbm_gbs * 1e9) * 1e3, "t_mma_ms": t_mma_ms}
+                "kernel": dom, "kernel_ms": k_ms, "alg_bytes_per_launch": alg_bytes,
+                "t_hbm_ms": alg_bytes / (hbm_gbs * 1e9) * 1e3, "t_mma_ms_sptc": t_mma_ms,
+                "kernels": kern}
     prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(prof) and world == 1:  # the committed capture is of the 1-GPU launch
         try:
             tr = json.load(open(prof)).get(args.workload)
-            if tr:
+            if tr and tr.get("kernel", "").startswith(dom) and tr.get("tau", tau) == tau:
                 roofline["traffic"] = tr["dram_bytes_per_launch"]
                 roofline["traffic_source"] = "profiles/ncu_traffic.json (%s)" % tr.get("round", "")
         except Exception:
@@ -371,7 +407,7 @@ def main():
                 "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": dt, "data": "synthetic",
                 "config": {"workload": args.workload, "graph": w["kind"], "n": n, "nnz": nnz, "F": F,
-                           "pattern": "%d:2:%d" % (V, M), "order": args.order,
+                           "pattern": "%d:2:%d" % (V, M), "order": args.order, "tau": tau,
                            "parallelism": "row-shard x%d" % world,
                            "l2": "flushed between steps (256 MiB write outside the event-timed intervals)"},
                 "gpu_launches": launches_per_step * args.steps,
@@ -387,6 +423,9 @@ def main():
                                max(1, info["packed_nnz"] + info["residual_nnz"]),
                                "x_rows_read": x_rows,
                                "residual_nnz": info["residual_nnz"],
+                               "residual_rows": res_rows, "x_rows_sptc": x_rows_sptc,
+                               "x_rows_residual": x_rows_res,
+                               "sptc_share_of_nnz": info["packed_nnz"] / max(1, nnz),
                                "packed_bytes": info["device_bytes"]},
                 "step_ms_median": statistics.median(step_ms), "sptc_ms_median": statistics.median(sptc_ms)}
         if cus and "ms" in cus:

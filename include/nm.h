@@ -154,6 +154,25 @@ NM_API nm_status nm_pack_ex(const nm_csr* A, const int32_t* perm, int V, int N, 
                             nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags,
                             void* stream, nm_packed** out);
 
+/* nm_pack_hybrid -- nm_pack_ex plus the hybrid split (reading #27; not in the
+ * paper, an extension of the lossless residual): meta-blocks are formed and their columns
+ * selected exactly as above, then every meta-block whose rows would keep fewer than `tau`
+ * values in total (sum over its Vp rows of min(2, entries in its 4 selected columns)) is not
+ * emitted and ALL of its entries go to the residual CSR.  tau = 0 is nm_pack_ex (plain
+ * canonical form); tau >= 1 never changes Y, only which kernel computes each product.
+ * Motivation: with 128-row panels a scattered graph yields meta-blocks that fill ~1 of their
+ * 256 value slots, which the CSR path moves with fewer bytes.  Errors as nm_pack_ex, plus
+ * INVALID_ARG for tau < 0.  Blocks until the pack is complete. */
+NM_API nm_status nm_pack_hybrid(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
+                                nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags,
+                                int tau, void* stream, nm_packed** out);
+
+/* nm_hybrid_tau -- the tau nm_pack_hybrid should use for an SpMM with F feature columns:
+ * the break-even number of kept values at which a meta-block's bytes through L2 (its share
+ * of a chunk record + 4 gathered X rows) equal those of the same values in the residual CSR
+ * (6 bytes + 1 gathered X row each).  DESIGN.md §6.  Returns 0 for F < 1. */
+NM_API int nm_hybrid_tau(int F);
+
 /* Sizes: #meta-blocks, #values kept in MMA slots, #residual nonzeros, device bytes held,
  * #K=32 chunks (8 meta-blocks each, padded per panel).  Any pointer may be NULL. */
 NM_API nm_status nm_packed_info(const nm_packed* P, int64_t* n_mb, int64_t* packed_nnz,

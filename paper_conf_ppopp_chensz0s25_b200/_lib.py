@@ -64,6 +64,10 @@ SIGNATURES = {
     "nm_pack_ex": (ctypes.c_int, [ctypes.POINTER(nm_csr), P32, ctypes.c_int, ctypes.c_int,
                                   ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int64,
                                   ctypes.c_int64, ctypes.c_int, VP, ctypes.POINTER(VP)]),
+    "nm_pack_hybrid": (ctypes.c_int, [ctypes.POINTER(nm_csr), P32, ctypes.c_int, ctypes.c_int,
+                                      ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int64,
+                                      ctypes.c_int64, ctypes.c_int, ctypes.c_int, VP, ctypes.POINTER(VP)]),
+    "nm_hybrid_tau": (ctypes.c_int, [ctypes.c_int]),
     "nm_packed_info": (ctypes.c_int, [VP, P64, P64, P64, P64, P64]),
     "nm_export_canonical": (ctypes.c_int, [VP, P64, P32, PU8, PU8, PU16, P64, P32, PU16]),
     "nm_packed_free": (None, [VP]),

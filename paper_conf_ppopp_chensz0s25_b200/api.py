@@ -111,25 +111,27 @@ class Packed:
         keys = ("n_mb", "packed_nnz", "residual_nnz", "device_bytes", "n_chunks")
         return {k: int(v.value) for k, v in zip(keys, vals)}
 
-    def export_canonical(self):
+    def export_canonical(self, residual_only=False):
+        """nm_export_canonical -> dict of host arrays (residual_only: just the residual CSR)."""
         inf = self.info()
         m, r = inf["n_mb"], inf["residual_nnz"]
         P = (self.rows + 127) // 128
-        out = dict(panel_ptr=np.zeros(P + 1, np.int64), mb_seg=np.zeros(max(m, 1), np.int32),
-                   sel=np.zeros(max(m, 1) * 4, np.uint8), nib=np.zeros(max(m, 1) * 128, np.uint8),
-                   vals=np.zeros(max(m, 1) * 256, np.uint16),
-                   res_rowptr=np.zeros(self.rows + 1, np.int64),
-                   res_col=np.zeros(max(r, 1), np.int32), res_val=np.zeros(max(r, 1), np.uint16))
+        out = dict(res_rowptr=np.zeros(self.rows + 1, np.int64), res_col=np.zeros(max(r, 1), np.int32),
+                   res_val=np.zeros(max(r, 1), np.uint16))
+        if not residual_only:
+            out.update(panel_ptr=np.zeros(P + 1, np.int64), mb_seg=np.zeros(max(m, 1), np.int32),
+                       sel=np.zeros(max(m, 1) * 4, np.uint8), nib=np.zeros(max(m, 1) * 128, np.uint8),
+                       vals=np.zeros(max(m, 1) * 256, np.uint16))
+        ptr = lambda k, t: out[k].ctypes.data_as(t) if k in out else None
         L.check(L.load().nm_export_canonical(
-            self.handle, out["panel_ptr"].ctypes.data_as(L.P64), out["mb_seg"].ctypes.data_as(L.P32),
-            out["sel"].ctypes.data_as(L.PU8), out["nib"].ctypes.data_as(L.PU8),
-            out["vals"].ctypes.data_as(L.PU16), out["res_rowptr"].ctypes.data_as(L.P64),
-            out["res_col"].ctypes.data_as(L.P32), out["res_val"].ctypes.data_as(L.PU16)),
+            self.handle, ptr("panel_ptr", L.P64), ptr("mb_seg", L.P32), ptr("sel", L.PU8), ptr("nib", L.PU8),
+            ptr("vals", L.PU16), ptr("res_rowptr", L.P64), ptr("res_col", L.P32), ptr("res_val", L.PU16)),
             "nm_export_canonical")
-        out["mb_seg"] = out["mb_seg"][:m]
-        out["sel"] = out["sel"][:m * 4]
-        out["nib"] = out["nib"][:m * 128]
-        out["vals"] = out["vals"][:m * 256]
+        if not residual_only:
+            out["mb_seg"] = out["mb_seg"][:m]
+            out["sel"] = out["sel"][:m * 4]
+            out["nib"] = out["nib"][:m * 128]
+            out["vals"] = out["vals"][:m * 256]
         out["res_col"] = out["res_col"][:r]
         out["res_val"] = out["res_val"][:r]
         out["n_mb"], out["res_nnz"] = m, r
@@ -148,10 +150,11 @@ class Packed:
 
 
 def pack(indptr, indices, perm, V: int, N: int, M: int, dtype="f16", val=None, val_dtype=None,
-         row_begin=None, row_end=None, stream=None, order="permuted"):
-    """nm_pack / nm_pack_rows / nm_pack_ex of B = P A P^T.  val: values per CSR entry (numpy,
-    dtype val_dtype in {'f16','bf16' (uint16 bits),'f32'}) or None for a binary adjacency.
-    order='original' folds the permutation into the SpMM (NM_PACK_ORIGINAL_ORDER)."""
+         row_begin=None, row_end=None, stream=None, order="permuted", tau=0):
+    """nm_pack / nm_pack_rows / nm_pack_ex / nm_pack_hybrid of B = P A P^T.  val: values per CSR
+    entry (numpy, dtype val_dtype in {'f16','bf16' (uint16 bits),'f32'}) or None for a binary
+    adjacency.  order='original' folds the permutation into the SpMM (NM_PACK_ORIGINAL_ORDER).
+    tau > 0: hybrid split (meta-blocks keeping fewer than tau values go to the residual)."""
     if val is not None and val_dtype is None:
         val_dtype = "f32" if val.dtype == np.float32 else ("f16" if val.dtype == np.float16 else "bf16")
     c, keep = _csr_struct(indptr, indices, val, val_dtype or "f16")
@@ -159,23 +162,30 @@ def pack(indptr, indices, perm, V: int, N: int, M: int, dtype="f16", val=None, v
     h = ctypes.c_void_p()
     pp = None if pm is None else pm.ctypes.data_as(L.P32)
     sp = _stream_ptr(stream)
-    if order == "original":
-        rb = 0 if row_begin is None else int(row_begin)
-        re = c.n if row_end is None else int(row_end)
-        L.check(L.load().nm_pack_ex(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], rb, re,
-                                    L.NM_PACK_ORIGINAL_ORDER, sp, ctypes.byref(h)), "nm_pack_ex")
-        P = Packed(h, c.n, rb, re, dtype)
-        P.order = "original"
-        return P
-    if row_begin is None:
-        L.check(L.load().nm_pack(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], sp, ctypes.byref(h)),
-                "nm_pack")
-        rb, re = 0, c.n
+    rb = 0 if row_begin is None else int(row_begin)
+    re = c.n if row_end is None else int(row_end)
+    flags = L.NM_PACK_ORIGINAL_ORDER if order == "original" else 0
+    lib = L.load()
+    if tau:
+        L.check(lib.nm_pack_hybrid(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], rb, re, flags, int(tau), sp,
+                                   ctypes.byref(h)), "nm_pack_hybrid")
+    elif order == "original":
+        L.check(lib.nm_pack_ex(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], rb, re, flags, sp,
+                               ctypes.byref(h)), "nm_pack_ex")
+    elif row_begin is None:
+        L.check(lib.nm_pack(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], sp, ctypes.byref(h)), "nm_pack")
     else:
-        rb, re = int(row_begin), int(row_end)
-        L.check(L.load().nm_pack_rows(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], rb, re, sp,
-                                      ctypes.byref(h)), "nm_pack_rows")
-    return Packed(h, c.n, rb, re, dtype)
+        L.check(lib.nm_pack_rows(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], rb, re, sp, ctypes.byref(h)),
+                "nm_pack_rows")
+    P = Packed(h, c.n, rb, re, dtype)
+    P.order = order
+    P.tau = int(tau)
+    return P
+
+
+def hybrid_tau(F: int) -> int:
+    """nm_hybrid_tau: the library's break-even hybrid-split threshold for F feature columns."""
+    return int(L.load().nm_hybrid_tau(int(F)))
 
 
 def spmm(P: Packed, PX, Yp, F=None, stream=None, part="all"):

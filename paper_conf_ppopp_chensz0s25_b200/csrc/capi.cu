@@ -3,6 +3,7 @@
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 
+#include <cmath>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -161,6 +162,19 @@ const char* nm_status_string(nm_status s) {
 const char* nm_last_error(void) { return g_last_error.c_str(); }
 
 int nm_version(void) { return 1; }
+
+// Hybrid-split threshold from a traffic model (reading #27): every byte either
+// path moves passes the L2 slices (LTS), which cap the whole chip's throughput, so compare
+// LTS bytes.  An emitted meta-block costs its share of a chunk record (kChunkBytes / 8) plus
+// its 4 gathered X rows (4 * 2F bytes); a residual value costs its column + value (6 bytes)
+// plus one gathered X row (2F bytes).  Blocks keeping fewer values than the break-even go to
+// the residual.
+int nm_hybrid_tau(int F) {
+  if (F < 1) return 0;
+  const double block = nm::kChunkBytes / 8.0 + 4.0 * 2.0 * F;
+  const double value = 6.0 + 2.0 * F;
+  return (int)ceil(block / value);
+}
 
 void nm_packed_free(nm_packed* P) {
   if (!P) return;

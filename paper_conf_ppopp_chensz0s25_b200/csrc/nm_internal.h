@@ -40,6 +40,7 @@ struct nm_packed {
   int64_t n = 0;                       // number of vertices (columns of B, rows of PX)
   int64_t row_begin = 0, row_end = 0;  // packed rows of B
   int V = 1, N = 2, M = 4, Vp = 128, Mp = 4;
+  int tau = 0;                         // hybrid split threshold (0 = plain canonical pack)
   nm_dtype dtype = NM_F16;
   int64_t n_panels = 0, n_mb = 0, n_chunks = 0, packed_nnz = 0, res_nnz = 0;
   // device arrays

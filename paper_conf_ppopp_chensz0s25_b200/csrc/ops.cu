@@ -15,42 +15,87 @@ __device__ __forceinline__ float h2f(uint16_t b, int bf) {
   return __half2float(h);
 }
 
-// Yp[l][f] += sum_k res_val[k] * PX[res_col[k]][f] -- one warp per row, 4 columns per lane
-// per pass (8-byte loads of 4 halves), fp32 accumulation.
-template <int BF>
+// Yp[l][f] += sum_k res_val[k] * PX[res_col[k]][f]  (the residual CSR, lossless remainder).
+// One warp per row.  The warp's lanes form SUB = 32 / LPR subgroups of LPR lanes; a subgroup
+// covers LPR * 8 features with one 16-byte X load per lane, and the subgroups take alternate
+// nonzeros of the row (so F = 128 keeps all 32 lanes busy with 16-byte loads).  The row's
+// (col, val) pairs are fetched 32 at a time with one coalesced load and broadcast with
+// shuffles; the nonzero loop is unrolled so several X rows are in flight per lane.  Partial
+// sums are combined across subgroups with xor-shuffles, then added into Y (fp32).
+// F tail: the 16-byte vector at column f0 < F is inside the row (ldx % 8 == 0), only the
+// accumulate/store is masked.
+template <int BF, int LPR>
 __global__ void __launch_bounds__(256) k_residual(const int64_t* __restrict__ rp, const int32_t* __restrict__ rc,
                                                   const uint16_t* __restrict__ rv, int64_t rows,
                                                   const int32_t* __restrict__ row_map,
                                                   const uint16_t* __restrict__ X, int64_t ldx,
                                                   float* __restrict__ Y, int64_t ldy, int F) {
+  constexpr int SUB = 32 / LPR;
+  constexpr int kUnroll = 4;
   const int lane = threadIdx.x & 31;
+  const int sub = lane / LPR, li = lane % LPR;
   const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+  const bool vec_y = ((ldy & 3) == 0) && ((((uintptr_t)Y) & 15) == 0);
   for (int64_t l = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; l < rows; l += nw) {
     const int64_t b = rp[l], e = rp[l + 1];
     if (b == e) continue;
-    for (int f0 = 0; f0 < F; f0 += 128) {
-      const int f = f0 + lane * 4;
-      float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
-      for (int64_t k = b; k < e; ++k) {
-        const float v = h2f(rv[k], BF);
-        const uint16_t* x = X + (int64_t)rc[k] * ldx + f;
-        if (f + 3 < F) {
-          uint2 q = *(const uint2*)x;
-          a0 += v * h2f((uint16_t)(q.x & 0xFFFF), BF);
-          a1 += v * h2f((uint16_t)(q.x >> 16), BF);
-          a2 += v * h2f((uint16_t)(q.y & 0xFFFF), BF);
-          a3 += v * h2f((uint16_t)(q.y >> 16), BF);
-        } else {
-          if (f < F) a0 += v * h2f(x[0], BF);
-          if (f + 1 < F) a1 += v * h2f(x[1], BF);
-          if (f + 2 < F) a2 += v * h2f(x[2], BF);
+    float* yrow = Y + (row_map ? (int64_t)row_map[l] : l) * ldy;
+    for (int f0 = li * 8; f0 - li * 8 < F; f0 += LPR * 8) {
+      float acc[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) acc[q] = 0.f;
+      for (int64_t base = b; base < e; base += 32) {
+        const int cnt = (int)min((int64_t)32, e - base);
+        int32_t c = 0;
+        float v = 0.f;
+        if (lane < cnt) {
+          c = __ldg(rc + base + lane);
+          v = h2f(__ldg(rv + base + lane), BF);
+        }
+        for (int j = 0; j < cnt; j += SUB * kUnroll) {
+          uint4 xv[kUnroll];
+          float vv[kUnroll];
+#pragma unroll
+          for (int u = 0; u < kUnroll; ++u) {
+            const int idx = j + u * SUB + sub;
+            const int32_t cc = __shfl_sync(0xffffffffu, c, idx & 31);
+            vv[u] = __shfl_sync(0xffffffffu, v, idx & 31);
+            if (idx < cnt && f0 < F)
+              xv[u] = __ldg((const uint4*)(X + (int64_t)cc * ldx + f0));
+            else {
+              xv[u] = make_uint4(0u, 0u, 0u, 0u);
+              vv[u] = 0.f;
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < kUnroll; ++u) {
+            const uint32_t w[4] = {xv[u].x, xv[u].y, xv[u].z, xv[u].w};
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              acc[2 * q] += vv[u] * h2f((uint16_t)(w[q] & 0xFFFF), BF);
+              acc[2 * q + 1] += vv[u] * h2f((uint16_t)(w[q] >> 16), BF);
+            }
+          }
         }
       }
-      float* y = Y + (row_map ? (int64_t)row_map[l] : l) * ldy + f;
-      if (f < F) y[0] += a0;
-      if (f + 1 < F) y[1] += a1;
-      if (f + 2 < F) y[2] += a2;
-      if (f + 3 < F) y[3] += a3;
+#pragma unroll
+      for (int o = LPR; o < 32; o <<= 1)
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc[q] += __shfl_xor_sync(0xffffffffu, acc[q], o);
+      if (sub == 0 && f0 < F) {
+        float* y = yrow + f0;
+        if (vec_y && f0 + 8 <= F) {
+          float4 y0 = *(float4*)y, y1 = *(float4*)(y + 4);
+          y0.x += acc[0]; y0.y += acc[1]; y0.z += acc[2]; y0.w += acc[3];
+          y1.x += acc[4]; y1.y += acc[5]; y1.z += acc[6]; y1.w += acc[7];
+          *(float4*)y = y0;
+          *(float4*)(y + 4) = y1;
+        } else {
+#pragma unroll
+          for (int q = 0; q < 8; ++q)
+            if (f0 + q < F) y[q] += acc[q];
+        }
+      }
     }
   }
 }
@@ -118,12 +163,23 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
   const int64_t rows = P->row_end - P->row_begin;
   if (P->res_nnz == 0 || rows == 0) return NM_OK;
   const int32_t* rcol = P->res_gather ? P->res_gather : P->res_col;
-  if (P->dtype == NM_BF16)
-    k_residual<1><<<grid_rows(rows, 8), 256, 0, s>>>(P->res_rowptr, rcol, P->res_val, rows, P->row_map,
-                                                     (const uint16_t*)PX, ldx, Yp, ldy, F);
-  else
-    k_residual<0><<<grid_rows(rows, 8), 256, 0, s>>>(P->res_rowptr, rcol, P->res_val, rows, P->row_map,
-                                                     (const uint16_t*)PX, ldx, Yp, ldy, F);
+  // lanes per row-slice: 8 features per lane, at most one warp per slice
+  const int lpr = F <= 32 ? 4 : F <= 64 ? 8 : F <= 128 ? 16 : 32;
+#define NM_RES_LAUNCH(BF, LPR)                                                                       \
+  k_residual<BF, LPR><<<grid_rows(rows, 8), 256, 0, s>>>(P->res_rowptr, rcol, P->res_val, rows, P->row_map, \
+                                                         (const uint16_t*)PX, ldx, Yp, ldy, F)
+  const int bf = P->dtype == NM_BF16;
+  switch (lpr * 2 + bf) {
+    case 8: NM_RES_LAUNCH(0, 4); break;
+    case 9: NM_RES_LAUNCH(1, 4); break;
+    case 16: NM_RES_LAUNCH(0, 8); break;
+    case 17: NM_RES_LAUNCH(1, 8); break;
+    case 32: NM_RES_LAUNCH(0, 16); break;
+    case 33: NM_RES_LAUNCH(1, 16); break;
+    case 64: NM_RES_LAUNCH(0, 32); break;
+    default: NM_RES_LAUNCH(1, 32); break;
+  }
+#undef NM_RES_LAUNCH
   NM_CUDA(cudaGetLastError());
   return NM_OK;
 }

@@ -158,16 +158,11 @@ __global__ void k_colcount(const int64_t* __restrict__ Brp, const int32_t* __res
   }
 }
 
-// selected columns (4 largest counts, ties -> smaller offset, ascending) and X row indices
-__global__ void k_select(const int32_t* __restrict__ cnt, int Mp, int64_t n_mb,
-                         const int64_t* __restrict__ mbkey, int64_t S, int64_t n,
-                         const int64_t* __restrict__ mbp, const int64_t* __restrict__ chp,
-                         int64_t P, int32_t* __restrict__ mb_seg, uint32_t* __restrict__ mb_sel,
-                         uint8_t* __restrict__ image) {
+// selected columns of every candidate meta-block: the 4 largest counts, ties -> smaller
+// offset, stored ascending (vertical constraint, L338-339; reading #19)
+__global__ void k_select(const int32_t* __restrict__ cnt, int Mp, int64_t n_mb, uint32_t* __restrict__ selc) {
   for (int64_t m = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; m < n_mb;
        m += (int64_t)gridDim.x * blockDim.x) {
-    int64_t panel = mbkey[m] / S, s = mbkey[m] % S;
-    mb_seg[m] = (int32_t)s;
     const int32_t* c = cnt + m * Mp;
     int sel[4];
     if (Mp == 4) {
@@ -188,26 +183,118 @@ __global__ void k_select(const int32_t* __restrict__ cnt, int Mp, int64_t n_mb,
         for (int b = a + 1; b < 4; ++b)
           if (sel[b] < sel[a]) { int t = sel[a]; sel[a] = sel[b]; sel[b] = t; }
     }
-    mb_sel[m] = (uint32_t)sel[0] | ((uint32_t)sel[1] << 8) | ((uint32_t)sel[2] << 16) |
-                ((uint32_t)sel[3] << 24);
-    int64_t local = m - mbp[panel];
-    int64_t chunk = chp[panel] + local / kChunkMB;
-    int g = (int)(local % kChunkMB);
+    selc[m] = (uint32_t)sel[0] | ((uint32_t)sel[1] << 8) | ((uint32_t)sel[2] << 16) | ((uint32_t)sel[3] << 24);
+  }
+}
+
+// index of column `col` (segment s) in the selection, -1 if not selected
+__device__ __forceinline__ int sel_index(uint32_t sel, int32_t col, int64_t s, int Mp) {
+  const int off = col - (int)(s * Mp);
+  for (int j = 0; j < 4; ++j)
+    if ((int)((sel >> (8 * j)) & 0xFF) == off) return j;
+  return -1;
+}
+
+// rank of entry k among the selected entries of its (row, segment) group, the group's
+// first two selected entries (ja/ka, jb) -- the group is contiguous and at most Mp long
+struct GroupPick {
+  int jk, rank, ja, jb;
+  int64_t ka;
+};
+__device__ __forceinline__ GroupPick group_pick(const int32_t* __restrict__ Bci, int64_t b, int64_t e, int64_t k,
+                                                int Mp, uint32_t sel) {
+  const int32_t col = Bci[k];
+  const int64_t s = col / Mp;
+  int64_t gs = k;
+  while (gs > b && Bci[gs - 1] / Mp == s) --gs;
+  int64_t ge = k + 1;
+  while (ge < e && Bci[ge] / Mp == s) ++ge;
+  GroupPick g{sel_index(sel, col, s, Mp), 0, -1, -1, -1};
+  for (int64_t t = gs; t < ge; ++t) {
+    const int jt = sel_index(sel, Bci[t], s, Mp);
+    if (jt < 0) continue;
+    if (t < k) ++g.rank;
+    if (g.ja < 0) { g.ja = jt; g.ka = t; }
+    else if (g.jb < 0) { g.jb = jt; }
+  }
+  return g;
+}
+
+// hybrid split (reading #27): values each candidate meta-block would keep
+// (per row min(2, entries in its selected columns)), one thread per entry
+__global__ void k_keep_count(const int64_t* __restrict__ Brp, const int32_t* __restrict__ Bci, int64_t rows,
+                             int Mp, const int64_t* __restrict__ emb, const uint32_t* __restrict__ selc,
+                             int32_t* __restrict__ keptc) {
+  int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kWarp;
+  int lane = threadIdx.x % kWarp;
+  int64_t nw = (int64_t)gridDim.x * blockDim.x / kWarp;
+  for (int64_t l = warp; l < rows; l += nw) {
+    const int64_t b = Brp[l], e = Brp[l + 1];
+    for (int64_t k = b + lane; k < e; k += kWarp) {
+      const GroupPick g = group_pick(Bci, b, e, k, Mp, selc[emb[k]]);
+      if (g.jk >= 0 && g.rank < 2) atomicAdd(&keptc[emb[k]], 1);
+    }
+  }
+}
+
+__global__ void k_survive(const int32_t* __restrict__ keptc, int64_t n, int tau, int64_t* __restrict__ flag) {
+  for (int64_t m = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; m < n; m += (int64_t)gridDim.x * blockDim.x)
+    flag[m] = keptc[m] >= tau ? 1 : 0;
+}
+
+// compaction of the surviving candidates (newid = exclusive scan of the survive flags)
+__global__ void k_compact(const int64_t* __restrict__ flag, const int64_t* __restrict__ newid, int64_t n,
+                          const int64_t* __restrict__ key_in, const uint32_t* __restrict__ sel_in,
+                          int64_t* __restrict__ key_out, uint32_t* __restrict__ sel_out,
+                          int64_t* __restrict__ cand_of) {
+  for (int64_t m = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; m < n; m += (int64_t)gridDim.x * blockDim.x) {
+    if (!flag[m]) continue;
+    const int64_t d = newid[m];
+    key_out[d] = key_in[m];
+    sel_out[d] = sel_in[m];
+    cand_of[d] = m;
+  }
+}
+
+__global__ void k_remap_emb(const int64_t* __restrict__ flag, const int64_t* __restrict__ newid,
+                            int64_t* __restrict__ emb, int64_t nnz) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nnz; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t m = emb[k];
+    emb[k] = flag[m] ? newid[m] : -1;
+  }
+}
+
+// per emitted meta-block: segment id, selection and the X row of each logical k
+__global__ void k_write_sel(const int32_t* __restrict__ cnt, const int64_t* __restrict__ cand_of, int Mp,
+                            int64_t n_mb, const int64_t* __restrict__ mbkey, int64_t S, int64_t n,
+                            const int64_t* __restrict__ mbp, const int64_t* __restrict__ chp,
+                            int32_t* __restrict__ mb_seg, uint32_t* __restrict__ mb_sel,
+                            uint8_t* __restrict__ image) {
+  for (int64_t m = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; m < n_mb;
+       m += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t panel = mbkey[m] / S, s = mbkey[m] % S;
+    mb_seg[m] = (int32_t)s;
+    const uint32_t sel = mb_sel[m];
+    const int32_t* c = cnt + (cand_of ? cand_of[m] : m) * Mp;
+    const int64_t local = m - mbp[panel];
+    const int64_t chunk = chp[panel] + local / kChunkMB;
+    const int g = (int)(local % kChunkMB);
     int32_t* xrow = (int32_t*)(image + chunk * kChunkBytes + kChunkXrowOff);
     for (int j = 0; j < 4; ++j) {
-      int64_t col = s * Mp + sel[j];
+      const int off = (int)((sel >> (8 * j)) & 0xFF);
+      const int64_t col = s * Mp + off;
       // zero-count or phantom columns gather nothing (zero-filled operand rows)
-      xrow[g * 4 + j] = (col < n && c[sel[j]] > 0) ? (int32_t)col : -1;
+      xrow[g * 4 + j] = (col < n && c[off] > 0) ? (int32_t)col : -1;
     }
   }
 }
 
 // Places every entry: MMA slot (value + nibble) or residual flag.  One thread per entry; the
-// entry inspects its (row, segment) group, which is contiguous and at most Mp long.
+// entry inspects its (row, segment) group, which is contiguous and at most Mp long.  Entries
+// of a meta-block dropped by the hybrid split (emb < 0) all go to the residual.
 __global__ void k_place(const int64_t* __restrict__ Brp, const int32_t* __restrict__ Bci,
                         const uint16_t* __restrict__ Bval, int64_t rows, int Mp,
                         const int64_t* __restrict__ emb, const uint32_t* __restrict__ mb_sel,
-                        const int64_t* __restrict__ mbkey, int64_t S,
                         const int64_t* __restrict__ mbp, const int64_t* __restrict__ chp,
                         uint8_t* __restrict__ image, uint8_t* __restrict__ resflag,
                         unsigned long long* __restrict__ kept_count) {
@@ -217,35 +304,13 @@ __global__ void k_place(const int64_t* __restrict__ Brp, const int32_t* __restri
   for (int64_t l = warp; l < rows; l += nw) {
     int64_t b = Brp[l], e = Brp[l + 1];
     for (int64_t k = b + lane; k < e; k += kWarp) {
-      int32_t col = Bci[k];
-      int64_t s = col / Mp;
-      uint32_t sel = mb_sel[emb[k]];
-      auto jof = [&](int32_t c) -> int {
-        int off = c - (int)(s * Mp);
-        for (int j = 0; j < 4; ++j)
-          if ((int)((sel >> (8 * j)) & 0xFF) == off) return j;
-        return -1;
-      };
-      // group bounds
-      int64_t gs = k;
-      while (gs > b && Bci[gs - 1] / Mp == s) --gs;
-      int64_t ge = k + 1;
-      while (ge < e && Bci[ge] / Mp == s) ++ge;
-      int jk = jof(col);
-      int rank = 0, ja = -1, jb = -1;
-      int64_t ka = -1;
-      for (int64_t t = gs; t < ge; ++t) {
-        int jt = jof(Bci[t]);
-        if (jt < 0) continue;
-        if (t < k) ++rank;
-        if (ja < 0) { ja = jt; ka = t; }
-        else if (jb < 0) { jb = jt; }
-      }
-      bool kept = jk >= 0 && rank < 2;
+      const int64_t m = emb[k];
+      if (m < 0) { resflag[k] = 1; continue; }
+      const GroupPick gp = group_pick(Bci, b, e, k, Mp, mb_sel[m]);
+      bool kept = gp.jk >= 0 && gp.rank < 2;
       resflag[k] = kept ? 0 : 1;
       if (!kept) continue;
       atomicAdd(kept_count, 1ull);
-      int64_t m = emb[k];
       int64_t panel = l / kPanelRows;
       int64_t local = m - mbp[panel];
       int64_t chunk = chp[panel] + local / kChunkMB;
@@ -255,18 +320,16 @@ __global__ void k_place(const int64_t* __restrict__ Brp, const int32_t* __restri
       // slot assignment (reading #19): two kept (a<b) -> (a,b) slots 0,1; one kept
       // at j<3 -> (j,3) slot 0; one kept at j=3 -> (0,3) slot 1
       int i0, i1, slot;
-      if (jb >= 0) { i0 = ja; i1 = jb; slot = (k == ka) ? 0 : 1; }
-      else if (ja < 3) { i0 = ja; i1 = 3; slot = 0; }
+      if (gp.jb >= 0) { i0 = gp.ja; i1 = gp.jb; slot = (k == gp.ka) ? 0 : 1; }
+      else if (gp.ja < 3) { i0 = gp.ja; i1 = 3; slot = 0; }
       else { i0 = 0; i1 = 3; slot = 1; }
       *(uint16_t*)(cv + val_off(r, 2 * g + slot)) = Bval[k];
-      if (k == ka) {
+      if (k == gp.ka) {
         int w, sh;
         meta_pos(r, g, &w, &sh);
         uint32_t nib = (uint32_t)(i0 | (i1 << 2));
         atomicXor((uint32_t*)(cv + kChunkValBytes) + w, (nib ^ 0x4u) << sh);
       }
-      (void)mbkey;
-      (void)S;
     }
   }
 }
@@ -356,7 +419,9 @@ __global__ void k_map(const int32_t* __restrict__ perm, int32_t* __restrict__ a,
 }
 
 nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int M, int Vp,
-                    nm_dtype dtype, int64_t rb, int64_t re, int flags, cudaStream_t s, nm_packed** out) {
+                    nm_dtype dtype, int64_t rb, int64_t re, int flags, int tau, cudaStream_t s,
+                    nm_packed** out) {
+  if (tau < 0) return fail(NM_ERR_INVALID_ARG, "nm_pack: tau < 0");
   if (!A || !out) return fail(NM_ERR_INVALID_ARG, "nm_pack: NULL argument");
   if (N != 2) return fail(NM_ERR_UNSUPPORTED, "nm_pack: N must be 2 (hardware 2:4, L496)");
   if (!(M == 4 || M == 8 || M == 16)) return fail(NM_ERR_UNSUPPORTED, "nm_pack: M must be 4, 8 or 16");
@@ -459,17 +524,59 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     NM_CUDA(cub::DeviceRunLengthEncode::Encode(tmp.p, bytes, d_mk2.as<int64_t>(), d_mbkey.as<int64_t>(),
                                                d_runs.as<int64_t>(), d_nruns.as<int64_t>(), bnnz, s));
   }
-  int64_t n_mb = 0;
+  int64_t n_cand = 0;  // candidate meta-blocks: distinct non-empty (panel, segment) pairs
   if (bnnz > 0) {
-    NM_CUDA(cudaMemcpyAsync(&n_mb, d_nruns.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    NM_CUDA(cudaMemcpyAsync(&n_cand, d_nruns.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     NM_CUDA(cudaStreamSynchronize(s));
+  }
+
+  // ---- 3. column counts, selection and (tau > 0) the hybrid split of thin meta-blocks ----
+  DevBuf d_cnt, d_emb, d_selc;
+  const int64_t nc1 = n_cand > 0 ? n_cand : 1;
+  NM_TRY(dalloc(d_cnt, sizeof(int32_t) * Mp * nc1, s));
+  NM_TRY(dalloc(d_emb, sizeof(int64_t) * bnnz, s));
+  NM_TRY(dalloc(d_selc, sizeof(uint32_t) * nc1, s));
+  NM_CUDA(cudaMemsetAsync(d_cnt.p, 0, sizeof(int32_t) * Mp * nc1, s));
+  if (bnnz) {
+    k_colcount<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, rows, Mp, S, d_mbkey.as<int64_t>(), n_cand,
+                                                       d_cnt.as<int32_t>(), d_emb.as<int64_t>());
+    k_select<<<grid_for(n_cand, 256), 256, 0, s>>>(d_cnt.as<int32_t>(), Mp, n_cand, d_selc.as<uint32_t>());
+  }
+  NM_CUDA(cudaGetLastError());
+  int64_t n_mb = n_cand;
+  const int64_t* mbkey = d_mbkey.as<int64_t>();
+  const uint32_t* selv = d_selc.as<uint32_t>();
+  DevBuf d_keptc, d_flag_mb, d_newid, d_key_c, d_sel_c, d_cand_of;
+  if (tau > 0 && n_cand > 0) {
+    NM_TRY(dalloc(d_keptc, sizeof(int32_t) * n_cand, s));
+    NM_TRY(dalloc(d_flag_mb, sizeof(int64_t) * (n_cand + 1), s));
+    NM_TRY(dalloc(d_newid, sizeof(int64_t) * (n_cand + 1), s));
+    NM_CUDA(cudaMemsetAsync(d_keptc.p, 0, sizeof(int32_t) * n_cand, s));
+    NM_CUDA(cudaMemsetAsync(d_flag_mb.p, 0, sizeof(int64_t) * (n_cand + 1), s));
+    k_keep_count<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, rows, Mp, d_emb.as<int64_t>(), selv,
+                                                         d_keptc.as<int32_t>());
+    k_survive<<<grid_for(n_cand, 256), 256, 0, s>>>(d_keptc.as<int32_t>(), n_cand, tau, d_flag_mb.as<int64_t>());
+    NM_TRY(scan_excl(d_flag_mb.as<int64_t>(), d_newid.as<int64_t>(), n_cand + 1, s));
+    NM_CUDA(cudaMemcpyAsync(&n_mb, d_newid.as<int64_t>() + n_cand, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    NM_CUDA(cudaStreamSynchronize(s));
+    NM_TRY(dalloc(d_key_c, sizeof(int64_t) * (n_mb > 0 ? n_mb : 1), s));
+    NM_TRY(dalloc(d_sel_c, sizeof(uint32_t) * (n_mb > 0 ? n_mb : 1), s));
+    NM_TRY(dalloc(d_cand_of, sizeof(int64_t) * (n_mb > 0 ? n_mb : 1), s));
+    k_compact<<<grid_for(n_cand, 256), 256, 0, s>>>(d_flag_mb.as<int64_t>(), d_newid.as<int64_t>(), n_cand, mbkey,
+                                                    selv, d_key_c.as<int64_t>(), d_sel_c.as<uint32_t>(),
+                                                    d_cand_of.as<int64_t>());
+    k_remap_emb<<<grid_for(bnnz, 256), 256, 0, s>>>(d_flag_mb.as<int64_t>(), d_newid.as<int64_t>(),
+                                                    d_emb.as<int64_t>(), bnnz);
+    NM_CUDA(cudaGetLastError());
+    mbkey = d_key_c.as<int64_t>();
+    selv = d_sel_c.as<uint32_t>();
   }
 
   nm_packed* Pk = new nm_packed();
   NM_CUDA(cudaGetDevice(&Pk->device));
   Pk->n = n; Pk->row_begin = rb; Pk->row_end = re;
   Pk->V = V; Pk->N = N; Pk->M = M; Pk->Vp = Vp; Pk->Mp = Mp; Pk->dtype = dtype;
-  Pk->n_panels = P; Pk->n_mb = n_mb;
+  Pk->n_panels = P; Pk->n_mb = n_mb; Pk->tau = tau;
   struct Guard {
     nm_packed* p;
     bool ok = false;
@@ -482,7 +589,7 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   };
   NM_TRY(palloc((void**)&Pk->panel_mb_ptr, sizeof(int64_t) * (P + 1)));
   NM_TRY(palloc((void**)&Pk->panel_chunk_ptr, sizeof(int64_t) * (P + 1)));
-  k_panel_ptr<<<grid_for(P + 1, 256), 256, 0, s>>>(d_mbkey.as<int64_t>(), n_mb, P, S, Pk->panel_mb_ptr, nullptr);
+  k_panel_ptr<<<grid_for(P + 1, 256), 256, 0, s>>>(mbkey, n_mb, P, S, Pk->panel_mb_ptr, nullptr);
   DevBuf d_nch;
   NM_TRY(dalloc(d_nch, sizeof(int64_t) * (P + 1), s));
   NM_CUDA(cudaMemsetAsync(d_nch.p, 0, sizeof(int64_t) * (P + 1), s));
@@ -524,18 +631,11 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     k_meta_init<<<grid_for(n_chunks * 128, 256), 256, 0, s>>>(Pk->image, n_chunks);
     k_xrow_map<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(nullptr, Pk->image, n_chunks);
   }
-
-  // ---- 3. column counts and selection ----
-  DevBuf d_cnt, d_emb;
-  NM_TRY(dalloc(d_cnt, sizeof(int32_t) * Mp * (n_mb > 0 ? n_mb : 1), s));
-  NM_TRY(dalloc(d_emb, sizeof(int64_t) * bnnz, s));
-  NM_CUDA(cudaMemsetAsync(d_cnt.p, 0, sizeof(int32_t) * Mp * (n_mb > 0 ? n_mb : 1), s));
-  if (bnnz) {
-    k_colcount<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, rows, Mp, S, d_mbkey.as<int64_t>(), n_mb,
-                                                       d_cnt.as<int32_t>(), d_emb.as<int64_t>());
-    k_select<<<grid_for(n_mb, 256), 256, 0, s>>>(d_cnt.as<int32_t>(), Mp, n_mb, d_mbkey.as<int64_t>(), S, n,
-                                                 Pk->panel_mb_ptr, Pk->panel_chunk_ptr, P, Pk->mb_seg,
-                                                 Pk->mb_sel, Pk->image);
+  if (n_mb) {
+    NM_CUDA(cudaMemcpyAsync(Pk->mb_sel, selv, sizeof(uint32_t) * n_mb, cudaMemcpyDeviceToDevice, s));
+    k_write_sel<<<grid_for(n_mb, 256), 256, 0, s>>>(d_cnt.as<int32_t>(), d_cand_of.p ? d_cand_of.as<int64_t>() : nullptr,
+                                                    Mp, n_mb, mbkey, S, n, Pk->panel_mb_ptr, Pk->panel_chunk_ptr,
+                                                    Pk->mb_seg, Pk->mb_sel, Pk->image);
   }
   NM_CUDA(cudaGetLastError());
 
@@ -548,9 +648,8 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   NM_CUDA(cudaMemsetAsync(d_rc.p, 0, sizeof(int64_t) * (rows + 1), s));
   if (bnnz) {
     k_place<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, Bval, rows, Mp, d_emb.as<int64_t>(), Pk->mb_sel,
-                                                    d_mbkey.as<int64_t>(), S, Pk->panel_mb_ptr,
-                                                    Pk->panel_chunk_ptr, Pk->image, d_flag.as<uint8_t>(),
-                                                    d_kept.as<unsigned long long>());
+                                                    Pk->panel_mb_ptr, Pk->panel_chunk_ptr, Pk->image,
+                                                    d_flag.as<uint8_t>(), d_kept.as<unsigned long long>());
     k_res_count<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, d_flag.as<uint8_t>(), rows, d_rc.as<int64_t>());
   }
   NM_CUDA(cudaGetLastError());
@@ -595,18 +694,25 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
 extern "C" nm_status nm_pack(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
                              nm_dtype dtype, void* stream, nm_packed** out) {
   if (!A) return nm::fail(NM_ERR_INVALID_ARG, "nm_pack: NULL graph");
-  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, 0, A->n, 0, (cudaStream_t)stream, out);
+  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, 0, A->n, 0, 0, (cudaStream_t)stream, out);
 }
 
 extern "C" nm_status nm_pack_rows(const nm_csr* A, const int32_t* perm, int V, int N, int M,
                                   int Vp, nm_dtype dtype, int64_t row_begin, int64_t row_end,
                                   void* stream, nm_packed** out) {
-  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, 0, (cudaStream_t)stream, out);
+  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, 0, 0, (cudaStream_t)stream, out);
 }
 
 extern "C" nm_status nm_pack_ex(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
                                 nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags, void* stream,
                                 nm_packed** out) {
   if (flags & ~NM_PACK_ORIGINAL_ORDER) return nm::fail(NM_ERR_INVALID_ARG, "nm_pack_ex: unknown flags");
-  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, flags, (cudaStream_t)stream, out);
+  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, flags, 0, (cudaStream_t)stream, out);
+}
+
+extern "C" nm_status nm_pack_hybrid(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
+                                    nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags, int tau,
+                                    void* stream, nm_packed** out) {
+  if (flags & ~NM_PACK_ORIGINAL_ORDER) return nm::fail(NM_ERR_INVALID_ARG, "nm_pack_hybrid: unknown flags");
+  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, flags, tau, (cudaStream_t)stream, out);
 }

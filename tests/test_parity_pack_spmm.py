@@ -237,3 +237,46 @@ def test_spmm_original_order_fused(kind, seed, V, M, dtype):
         api.spmm(Ps, X, Y2)
     torch.cuda.synchronize()
     assert torch.equal(Y, Y2)
+
+
+# ------------------------------------------------------------------------------------------
+# hybrid split (nm_pack_hybrid, reading #27): thin meta-blocks go to the residual
+# ------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("kind,seed,V,M,tau", [("c1", 1, 1, 4, 3), ("pl", 3, 1, 4, 8), ("pl", 6, 128, 16, 2),
+                                               ("band", 5, 64, 8, 5), ("er", 7, 8, 8, 40),
+                                               ("band", 4, 1, 4, 10 ** 6)])
+@pytest.mark.parametrize("order", ["permuted", "original"])
+def test_pack_hybrid_canonical_bit_exact(kind, seed, V, M, tau, order):
+    _cuda()
+    ip, ic = _graph(kind, seed)
+    perm, _ = api.reorder(ip, ic, V, 2, M)
+    v32, bits, _ = _values(ip, ic, "f16", seed)
+    Mp = 4 if V == 1 else M
+    ref = oracle.pack(ip, ic, bits, 0, perm, 128, Mp, tau=tau)
+    P = api.pack(ip, ic, perm, V, 2, M, dtype="f16", val=v32, tau=tau, order=order)
+    got = P.export_canonical()
+    for k in ("panel_ptr", "mb_seg", "sel", "nib", "vals", "res_rowptr", "res_col", "res_val"):
+        assert np.array_equal(ref[k], got[k]), k
+    inf = P.info()
+    assert inf["n_mb"] == ref["n_mb"] and inf["residual_nnz"] == ref["res_nnz"]
+    assert inf["packed_nnz"] + inf["residual_nnz"] == ip[-1]
+
+
+@pytest.mark.parametrize("kind,seed,V,M,tau", [("pl", 3, 1, 4, 8), ("band", 5, 64, 8, 5), ("c1", 1, 1, 4, 10 ** 6)])
+def test_spmm_hybrid_parity(kind, seed, V, M, tau):
+    """Y of the hybrid pack (original order, fused permutation) within the north-star bound."""
+    dev = _cuda()
+    ip, ic = _graph(kind, seed)
+    n = len(ip) - 1
+    F = 128
+    perm, _ = api.reorder(ip, ic, V, 2, M)
+    v32, bits, v64 = _values(ip, ic, "f16", seed)
+    xbits, x64 = graphs.round16(graphs.features(n, F, seed + 2), "f16")
+    Y_ref, E, _ = oracle.spmm(ip, ic, v64, x64)
+    X = torch.from_numpy(xbits.view(np.int16)).to(dev).view(torch.float16)
+    P = api.pack(ip, ic, perm, V, 2, M, dtype="f16", val=v32, order="original", tau=tau)
+    Y = torch.full((n, F), float("nan"), device=dev)
+    api.spmm(P, X, Y)
+    torch.cuda.synchronize()
+    err = np.abs(Y.cpu().numpy().astype(np.float64) - Y_ref)
+    assert (err <= TOL * E).all(), err.max()
