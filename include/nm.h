@@ -178,6 +178,16 @@ NM_API int nm_hybrid_tau(int F);
 NM_API nm_status nm_packed_info(const nm_packed* P, int64_t* n_mb, int64_t* packed_nnz,
                          int64_t* residual_nnz, int64_t* device_bytes, int64_t* n_chunks);
 
+/* All sizes of a packed matrix (superset of nm_packed_info).  image_bytes = the compressed
+ * chunk records nm_spmm streams from HBM; residual_items = warp work items of
+ * the residual SpMM (<= 256 nonzeros each), residual_split_rows = rows cut into several. */
+typedef struct {
+  int64_t n, row_begin, row_end, n_panels, n_mb, n_chunks, packed_nnz, residual_nnz;
+  int64_t image_bytes, device_bytes, residual_items, residual_split_rows;
+  int32_t V, M, Mp, Vp, tau, flags;
+} nm_packed_stat;
+NM_API nm_status nm_packed_stats(const nm_packed* P, nm_packed_stat* st);
+
 /* Copies the canonical form back to host arrays (caller-allocated, sizes from
  * nm_packed_info; rows = row_end - row_begin, panels = ceil(rows / Vp)):
  *   panel_ptr int64[panels+1], mb_seg int32[n_mb], sel uint8[n_mb*4] (ascending offsets),

@@ -45,6 +45,13 @@ class nm_reorder_stats(ctypes.Structure):
                 ("seconds", ctypes.c_double)]
 
 
+class nm_packed_stat(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_int64) for k in ("n", "row_begin", "row_end", "n_panels", "n_mb", "n_chunks",
+                                              "packed_nnz", "residual_nnz", "image_bytes", "device_bytes",
+                                              "residual_items", "residual_split_rows")] + \
+               [(k, ctypes.c_int32) for k in ("V", "M", "Mp", "Vp", "tau", "flags")]
+
+
 # name -> (restype, argtypes); mirrors include/nm.h exactly
 SIGNATURES = {
     "nm_reorder": (ctypes.c_int, [ctypes.POINTER(nm_csr), ctypes.c_int, ctypes.c_int, ctypes.c_int,
@@ -69,6 +76,7 @@ SIGNATURES = {
                                       ctypes.c_int64, ctypes.c_int, ctypes.c_int, VP, ctypes.POINTER(VP)]),
     "nm_hybrid_tau": (ctypes.c_int, [ctypes.c_int]),
     "nm_packed_info": (ctypes.c_int, [VP, P64, P64, P64, P64, P64]),
+    "nm_packed_stats": (ctypes.c_int, [VP, ctypes.POINTER(nm_packed_stat)]),
     "nm_export_canonical": (ctypes.c_int, [VP, P64, P32, PU8, PU8, PU16, P64, P32, PU16]),
     "nm_packed_free": (None, [VP]),
     "nm_permute_rows": (ctypes.c_int, [VP, VP, VP, ctypes.c_int64, ctypes.c_int, ctypes.c_int64,

@@ -111,6 +111,12 @@ class Packed:
         keys = ("n_mb", "packed_nnz", "residual_nnz", "device_bytes", "n_chunks")
         return {k: int(v.value) for k, v in zip(keys, vals)}
 
+    def stats(self):
+        """nm_packed_stats: every size of the packed matrix as a dict."""
+        st = L.nm_packed_stat()
+        L.check(L.load().nm_packed_stats(self.handle, ctypes.byref(st)), "nm_packed_stats")
+        return {f: getattr(st, f) for f, _ in L.nm_packed_stat._fields_}
+
     def export_canonical(self, residual_only=False):
         """nm_export_canonical -> dict of host arrays (residual_only: just the residual CSR)."""
         inf = self.info()

@@ -23,6 +23,8 @@ SOURCES = ["capi.cu", "pack.cu", "spmm_sm100.cu", "ops.cu", "counts.cu", "gcn.cu
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-lineinfo", "-std=c++17", "-I" + os.path.join(ROOT, "include"),
           "-Xcompiler", "-fPIC,-fopenmp,-fvisibility=hidden", "--expt-relaxed-constexpr"]
+# tuning experiments only (e.g. NM_NVCC_FLAGS="-DNM_LOAD_GROUPS=4"); the product build sets none
+COMMON += os.environ.get("NM_NVCC_FLAGS", "").split()
 
 
 def _deps_mtime() -> float:

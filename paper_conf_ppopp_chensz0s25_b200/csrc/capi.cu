@@ -183,7 +183,7 @@ void nm_packed_free(nm_packed* P) {
   cudaSetDevice(P->device);
   void* ptrs[] = {P->panel_mb_ptr, P->panel_chunk_ptr, P->unit_info, P->mb_seg, P->mb_sel,
                   P->image, P->res_rowptr, P->res_col, P->res_val, P->row_map,
-                  P->res_gather};
+                  P->res_gather, P->res_segs, P->res_ws, P->res_cnt, P->rec_len16};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   cudaSetDevice(cur);
@@ -198,6 +198,29 @@ nm_status nm_packed_info(const nm_packed* P, int64_t* n_mb, int64_t* packed_nnz,
   if (residual_nnz) *residual_nnz = P->res_nnz;
   if (device_bytes) *device_bytes = (int64_t)P->device_bytes;
   if (n_chunks) *n_chunks = P->n_chunks;
+  return NM_OK;
+}
+
+nm_status nm_packed_stats(const nm_packed* P, nm_packed_stat* st) {
+  if (!P || !st) return fail(NM_ERR_INVALID_ARG, "nm_packed_stats: NULL argument");
+  st->n = P->n;
+  st->row_begin = P->row_begin;
+  st->row_end = P->row_end;
+  st->n_panels = P->n_panels;
+  st->n_mb = P->n_mb;
+  st->n_chunks = P->n_chunks;
+  st->packed_nnz = P->packed_nnz;
+  st->residual_nnz = P->res_nnz;
+  st->image_bytes = P->image_bytes;
+  st->device_bytes = (int64_t)P->device_bytes;
+  st->residual_items = P->n_res_segs;
+  st->residual_split_rows = P->n_res_split;
+  st->V = P->V;
+  st->M = P->M;
+  st->Mp = P->Mp;
+  st->Vp = P->Vp;
+  st->tau = P->tau;
+  st->flags = P->flags;
   return NM_OK;
 }
 
@@ -224,8 +247,43 @@ nm_status nm_export_canonical(const nm_packed* P, int64_t* panel_ptr, int32_t* m
       for (int j = 0; j < 4; ++j) sel[m * 4 + j] = (uint8_t)((s[m] >> (8 * j)) & 0xFF);
   }
   if ((nib || vals) && P->n_mb) {
-    std::vector<uint8_t> img((size_t)P->n_chunks * kChunkBytes);
-    NM_CUDA(cudaMemcpy(img.data(), P->image, img.size(), cudaMemcpyDeviceToHost));
+    // expand the compressed HBM records (nm_internal.h kRec* layout) back into full MMA-layout
+    // records -- a host decoder independent of the SpMM kernel's shared-memory expansion
+    std::vector<uint8_t> cimg((size_t)P->image_bytes);
+    std::vector<uint16_t> len16(P->n_chunks);
+    NM_CUDA(cudaMemcpy(cimg.data(), P->image, cimg.size(), cudaMemcpyDeviceToHost));
+    NM_CUDA(cudaMemcpy(len16.data(), P->rec_len16, sizeof(uint16_t) * P->n_chunks, cudaMemcpyDeviceToHost));
+    std::vector<uint8_t> img((size_t)P->n_chunks * kChunkBytes, 0);
+    size_t off = 0;
+    for (int64_t c = 0; c < P->n_chunks; ++c) {
+      const uint8_t* rec = cimg.data() + off;
+      off += (size_t)len16[c] * 16;
+      uint8_t* fr = img.data() + (size_t)c * kChunkBytes;
+      memcpy(fr + kChunkXrowOff, rec, kChunkXrowBytes);
+      uint16_t ne, nr;
+      memcpy(&ne, rec + kRecTotOff, 2);
+      memcpy(&nr, rec + kRecTotOff + 2, 2);
+      const uint8_t* pv = rec + kRecHdrBytes;
+      const uint8_t* pn = pv + 4 * (size_t)ne;
+      uint32_t* meta = (uint32_t*)(fr + kChunkValBytes);
+      for (int w = 0; w < 128; ++w) meta[w] = 0;
+      for (int r = 0; r < kPanelRows; ++r) {
+        const uint8_t mask = rec[kRecMaskOff + r];
+        uint32_t W = kMetaNone;
+        if (mask) { memcpy(&W, pn, 4); pn += 4; }
+        for (int g = 0; g < kChunkMB; ++g) {
+          uint32_t v = 0;
+          if (mask & (1u << g)) { memcpy(&v, pv, 4); pv += 4; }
+          for (int slot = 0; slot < 2; ++slot) {
+            const int k = 2 * g + slot;
+            const uint16_t h = (uint16_t)(v >> (16 * slot));
+            memcpy(fr + (r % 8) * 16 + (r / 8) * 256 + (k / 8) * 128 + (k % 8) * 2, &h, 2);
+          }
+          const int lane = (r % 8) + 8 * (g / 4) + 16 * (r / 16);
+          meta[lane] |= ((W >> (4 * g)) & 0xFu) << (16 * ((r / 8) % 2) + 4 * (g % 4));
+        }
+      }
+    }
     for (int64_t p = 0; p < P->n_panels; ++p) {
       for (int64_t m = mbp[p]; m < mbp[p + 1]; ++m) {
         int64_t local = m - mbp[p];

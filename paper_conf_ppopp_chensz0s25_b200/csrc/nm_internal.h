@@ -33,6 +33,39 @@ constexpr int kChunkBytes = kChunkValBytes + kChunkMetaBytes + kChunkXrowBytes;
 constexpr int kChunkXrowOff = kChunkValBytes + kChunkMetaBytes;
 constexpr uint32_t kMetaNone = 0x44444444u;  // every nibble = (0,1): legal code, zero values
 
+// ---- compressed chunk record in HBM (the "SPTC required form on the fly" of L492) ----------
+// The MMA operands above are what the tensor core reads from shared memory; in HBM a chunk is
+// stored without its empty (row, meta-block) slots and the SpMM's loader warps expand it in
+// shared memory.  (row r, group g) is empty iff its nibble is the no-value code 0x4 and both
+// value slots are +0 bits.  Layout (variable size, padded to 16 bytes):
+//   [  0..128) xrow  int32[32]  gather row per logical k (as in the full record)
+//   [128..256) mask  uint8[128] bit g of row r = (r, g) not empty
+//   [256..264) qv    uint16[4]  first value entry of each 32-row quarter
+//   [264..272) qn    uint16[4]  first nibble word of each 32-row quarter
+//   [272..276) ne, nr uint16    #value entries, #non-empty rows
+//   [276]      cmask uint8     bit q: gather rows 8q..8q+7 are 8 consecutive rows of X (one
+//                               TMA tile load instead of 8 row gathers);  [277..288) zero
+//   [288 ..  ) vals  uint32[ne] slot0 | slot1 << 16 per non-empty (r, g), row-major
+//   then       nibs  uint32[nr] nibble word of each non-empty row (group g at bits 4g)
+constexpr int kRecMaskOff = 128, kRecQvOff = 256, kRecQnOff = 264, kRecTotOff = 272, kRecContOff = 276;
+constexpr int kRecHdrBytes = 288;
+constexpr int kRecMaxBytes = kRecHdrBytes + 4 * (kPanelRows + kPanelRows * kChunkMB);  // 4896
+
+// Residual work items (DESIGN.md §6 k_residual): each row's residual nonzeros are cut into
+// segments of at most kResSeg entries, one warp each, so hub rows of power-law graphs spread
+// over many warps.  A row cut into several segments combines its segments' partial sums
+// deterministically: each writes its partial to its workspace slot, and the last segment to
+// finish (per-row arrival counter) adds all partials in segment order into Y.
+constexpr int kResSeg = 256;   // max residual nonzeros per work item
+constexpr int kResSlab = 256;  // features per residual launch (partial-sum slot width)
+struct ResSeg {
+  int64_t kb;        // first residual entry
+  int32_t row, len;  // packed row (local), #entries
+  int32_t slot;      // first workspace slot of the row's partials, -1 = single-segment row
+  int32_t split_id;  // arrival counter of the row (split rows only)
+  int32_t nseg, idx; // segments of the row, index of this one
+};
+
 }  // namespace nm
 
 struct nm_packed {
@@ -46,10 +79,13 @@ struct nm_packed {
   // device arrays
   int64_t* panel_mb_ptr = nullptr;     // [n_panels+1]
   int64_t* panel_chunk_ptr = nullptr;  // [n_panels+1]
-  int4* unit_info = nullptr;           // [n_panels] schedule: {panel, #chunks, first chunk lo, hi}
+  int4* unit_info = nullptr;           // [2 * n_panels] schedule: {panel, #chunks, first chunk lo, hi},
+                                       //   {record byte offset lo, hi, record bytes lo, hi}
+  uint16_t* rec_len16 = nullptr;       // [n_chunks] compressed record size / 16
+  int64_t image_bytes = 0;             // compressed image size
   int32_t* mb_seg = nullptr;           // [n_mb]
   uint32_t* mb_sel = nullptr;          // [n_mb] byte j = sel[j]
-  uint8_t* image = nullptr;            // [n_chunks * kChunkBytes] chunk records
+  uint8_t* image = nullptr;            // compressed chunk records (kRec* layout), image_bytes
   int64_t* res_rowptr = nullptr;       // [rows+1]
   int32_t* res_col = nullptr;          // [res_nnz] canonical (permuted) column
   uint16_t* res_val = nullptr;         // [res_nnz]
@@ -57,6 +93,12 @@ struct nm_packed {
   int flags = 0;
   int32_t* row_map = nullptr;          // [rows] output row of Y = perm[row_begin + l]
   int32_t* res_gather = nullptr;       // [res_nnz] X row to gather = perm[res_col]
+  // residual work list (kResSeg-entry segments) and the split rows' partial-sum workspace;
+  // the workspace makes concurrent nm_spmm calls on one handle unsafe (stream-order them)
+  nm::ResSeg* res_segs = nullptr;      // [n_res_segs]
+  int64_t n_res_segs = 0, n_res_slots = 0, n_res_split = 0;
+  float* res_ws = nullptr;             // [n_res_slots * kResSlab]
+  int32_t* res_cnt = nullptr;          // [n_res_split] arrival counters (0 between launches)
   size_t device_bytes = 0;
 };
 

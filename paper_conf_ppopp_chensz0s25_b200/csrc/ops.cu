@@ -8,93 +8,143 @@
 namespace nm {
 namespace {
 
-__device__ __forceinline__ float h2f(uint16_t b, int bf) {
-  if (bf) return __uint_as_float(((uint32_t)b) << 16);
-  __half h;
-  *(uint16_t*)&h = b;
-  return __half2float(h);
+// c + a * b with a, b 16-bit (fp16 or bf16 bits) and c fp32: one mixed-precision FMA
+// (FHFMA; the product of two 16-bit values is exact in fp32, so this equals converting both
+// and using an fp32 FMA)
+template <int BF>
+__device__ __forceinline__ float fma16(unsigned short a, unsigned short b, float c) {
+  float d;
+  if (BF)
+    asm("fma.rn.f32.bf16 %0, %1, %2, %3;" : "=f"(d) : "h"(a), "h"(b), "f"(c));
+  else
+    asm("fma.rn.f32.f16 %0, %1, %2, %3;" : "=f"(d) : "h"(a), "h"(b), "f"(c));
+  return d;
 }
 
 // Yp[l][f] += sum_k res_val[k] * PX[res_col[k]][f]  (the residual CSR, lossless remainder).
-// One warp per row.  The warp's lanes form SUB = 32 / LPR subgroups of LPR lanes; a subgroup
-// covers LPR * 8 features with one 16-byte X load per lane, and the subgroups take alternate
-// nonzeros of the row (so F = 128 keeps all 32 lanes busy with 16-byte loads).  The row's
+// One warp per work item (<= kResSeg nonzeros of one row, ResSeg), features [f0, f0 + LPR*8)
+// of this launch's slab.  The warp's lanes form SUB = 32 / LPR subgroups of LPR lanes; a
+// subgroup covers LPR * 8 features with one 16-byte X load per lane and the subgroups take
+// alternate nonzeros (so F = 128 keeps all 32 lanes busy with 16-byte loads).  The item's
 // (col, val) pairs are fetched 32 at a time with one coalesced load and broadcast with
-// shuffles; the nonzero loop is unrolled so several X rows are in flight per lane.  Partial
-// sums are combined across subgroups with xor-shuffles, then added into Y (fp32).
-// F tail: the 16-byte vector at column f0 < F is inside the row (ldx % 8 == 0), only the
+// shuffles; the loop is unrolled so several X rows are in flight per lane.  Subgroup partial
+// sums are combined with xor-shuffles.  A row with one item adds its sum into Y; the items of
+// a split row (hub rows) write partials to their workspace slots and the last one to arrive
+// (per-row counter) adds the partials in item order -- deterministic, no float atomics.
+// F tail: the 16-byte vector at column f < F is inside the row (ldx % 8 == 0), only the
 // accumulate/store is masked.
 template <int BF, int LPR>
-__global__ void __launch_bounds__(256) k_residual(const int64_t* __restrict__ rp, const int32_t* __restrict__ rc,
-                                                  const uint16_t* __restrict__ rv, int64_t rows,
+__global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ segs, int64_t n_segs,
+                                                  const int32_t* __restrict__ rc, const uint16_t* __restrict__ rv,
                                                   const int32_t* __restrict__ row_map,
                                                   const uint16_t* __restrict__ X, int64_t ldx,
-                                                  float* __restrict__ Y, int64_t ldy, int F) {
+                                                  float* __restrict__ Y, int64_t ldy, int F, int f_base,
+                                                  float* __restrict__ ws, int32_t* __restrict__ cnt) {
   constexpr int SUB = 32 / LPR;
   constexpr int kUnroll = 4;
   const int lane = threadIdx.x & 31;
   const int sub = lane / LPR, li = lane % LPR;
+  const int f = f_base + li * 8;  // first feature of this lane
   const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
   const bool vec_y = ((ldy & 3) == 0) && ((((uintptr_t)Y) & 15) == 0);
-  for (int64_t l = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; l < rows; l += nw) {
-    const int64_t b = rp[l], e = rp[l + 1];
-    if (b == e) continue;
-    float* yrow = Y + (row_map ? (int64_t)row_map[l] : l) * ldy;
-    for (int f0 = li * 8; f0 - li * 8 < F; f0 += LPR * 8) {
-      float acc[8];
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < n_segs; w += nw) {
+    const ResSeg g = segs[w];
+    float acc[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) acc[q] = 0.f;
+    for (int base = 0; base < g.len; base += 32) {
+      const int cnt_ = min(32, g.len - base);
+      int32_t c = 0;
+      uint32_t v = 0u;  // 16-bit value bits (a zero value adds exact zeros)
+      if (lane < cnt_) {
+        c = __ldg(rc + g.kb + base + lane);
+        v = __ldg(rv + g.kb + base + lane);
+      }
+      for (int j = 0; j < cnt_; j += SUB * kUnroll) {
+        uint4 xv[kUnroll];
+        uint32_t vv[kUnroll];
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+          const int idx = j + u * SUB + sub;
+          const int32_t cc = __shfl_sync(0xffffffffu, c, idx & 31);
+          vv[u] = __shfl_sync(0xffffffffu, v, idx & 31);
+          if (idx < cnt_ && f < F) {
+            xv[u] = __ldg((const uint4*)(X + (int64_t)cc * ldx + f));
+          } else {
+            xv[u] = make_uint4(0u, 0u, 0u, 0u);
+            vv[u] = 0u;
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+          const uint32_t wv[4] = {xv[u].x, xv[u].y, xv[u].z, xv[u].w};
+          const unsigned short a = (unsigned short)vv[u];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            acc[2 * q] = fma16<BF>(a, (unsigned short)(wv[q] & 0xFFFFu), acc[2 * q]);
+            acc[2 * q + 1] = fma16<BF>(a, (unsigned short)(wv[q] >> 16), acc[2 * q + 1]);
+          }
+        }
+      }
+    }
+#pragma unroll
+    for (int o = LPR; o < 32; o <<= 1)
+#pragma unroll
+      for (int q = 0; q < 8; ++q) acc[q] += __shfl_xor_sync(0xffffffffu, acc[q], o);
+    float* y = Y + (row_map ? (int64_t)row_map[g.row] : (int64_t)g.row) * ldy + f;
+    if (g.slot >= 0) {
+      // split row: publish this item's partial, the last arrival reduces in item order
+      float* part = ws + ((int64_t)(g.slot + g.idx) * kResSlab) + li * 8;
+      if (sub == 0) {
+        *(float4*)part = make_float4(acc[0], acc[1], acc[2], acc[3]);
+        *(float4*)(part + 4) = make_float4(acc[4], acc[5], acc[6], acc[7]);
+      }
+      __threadfence();
+      __syncwarp();
+      int last = 0;
+      if (lane == 0) last = atomicAdd(cnt + g.split_id, 1) == g.nseg - 1;
+      last = __shfl_sync(0xffffffffu, last, 0);
+      if (!last) continue;
+      __threadfence();
 #pragma unroll
       for (int q = 0; q < 8; ++q) acc[q] = 0.f;
-      for (int64_t base = b; base < e; base += 32) {
-        const int cnt = (int)min((int64_t)32, e - base);
-        int32_t c = 0;
-        float v = 0.f;
-        if (lane < cnt) {
-          c = __ldg(rc + base + lane);
-          v = h2f(__ldg(rv + base + lane), BF);
+      // subgroup j sums the partials i = j (mod SUB), kUnroll loads in flight per lane; the
+      // assignment is fixed, so the summation order is too
+      for (int i0 = 0; i0 < g.nseg; i0 += SUB * kUnroll) {
+        float4 pa[kUnroll], pb[kUnroll];
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+          const int i = i0 + u * SUB + sub;
+          pa[u] = pb[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+          if (i < g.nseg) {
+            const float* pi = ws + ((int64_t)(g.slot + i) * kResSlab) + li * 8;
+            pa[u] = __ldcg((const float4*)pi);
+            pb[u] = __ldcg((const float4*)(pi + 4));
+          }
         }
-        for (int j = 0; j < cnt; j += SUB * kUnroll) {
-          uint4 xv[kUnroll];
-          float vv[kUnroll];
 #pragma unroll
-          for (int u = 0; u < kUnroll; ++u) {
-            const int idx = j + u * SUB + sub;
-            const int32_t cc = __shfl_sync(0xffffffffu, c, idx & 31);
-            vv[u] = __shfl_sync(0xffffffffu, v, idx & 31);
-            if (idx < cnt && f0 < F)
-              xv[u] = __ldg((const uint4*)(X + (int64_t)cc * ldx + f0));
-            else {
-              xv[u] = make_uint4(0u, 0u, 0u, 0u);
-              vv[u] = 0.f;
-            }
-          }
-#pragma unroll
-          for (int u = 0; u < kUnroll; ++u) {
-            const uint32_t w[4] = {xv[u].x, xv[u].y, xv[u].z, xv[u].w};
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              acc[2 * q] += vv[u] * h2f((uint16_t)(w[q] & 0xFFFF), BF);
-              acc[2 * q + 1] += vv[u] * h2f((uint16_t)(w[q] >> 16), BF);
-            }
-          }
+        for (int u = 0; u < kUnroll; ++u) {
+          acc[0] += pa[u].x; acc[1] += pa[u].y; acc[2] += pa[u].z; acc[3] += pa[u].w;
+          acc[4] += pb[u].x; acc[5] += pb[u].y; acc[6] += pb[u].z; acc[7] += pb[u].w;
         }
       }
 #pragma unroll
       for (int o = LPR; o < 32; o <<= 1)
 #pragma unroll
         for (int q = 0; q < 8; ++q) acc[q] += __shfl_xor_sync(0xffffffffu, acc[q], o);
-      if (sub == 0 && f0 < F) {
-        float* y = yrow + f0;
-        if (vec_y && f0 + 8 <= F) {
-          float4 y0 = *(float4*)y, y1 = *(float4*)(y + 4);
-          y0.x += acc[0]; y0.y += acc[1]; y0.z += acc[2]; y0.w += acc[3];
-          y1.x += acc[4]; y1.y += acc[5]; y1.z += acc[6]; y1.w += acc[7];
-          *(float4*)y = y0;
-          *(float4*)(y + 4) = y1;
-        } else {
+      if (lane == 0) cnt[g.split_id] = 0;  // ready for the next launch
+    }
+    if (sub == 0 && f < F) {
+      if (vec_y && f + 8 <= F) {
+        float4 y0 = *(float4*)y, y1 = *(float4*)(y + 4);
+        y0.x += acc[0]; y0.y += acc[1]; y0.z += acc[2]; y0.w += acc[3];
+        y1.x += acc[4]; y1.y += acc[5]; y1.z += acc[6]; y1.w += acc[7];
+        *(float4*)y = y0;
+        *(float4*)(y + 4) = y1;
+      } else {
 #pragma unroll
-          for (int q = 0; q < 8; ++q)
-            if (f0 + q < F) y[q] += acc[q];
-        }
+        for (int q = 0; q < 8; ++q)
+          if (f + q < F) y[q] += acc[q];
       }
     }
   }
@@ -163,21 +213,26 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
   const int64_t rows = P->row_end - P->row_begin;
   if (P->res_nnz == 0 || rows == 0) return NM_OK;
   const int32_t* rcol = P->res_gather ? P->res_gather : P->res_col;
-  // lanes per row-slice: 8 features per lane, at most one warp per slice
+  // lanes per item: 8 features per lane; one launch per slab of LPR * 8 features
   const int lpr = F <= 32 ? 4 : F <= 64 ? 8 : F <= 128 ? 16 : 32;
-#define NM_RES_LAUNCH(BF, LPR)                                                                       \
-  k_residual<BF, LPR><<<grid_rows(rows, 8), 256, 0, s>>>(P->res_rowptr, rcol, P->res_val, rows, P->row_map, \
-                                                         (const uint16_t*)PX, ldx, Yp, ldy, F)
   const int bf = P->dtype == NM_BF16;
-  switch (lpr * 2 + bf) {
-    case 8: NM_RES_LAUNCH(0, 4); break;
-    case 9: NM_RES_LAUNCH(1, 4); break;
-    case 16: NM_RES_LAUNCH(0, 8); break;
-    case 17: NM_RES_LAUNCH(1, 8); break;
-    case 32: NM_RES_LAUNCH(0, 16); break;
-    case 33: NM_RES_LAUNCH(1, 16); break;
-    case 64: NM_RES_LAUNCH(0, 32); break;
-    default: NM_RES_LAUNCH(1, 32); break;
+  int64_t g = (P->n_res_segs + 7) / 8;
+  if (g > 148 * 16) g = 148 * 16;
+#define NM_RES_LAUNCH(BF, LPR)                                                                            \
+  k_residual<BF, LPR><<<(unsigned)g, 256, 0, s>>>(P->res_segs, P->n_res_segs, rcol, P->res_val, P->row_map, \
+                                                  (const uint16_t*)PX, ldx, Yp, ldy, F, f_base, P->res_ws,      \
+                                                  P->res_cnt)
+  for (int f_base = 0; f_base < F; f_base += lpr * 8) {
+    switch (lpr * 2 + bf) {
+      case 8: NM_RES_LAUNCH(0, 4); break;
+      case 9: NM_RES_LAUNCH(1, 4); break;
+      case 16: NM_RES_LAUNCH(0, 8); break;
+      case 17: NM_RES_LAUNCH(1, 8); break;
+      case 32: NM_RES_LAUNCH(0, 16); break;
+      case 33: NM_RES_LAUNCH(1, 16); break;
+      case 64: NM_RES_LAUNCH(0, 32); break;
+      default: NM_RES_LAUNCH(1, 32); break;
+    }
   }
 #undef NM_RES_LAUNCH
   NM_CUDA(cudaGetLastError());

@@ -370,6 +370,122 @@ __global__ void k_res_fill(const int64_t* __restrict__ Brp, const int32_t* __res
   }
 }
 
+// Compression of the full chunk records into the HBM form (nm_internal.h kRec* layout).
+// One 128-thread block per chunk, thread r = row r.  WRITE = false: record sizes only.
+template <bool WRITE>
+__global__ void __launch_bounds__(128) k_compress(const uint8_t* __restrict__ full, int64_t n_chunks,
+                                                  int64_t* __restrict__ size16, const int64_t* __restrict__ off,
+                                                  uint8_t* __restrict__ out) {
+  __shared__ int s_ne[4], s_nr[4];
+  const int r = threadIdx.x, lane = r & 31, q = r >> 5;
+  for (int64_t c = blockIdx.x; c < n_chunks; c += gridDim.x) {
+    const uint8_t* rec = full + c * kChunkBytes;
+    const uint32_t* meta = (const uint32_t*)(rec + kChunkValBytes);
+    uint32_t vals[kChunkMB];
+    uint32_t W = 0, mask = 0;
+#pragma unroll
+    for (int g = 0; g < kChunkMB; ++g) {
+      const uint32_t v0 = *(const uint16_t*)(rec + val_off(r, 2 * g));
+      const uint32_t v1 = *(const uint16_t*)(rec + val_off(r, 2 * g + 1));
+      int w, sh;
+      meta_pos(r, g, &w, &sh);
+      const uint32_t nb = (meta[w] >> sh) & 0xFu;
+      W |= nb << (4 * g);
+      vals[g] = v0 | (v1 << 16);
+      if (!(nb == 0x4u && v0 == 0 && v1 == 0)) mask |= 1u << g;
+    }
+    const int ne = __popc(mask), nr = mask != 0;
+    int ve = ne, vn = nr;  // inclusive warp scans
+    for (int o = 1; o < 32; o <<= 1) {
+      const int a = __shfl_up_sync(0xffffffffu, ve, o), b = __shfl_up_sync(0xffffffffu, vn, o);
+      if (lane >= o) { ve += a; vn += b; }
+    }
+    if (lane == 31) { s_ne[q] = ve; s_nr[q] = vn; }
+    __syncthreads();
+    int qv = 0, qn = 0, NE = 0, NR = 0;
+    for (int j = 0; j < 4; ++j) {
+      if (j < q) { qv += s_ne[j]; qn += s_nr[j]; }
+      NE += s_ne[j];
+      NR += s_nr[j];
+    }
+    const int bytes = (kRecHdrBytes + 4 * (NE + NR) + 15) & ~15;
+    if (!WRITE) {
+      if (r == 0) size16[c] = bytes / 16;
+    } else {
+      uint8_t* dst = out + off[c];
+      if (r < 32) ((int32_t*)dst)[r] = ((const int32_t*)(rec + kChunkXrowOff))[r];
+      dst[kRecMaskOff + r] = (uint8_t)mask;
+      if (lane == 0) {
+        ((uint16_t*)(dst + kRecQvOff))[q] = (uint16_t)qv;
+        ((uint16_t*)(dst + kRecQnOff))[q] = (uint16_t)qn;
+      }
+      if (r < 4) ((uint32_t*)(dst + kRecTotOff))[r] = r == 0 ? ((uint32_t)NE | ((uint32_t)NR << 16)) : 0u;
+      __syncthreads();  // the zeroed header word above before the contiguity byte below
+      if (r < 4) {  // gather rows 8r..8r+7 consecutive rows of X?
+        const int32_t* xr = (const int32_t*)(rec + kChunkXrowOff) + 8 * r;
+        bool cont = xr[0] >= 0;
+        for (int j = 1; j < 8; ++j) cont = cont && xr[j] == xr[0] + j;
+        if (cont) atomicOr((unsigned int*)(dst + kRecTotOff + 4), 1u << r);
+      }
+      uint32_t* dv = (uint32_t*)(dst + kRecHdrBytes);
+      int e = qv + ve - ne;  // exclusive offset of this row's first entry
+#pragma unroll
+      for (int g = 0; g < kChunkMB; ++g)
+        if (mask & (1u << g)) dv[e++] = vals[g];
+      if (nr) dv[NE + qn + vn - 1] = W;
+      const int used = kRecHdrBytes + 4 * (NE + NR);
+      if (r < (bytes - used) / 4) ((uint32_t*)(dst + used))[r] = 0u;  // padding
+    }
+    __syncthreads();
+  }
+}
+
+// residual work list: per row #segments, #partial slots (split rows only), split flag
+__global__ void k_seg_count(const int64_t* __restrict__ rrp, int64_t rows, int64_t* __restrict__ nseg,
+                            int64_t* __restrict__ nslot, int64_t* __restrict__ nsplit) {
+  for (int64_t l = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; l < rows; l += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t len = rrp[l + 1] - rrp[l];
+    const int64_t k = (len + kResSeg - 1) / kResSeg;
+    nseg[l] = k;
+    nslot[l] = k > 1 ? k : 0;
+    nsplit[l] = k > 1 ? 1 : 0;
+  }
+}
+
+__global__ void k_seg_fill(const int64_t* __restrict__ rrp, int64_t rows, const int64_t* __restrict__ seg_ptr,
+                           const int64_t* __restrict__ slot_ptr, const int64_t* __restrict__ split_ptr,
+                           ResSeg* __restrict__ segs) {
+  for (int64_t l = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; l < rows; l += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = rrp[l], len = rrp[l + 1] - b;
+    const int64_t k = seg_ptr[l + 1] - seg_ptr[l];
+    for (int64_t i = 0; i < k; ++i) {
+      ResSeg g;
+      g.kb = b + i * kResSeg;
+      g.row = (int32_t)l;
+      g.len = (int32_t)min((int64_t)kResSeg, len - i * kResSeg);
+      g.slot = k > 1 ? (int32_t)slot_ptr[l] : -1;
+      g.split_id = k > 1 ? (int32_t)split_ptr[l] : -1;
+      g.nseg = (int32_t)k;
+      g.idx = (int32_t)i;
+      segs[seg_ptr[l] + i] = g;
+    }
+  }
+}
+
+__global__ void k_seg_key(const ResSeg* __restrict__ segs, int64_t n, uint32_t* __restrict__ key,
+                          int32_t* __restrict__ idx) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    key[i] = (uint32_t)(kResSeg - segs[i].len);  // ascending key = longest first
+    idx[i] = (int32_t)i;
+  }
+}
+
+__global__ void k_seg_gather(const ResSeg* __restrict__ in, const int32_t* __restrict__ idx, int64_t n,
+                             ResSeg* __restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = in[idx[i]];
+}
+
 struct DevBuf {
   void* p = nullptr;
   cudaStream_t s = nullptr;
@@ -601,41 +717,22 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   const int64_t n_chunks = chp[P];
   Pk->n_chunks = n_chunks;
 
-  // unit schedule: natural panel order (consecutive panels run concurrently on the persistent
-  // grid, so their X neighbourhoods are shared in L2); NM_UNIT_ORDER=heavy sorts by chunk
-  // count instead.  One 16-byte descriptor per panel: {panel, #chunks, first chunk}.
-  {
-    std::vector<int32_t> order(P);
-    std::iota(order.begin(), order.end(), 0);
-    const char* ord = getenv("NM_UNIT_ORDER");
-    if (ord && std::string(ord) == "heavy")
-      std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
-        return (chp[a + 1] - chp[a]) > (chp[b + 1] - chp[b]);
-      });
-    std::vector<int4> info(P);
-    for (int64_t j = 0; j < P; ++j) {
-      const int32_t r = order[j];
-      const int64_t c0 = chp[r];
-      info[j] = make_int4(r, (int32_t)(chp[r + 1] - c0), (int32_t)(c0 & 0xFFFFFFFF), (int32_t)(c0 >> 32));
-    }
-    NM_TRY(palloc((void**)&Pk->unit_info, sizeof(int4) * P));
-    NM_CUDA(cudaMemcpyAsync(Pk->unit_info, info.data(), sizeof(int4) * P, cudaMemcpyHostToDevice, s));
-    NM_CUDA(cudaStreamSynchronize(s));
-  }
-
   NM_TRY(palloc((void**)&Pk->mb_seg, sizeof(int32_t) * n_mb));
   NM_TRY(palloc((void**)&Pk->mb_sel, sizeof(uint32_t) * n_mb));
-  NM_TRY(palloc((void**)&Pk->image, (size_t)kChunkBytes * n_chunks));
-  NM_CUDA(cudaMemsetAsync(Pk->image, 0, (size_t)kChunkBytes * n_chunks, s));
+  // the full MMA-layout records are assembled in a scratch buffer, then compressed (step 5)
+  DevBuf d_full;
+  NM_TRY(dalloc(d_full, (size_t)kChunkBytes * n_chunks, s));
+  uint8_t* full = d_full.as<uint8_t>();
   if (n_chunks) {
-    k_meta_init<<<grid_for(n_chunks * 128, 256), 256, 0, s>>>(Pk->image, n_chunks);
-    k_xrow_map<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(nullptr, Pk->image, n_chunks);
+    NM_CUDA(cudaMemsetAsync(full, 0, (size_t)kChunkBytes * n_chunks, s));
+    k_meta_init<<<grid_for(n_chunks * 128, 256), 256, 0, s>>>(full, n_chunks);
+    k_xrow_map<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(nullptr, full, n_chunks);
   }
   if (n_mb) {
     NM_CUDA(cudaMemcpyAsync(Pk->mb_sel, selv, sizeof(uint32_t) * n_mb, cudaMemcpyDeviceToDevice, s));
     k_write_sel<<<grid_for(n_mb, 256), 256, 0, s>>>(d_cnt.as<int32_t>(), d_cand_of.p ? d_cand_of.as<int64_t>() : nullptr,
                                                     Mp, n_mb, mbkey, S, n, Pk->panel_mb_ptr, Pk->panel_chunk_ptr,
-                                                    Pk->mb_seg, Pk->mb_sel, Pk->image);
+                                                    Pk->mb_seg, Pk->mb_sel, full);
   }
   NM_CUDA(cudaGetLastError());
 
@@ -648,7 +745,7 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   NM_CUDA(cudaMemsetAsync(d_rc.p, 0, sizeof(int64_t) * (rows + 1), s));
   if (bnnz) {
     k_place<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, Bval, rows, Mp, d_emb.as<int64_t>(), Pk->mb_sel,
-                                                    Pk->panel_mb_ptr, Pk->panel_chunk_ptr, Pk->image,
+                                                    Pk->panel_mb_ptr, Pk->panel_chunk_ptr, full,
                                                     d_flag.as<uint8_t>(), d_kept.as<unsigned long long>());
     k_res_count<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, d_flag.as<uint8_t>(), rows, d_rc.as<int64_t>());
   }
@@ -668,6 +765,54 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     k_res_fill<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, Bval, d_flag.as<uint8_t>(), rows,
                                                        Pk->res_rowptr, Pk->res_col, Pk->res_val);
   NM_CUDA(cudaGetLastError());
+  if (res_nnz) {
+    // residual work list (kResSeg-entry segments) + the split rows' workspace
+    DevBuf d_nseg, d_nslot, d_nsplit, d_segp, d_slotp, d_splitp;
+    for (DevBuf* b : {&d_nseg, &d_nslot, &d_nsplit, &d_segp, &d_slotp, &d_splitp})
+      NM_TRY(dalloc(*b, sizeof(int64_t) * (rows + 1), s));
+    NM_CUDA(cudaMemsetAsync(d_nseg.p, 0, sizeof(int64_t) * (rows + 1), s));
+    NM_CUDA(cudaMemsetAsync(d_nslot.p, 0, sizeof(int64_t) * (rows + 1), s));
+    NM_CUDA(cudaMemsetAsync(d_nsplit.p, 0, sizeof(int64_t) * (rows + 1), s));
+    k_seg_count<<<grid_for(rows, 256), 256, 0, s>>>(Pk->res_rowptr, rows, d_nseg.as<int64_t>(),
+                                                    d_nslot.as<int64_t>(), d_nsplit.as<int64_t>());
+    NM_TRY(scan_excl(d_nseg.as<int64_t>(), d_segp.as<int64_t>(), rows + 1, s));
+    NM_TRY(scan_excl(d_nslot.as<int64_t>(), d_slotp.as<int64_t>(), rows + 1, s));
+    NM_TRY(scan_excl(d_nsplit.as<int64_t>(), d_splitp.as<int64_t>(), rows + 1, s));
+    int64_t tot[3];
+    NM_CUDA(cudaMemcpyAsync(&tot[0], d_segp.as<int64_t>() + rows, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    NM_CUDA(cudaMemcpyAsync(&tot[1], d_slotp.as<int64_t>() + rows, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    NM_CUDA(cudaMemcpyAsync(&tot[2], d_splitp.as<int64_t>() + rows, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    NM_CUDA(cudaStreamSynchronize(s));
+    Pk->n_res_segs = tot[0];
+    Pk->n_res_slots = tot[1];
+    Pk->n_res_split = tot[2];
+    NM_TRY(palloc((void**)&Pk->res_segs, sizeof(ResSeg) * tot[0]));
+    NM_TRY(palloc((void**)&Pk->res_ws, sizeof(float) * kResSlab * tot[1]));
+    NM_TRY(palloc((void**)&Pk->res_cnt, sizeof(int32_t) * tot[2]));
+    NM_CUDA(cudaMemsetAsync(Pk->res_cnt, 0, sizeof(int32_t) * (tot[2] > 0 ? tot[2] : 1), s));
+    DevBuf d_segs, d_k1, d_k2, d_i1, d_i2;
+    NM_TRY(dalloc(d_segs, sizeof(ResSeg) * tot[0], s));
+    k_seg_fill<<<grid_for(rows, 256), 256, 0, s>>>(Pk->res_rowptr, rows, d_segp.as<int64_t>(), d_slotp.as<int64_t>(),
+                                                   d_splitp.as<int64_t>(), d_segs.as<ResSeg>());
+    // longest work items first (a stable sort by length): the persistent grid's first wave
+    // takes the hub rows' items, so they do not form the kernel's tail
+    NM_TRY(dalloc(d_k1, sizeof(uint32_t) * tot[0], s));
+    NM_TRY(dalloc(d_k2, sizeof(uint32_t) * tot[0], s));
+    NM_TRY(dalloc(d_i1, sizeof(int32_t) * tot[0], s));
+    NM_TRY(dalloc(d_i2, sizeof(int32_t) * tot[0], s));
+    k_seg_key<<<grid_for(tot[0], 256), 256, 0, s>>>(d_segs.as<ResSeg>(), tot[0], d_k1.as<uint32_t>(), d_i1.as<int32_t>());
+    {
+      size_t bytes = 0;
+      NM_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, bytes, d_k1.as<uint32_t>(), d_k2.as<uint32_t>(),
+                                              d_i1.as<int32_t>(), d_i2.as<int32_t>(), tot[0], 0, 9, s));
+      DevBuf tmp;
+      NM_TRY(dalloc(tmp, bytes, s));
+      NM_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, bytes, d_k1.as<uint32_t>(), d_k2.as<uint32_t>(),
+                                              d_i1.as<int32_t>(), d_i2.as<int32_t>(), tot[0], 0, 9, s));
+    }
+    k_seg_gather<<<grid_for(tot[0], 256), 256, 0, s>>>(d_segs.as<ResSeg>(), d_i2.as<int32_t>(), tot[0], Pk->res_segs);
+    NM_CUDA(cudaGetLastError());
+  }
   if (flags & NM_PACK_ORIGINAL_ORDER) {
     // fold P into the operand indices: gather X[perm[q]], write Y[perm[p]]
     Pk->flags = flags;
@@ -675,13 +820,64 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     NM_TRY(palloc((void**)&Pk->res_gather, sizeof(int32_t) * res_nnz));
     const int32_t* pm = d_perm.as<int32_t>();
     k_map<<<grid_for(rows, 256), 256, 0, s>>>(pm + rb, Pk->row_map, rows, 1);
-    if (n_chunks) k_xrow_map<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(pm, Pk->image, n_chunks);
+    if (n_chunks) k_xrow_map<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(pm, full, n_chunks);
     if (res_nnz) {
       NM_CUDA(cudaMemcpyAsync(Pk->res_gather, Pk->res_col, sizeof(int32_t) * res_nnz, cudaMemcpyDeviceToDevice, s));
       k_map<<<grid_for(res_nnz, 256), 256, 0, s>>>(pm, Pk->res_gather, res_nnz, 0);
     }
     NM_CUDA(cudaGetLastError());
   }
+  // ---- 5. compression of the records (HBM form) ----
+  std::vector<int64_t> coff(n_chunks + 1, 0);
+  {
+    DevBuf d_sz, d_off;
+    NM_TRY(dalloc(d_sz, sizeof(int64_t) * (n_chunks + 1), s));
+    NM_TRY(dalloc(d_off, sizeof(int64_t) * (n_chunks + 1), s));
+    NM_CUDA(cudaMemsetAsync(d_sz.p, 0, sizeof(int64_t) * (n_chunks + 1), s));
+    const int cgrid = (int)std::min<int64_t>(std::max<int64_t>(n_chunks, 1), 148 * 16);
+    if (n_chunks)
+      k_compress<false><<<cgrid, 128, 0, s>>>(full, n_chunks, d_sz.as<int64_t>(), nullptr, nullptr);
+    NM_TRY(scan_excl(d_sz.as<int64_t>(), d_off.as<int64_t>(), n_chunks + 1, s));
+    NM_CUDA(cudaMemcpyAsync(coff.data(), d_off.p, sizeof(int64_t) * (n_chunks + 1), cudaMemcpyDeviceToHost, s));
+    NM_CUDA(cudaStreamSynchronize(s));
+    for (auto& o : coff) o *= 16;  // units of 16 bytes -> bytes
+    NM_CUDA(cudaMemcpyAsync(d_off.p, coff.data(), sizeof(int64_t) * (n_chunks + 1), cudaMemcpyHostToDevice, s));
+    Pk->image_bytes = coff[n_chunks];
+    NM_TRY(palloc((void**)&Pk->image, (size_t)Pk->image_bytes));
+    std::vector<uint16_t> len16(n_chunks > 0 ? n_chunks : 1);
+    for (int64_t c = 0; c < n_chunks; ++c) len16[c] = (uint16_t)((coff[c + 1] - coff[c]) / 16);
+    NM_TRY(palloc((void**)&Pk->rec_len16, sizeof(uint16_t) * len16.size()));
+    NM_CUDA(cudaMemcpyAsync(Pk->rec_len16, len16.data(), sizeof(uint16_t) * len16.size(), cudaMemcpyHostToDevice, s));
+    if (n_chunks)
+      k_compress<true><<<cgrid, 128, 0, s>>>(full, n_chunks, nullptr, d_off.as<int64_t>(), Pk->image);
+    NM_CUDA(cudaGetLastError());
+    NM_CUDA(cudaStreamSynchronize(s));
+  }
+
+  // unit schedule: natural panel order (consecutive panels run concurrently on the persistent
+  // grid, so their X neighbourhoods are shared in L2); NM_UNIT_ORDER=heavy sorts by chunk
+  // count instead.  One 16-byte descriptor per panel: {panel, #chunks, first chunk}.
+  {
+    std::vector<int32_t> order(P);
+    std::iota(order.begin(), order.end(), 0);
+    const char* ord = getenv("NM_UNIT_ORDER");
+    if (ord && std::string(ord) == "heavy")
+      std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+        return (chp[a + 1] - chp[a]) > (chp[b + 1] - chp[b]);
+      });
+    std::vector<int4> info(2 * P);
+    for (int64_t j = 0; j < P; ++j) {
+      const int32_t r = order[j];
+      const int64_t c0 = chp[r], b0 = coff[c0], b1 = coff[chp[r + 1]];
+      info[2 * j] = make_int4(r, (int32_t)(chp[r + 1] - c0), (int32_t)(c0 & 0xFFFFFFFF), (int32_t)(c0 >> 32));
+      info[2 * j + 1] = make_int4((int32_t)(b0 & 0xFFFFFFFF), (int32_t)(b0 >> 32), (int32_t)((b1 - b0) & 0xFFFFFFFF),
+                                  (int32_t)((b1 - b0) >> 32));
+    }
+    NM_TRY(palloc((void**)&Pk->unit_info, sizeof(int4) * 2 * P));
+    NM_CUDA(cudaMemcpyAsync(Pk->unit_info, info.data(), sizeof(int4) * 2 * P, cudaMemcpyHostToDevice, s));
+    NM_CUDA(cudaStreamSynchronize(s));
+  }
+
   NM_CUDA(cudaStreamSynchronize(s));
   guard.ok = true;
   *out = Pk;

@@ -3,21 +3,27 @@
 // One work unit = (panel of 128 rows of B, 64..256-column tile of F).  The K dimension of a
 // panel is its list of non-empty meta-blocks; 8 meta-blocks (4 selected columns each) form
 // one K = 32 chunk, i.e. one tcgen05.mma.sp.cta_group::1.kind::f16 with M = 128, N = BN:
-//   record (A values, 2:4 metadata, 32 gather rows; 4736 B) <- one cp.async.bulk (HBM stream)
+//   record (compressed chunk, nm_internal.h kRec*)  <- one cp.async.bulk (HBM stream)
+//   A (128 x 16 physical values, K-major)          <- expanded from the record by the loaders
 //   B (32 gathered rows of X x BN, SWIZZLE_128B MN-major)  <- cp.async 16-byte gathers
-//   E (metadata, 128 lanes x 32 b)                          <- tcgen05.st from shared memory
-//   D (fp32, 128 x BN)                                      in tensor memory (tcgen05.ld out)
-// Warp roles (persistent, one CTA per SM, 18 warps):
-//   w0 record TMA + L2 prefetch of the next units' records
-//   w1-8 loaders, two groups of 4 warps taking alternate chunks: X gathers + metadata
-//   w9 MMA issuer (+ TMEM allocation)
-//   w10-17 epilogue, two warps per TMEM lane quarter: tcgen05.ld 16x256b -> 32-byte
+//   E (metadata, 128 lanes x 32 b)                  <- tcgen05.st of the expanded nibbles
+//   D (fp32, 128 x BN)                              in tensor memory (tcgen05.ld out)
+// The record is the paper's matrix put "into the SPTC required form on the fly" (L492): HBM
+// holds only the non-empty (row, meta-block) slots; the dense operand exists only in SMEM.
+// Warp roles (persistent, one CTA per SM, 22 warps):
+//   w0 record TMA (own ring of kRecSlots) + L2 prefetch of the next units' records
+//   w1-12 loaders, three groups of 4 warps, group g owns the stages s = g (mod 3): X gathers,
+//         record expansion into the A tile, metadata into TMEM
+//   w13 MMA issuer (+ TMEM allocation)
+//   w14-21 epilogue, two warps per TMEM lane quarter: tcgen05.ld 16x256b -> 32-byte
 //   sector-aligned stores of Y rows (no shared-memory staging).
 // All hand-offs are mbarriers; the pipeline runs across work units, so consecutive panels
-// overlap, and every role prefetches the next unit's 16-byte schedule entry.  Design
-// evidence: TMA tile::gather4 costs ~57 cycles per instruction on B200, so X
-// rows are gathered with cp.async; a single loader group spent ~950 cycles per chunk
-// (clock64 timeline, tools/trace_spmm.py), so two groups alternate.
+// overlap, and every role prefetches the next unit's schedule entry.  Design evidence
+// (DESIGN.md §6): TMA tile::gather4 costs ~57 cycles per instruction on B200, so X rows are
+// gathered with cp.async; one loader group spent ~950 cycles per chunk (clock64 timeline,
+// tools/trace_spmm.py), so three groups share the stages.
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 
@@ -37,10 +43,18 @@ constexpr int kWarpMma = kWarpLoad0 + 4 * kLoadGroups, kWarpEpi0 = kWarpMma + 1,
 constexpr int kThreads = (kWarpEpi0 + kEpiWarps) * 32;  // 576
 constexpr int kGroupThreads = 128;                     // loader threads per group
 constexpr int kPrefetchUnits = 2;                      // record L2-prefetch distance (units)
+// compressed records land in a byte ring of kRecRing bytes (allocated in chunk order; a
+// record that runs past the end continues into a kRecMaxBytes pad, so every record is
+// contiguous without skipping) described by kRecSlots descriptors; descriptor i % kRecSlots
+// belongs to chunk i, so loader group g only ever waits on descriptors = g (mod 3)
+constexpr int kRecSlots = 10 * kLoadGroups;
+constexpr int kRecRing = 32 * 1024;  // power of two
+constexpr int kIssueLanes = 8;       // records whose bulk copies are issued together
 
 struct SpmmParams {
   const uint8_t* image;
-  const int4* unit_info;   // per scheduled panel: {panel, #chunks, first chunk lo, hi}
+  const int4* unit_info;   // 2 per scheduled panel: {panel, #chunks, first chunk lo, hi}, {byte off, bytes}
+  const uint16_t* rec_len16;  // compressed record size / 16 per chunk
   const int32_t* row_map;  // nullable: output row of Y for packed row l
   const uint16_t* X;
   int64_t ldx;
@@ -66,6 +80,22 @@ struct SpmmParams {
   } while (0)
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ uint32_t lds8(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ uint32_t lds16(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ void sts128(uint32_t a, uint32_t x, uint32_t y, uint32_t z, uint32_t w) {
+  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(x), "r"(y), "r"(z), "r"(w) : "memory");
+}
 
 __device__ __forceinline__ uint32_t lds32(uint32_t a) {
   uint32_t v;
@@ -116,52 +146,67 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t
   return d;
 }
 
-// schedule entry of unit u (prefetched one unit ahead by every role)
+// schedule entry of unit u (prefetched one unit ahead by every role): {panel, #chunks, c0}
 __device__ __forceinline__ int4 unit_entry(const SpmmParams& p, int64_t u) {
-  return u < p.n_units ? __ldg(p.unit_info + u / p.n_ftiles) : make_int4(0, 0, 0, 0);
+  return u < p.n_units ? __ldg(p.unit_info + 2 * (u / p.n_ftiles)) : make_int4(0, 0, 0, 0);
+}
+// {record byte offset lo, hi, record bytes lo, hi} of unit u
+__device__ __forceinline__ int4 unit_bytes(const SpmmParams& p, int64_t u) {
+  return u < p.n_units ? __ldg(p.unit_info + 2 * (u / p.n_ftiles) + 1) : make_int4(0, 0, 0, 0);
 }
 __device__ __forceinline__ int64_t entry_c0(int4 e) { return (int64_t)(uint32_t)e.z | ((int64_t)e.w << 32); }
+__device__ __forceinline__ int64_t lo_hi(int a, int b) { return (int64_t)(uint32_t)a | ((int64_t)b << 32); }
 
 template <int BN>
 struct Cfg {
-  static constexpr int kRecBytes = kChunkBytes;                 // 4736
+  static constexpr int kABytes = kChunkValBytes;                // 128 x 16 values (4096)
   static constexpr int kBBytes = 32 * BN * 2;                   // 32 K-rows x BN halves
-  static constexpr int kStageBytes = kRecBytes + kBBytes;
-  static constexpr int kStagesRaw = (214 * 1024) / kStageBytes;
+  static constexpr int kStageBytes = kABytes + kBBytes;
+  static constexpr int kRecRegion = kRecRing + kRecMaxBytes;
+  static constexpr int kStagesRaw = (214 * 1024 - kRecRegion) / kStageBytes;
   // a multiple of the loader-group count: group g owns stages s % kLoadGroups == g, so every
   // stage has one consumer group that visits it in chunk order (parity waits stay valid)
   static constexpr int kStages = ((kStagesRaw > 16 ? 16 : kStagesRaw) / kLoadGroups) * kLoadGroups;
   static constexpr int kNAcc = (2 * BN + kStages <= 512) ? 2 : 1;
   static constexpr int kMeta0 = kNAcc * BN;                     // metadata column of stage s: kMeta0 + s
-  static constexpr int kRecRegion = ((kStages * kRecBytes + 1023) / 1024) * 1024;
-  static constexpr int kSmem = 1024 + kRecRegion + kStages * kBBytes + 1024;
+  static constexpr int kBRegion = kStages * kBBytes;            // 1024-aligned tiles (SW128)
+  static constexpr int kSmem = 1024 + kBRegion + kStages * kABytes + kRecRegion + 2048;
   static_assert(kMeta0 + kStages <= 512, "TMEM budget");
   static_assert(BN % 64 == 0 && BN >= 64 && BN <= 256, "BN");
   static_assert(kSmem <= 227 * 1024, "smem");
+  static_assert(kRecSlots % kLoadGroups == 0 && kRecMaxBytes % 16 == 0 && kRecRing >= 2 * kRecMaxBytes,
+                "record ring");
 };
 
 template <int BN>
-__global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
+__global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, const __grid_constant__ CUtensorMap tmX) {
   using C = Cfg<BN>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  const uint32_t sRec = smem_u32(smem);      // kStages records (16-byte aligned)
-  const uint32_t sB = sRec + C::kRecRegion;  // kStages B tiles (1024-aligned)
-  uint64_t* bars = (uint64_t*)(smem + C::kRecRegion + C::kStages * C::kBBytes);
-  uint64_t* full_a = bars;                  // record landed (tx)
-  uint64_t* full_b = bars + C::kStages;     // gathers + metadata ready
-  uint64_t* empty = bars + 2 * C::kStages;  // MMA done with the stage (tcgen05.commit)
-  uint64_t* tfull = bars + 3 * C::kStages;  // accumulator ready (2)
+  const uint32_t sB = smem_u32(smem);                  // kStages B tiles (1024-aligned)
+  const uint32_t sA = sB + C::kBRegion;                // kStages A tiles
+  const uint32_t sRec = sA + C::kStages * C::kABytes;  // kRecSlots compressed records
+  uint64_t* bars = (uint64_t*)(smem + C::kBRegion + C::kStages * C::kABytes + C::kRecRegion);
+  uint64_t* rec_full = bars;                // record landed (tx)
+  uint64_t* rec_empty = bars + kRecSlots;   // record expanded by its loader group
+  uint64_t* full_b = rec_empty + kRecSlots; // A tile + gathers + metadata ready
+  uint64_t* empty = full_b + C::kStages;    // MMA done with the stage (tcgen05.commit)
+  uint64_t* tfull = empty + C::kStages;     // accumulator ready (2)
   uint64_t* tempty = tfull + 2;             // accumulator drained (2)
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  uint32_t* rec_off = tmem_slot + 4;        // [kRecSlots] ring offset of each descriptor's record
+  uint32_t* rec_end = rec_off + kRecSlots;  // [kRecSlots] producer-private: cumulative end of each record
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
 
   if (threadIdx.x == 0) {
+    for (int s = 0; s < kRecSlots; ++s) {
+      mbar_init(smem_u32(&rec_full[s]), 1);
+      mbar_init(smem_u32(&rec_empty[s]), kGroupThreads);
+    }
     for (int s = 0; s < C::kStages; ++s) {
-      mbar_init(smem_u32(&full_a[s]), 1);
-      mbar_init(smem_u32(&full_b[s]), 2 * kGroupThreads);  // cp.async completions + metadata stores
+      mbar_init(smem_u32(&full_b[s]), 2 * kGroupThreads);  // cp.async completions + A/metadata stores
       mbar_init(smem_u32(&empty[s]), 1);
     }
     for (int a = 0; a < 2; ++a) {
@@ -182,85 +227,202 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
 
   if (warp == kWarpRec) {
     // ------------------------------------------------------------ record producer (HBM stream)
-    if (lane == 0) {
-      int64_t i = 0;
-      int4 nxt = unit_entry(p, blockIdx.x);
-      // the records of a panel are contiguous: stream the next units' records into L2 ahead
-      // of their bulk copies (one bulk prefetch per unit, kPrefetchUnits units ahead)
-      auto prefetch_unit = [&](int4 e) {
-        if (e.y > 0)
-          asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p.image + entry_c0(e) * kChunkBytes),
-                       "r"((uint32_t)(e.y * kChunkBytes))
-                       : "memory");
-      };
-      for (int k = 0; k < kPrefetchUnits; ++k) prefetch_unit(unit_entry(p, blockIdx.x + k * ustep));
-      int s = 0;
-      uint32_t ph = 0;
-      for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
-        const int4 cur = nxt;
-        nxt = unit_entry(p, u + ustep);
-        prefetch_unit(unit_entry(p, u + kPrefetchUnits * ustep));
-        const int64_t c0 = entry_c0(cur), c1 = c0 + cur.y;
-        for (int64_t c = c0; c < c1; ++c, ++i) {
-          mbar_wait(smem_u32(&empty[s]), ph ^ 1);
-          NM_TRACE(0);
-          mbar_arrive_tx(smem_u32(&full_a[s]), C::kRecBytes);
-          bulk_g2s(sRec + s * C::kRecBytes, p.image + c * kChunkBytes, C::kRecBytes, smem_u32(&full_a[s]));
-          if (++s == C::kStages) { s = 0; ph ^= 1; }
+    // the warp reads the record sizes of 32 chunks at a time (one unit ahead); lane 0
+    // allocates ring space -- waiting, oldest first, for the loader groups to release older
+    // records -- and issues the bulk copies.  Lane 0's per-record path is kept short (32-bit
+    // wrapping counters, no divisions): it is a serial chain on one thread.
+    uint32_t head = 0, tail = 0;       // cumulative ring bytes allocated / released (mod 2^32)
+    int ds = 0, os = 0;                // next descriptor to fill / oldest one not yet released
+    uint32_t oph = 0;                  // use parity of the oldest descriptor
+    int in_flight = 0;                 // records issued and not yet known to be released
+    int64_t i = 0;                     // chunk counter (trace only)
+    auto prefetch_unit = [&](int4 b) {  // the records of a panel are contiguous: one L2 prefetch
+      const int64_t len = lo_hi(b.z, b.w);
+      if (lane == 0 && len > 0)
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p.image + lo_hi(b.x, b.y)),
+                     "r"((uint32_t)len)
+                     : "memory");
+    };
+    auto first_lens = [&](int4 e) -> uint32_t {  // sizes of a unit's first 32 records (lane j)
+      return lane < e.y ? 16u * __ldg(p.rec_len16 + entry_c0(e) + lane) : 0u;
+    };
+    for (int k = 0; k < kPrefetchUnits; ++k) prefetch_unit(unit_bytes(p, blockIdx.x + k * ustep));
+    int4 nxt = unit_entry(p, blockIdx.x), nxtb = unit_bytes(p, blockIdx.x);
+    int4 pfb = unit_bytes(p, blockIdx.x + kPrefetchUnits * ustep);
+    uint32_t nlen = first_lens(nxt);
+    for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
+      const int4 cur = nxt, curb = nxtb;
+      uint32_t len = nlen;
+      nxt = unit_entry(p, u + ustep);
+      nxtb = unit_bytes(p, u + ustep);
+      prefetch_unit(pfb);
+      pfb = unit_bytes(p, u + (kPrefetchUnits + 1) * ustep);
+      const int64_t c0 = entry_c0(cur);
+      const int nch = cur.y;
+      int64_t boff = lo_hi(curb.x, curb.y);
+      for (int b0 = 0; b0 < nch; b0 += 32) {
+        const int cnt = min(32, nch - b0);
+        if (b0 > 0) len = lane < cnt ? 16u * __ldg(p.rec_len16 + c0 + b0 + lane) : 0u;
+        if (b0 + 32 >= nch) nlen = first_lens(nxt);  // next unit's sizes, ahead of use
+        uint32_t incl = len;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t a = __shfl_up_sync(0xffffffffu, incl, o);
+          if (lane >= o) incl += a;
         }
+        // sub-batches of up to kIssueLanes records: lane 0 makes room for all of them, then
+        // each lane issues its own record's bulk copy (the issues overlap across lanes)
+        const uint32_t excl = incl - len;
+        for (int sb = 0, m = 0; sb < cnt; sb += m) {
+          // the sub-batch: up to kIssueLanes records totalling at most half the ring
+          const uint32_t e0 = __shfl_sync(0xffffffffu, excl, sb);
+          m = __popc(__ballot_sync(0xffffffffu, lane >= sb && lane < sb + kIssueLanes && lane < cnt &&
+                                                    incl - e0 <= (uint32_t)(kRecRing / 2)));
+          const uint32_t total = __shfl_sync(0xffffffffu, incl, sb + m - 1) - e0;
+          if (lane == 0) {
+            while (head + total - tail > (uint32_t)kRecRing || in_flight + m > kRecSlots) {
+              mbar_wait(smem_u32(&rec_empty[os]), oph);
+              tail = rec_end[os];
+              --in_flight;
+              if (++os == kRecSlots) { os = 0; oph ^= 1; }
+            }
+          }
+          const uint32_t h0 = __shfl_sync(0xffffffffu, head, 0);
+          const int d0 = __shfl_sync(0xffffffffu, ds, 0);
+          if (lane >= sb && lane < sb + m) {
+            int d = d0 + (lane - sb);
+            if (d >= kRecSlots) d -= kRecSlots;
+            const uint32_t start = h0 + (excl - e0);
+            const uint32_t pos = start & (uint32_t)(kRecRing - 1);
+            rec_end[d] = start + len;
+            rec_off[d] = pos;
+            mbar_arrive_tx(smem_u32(&rec_full[d]), len);
+            bulk_g2s(sRec + pos, p.image + boff + excl, len, smem_u32(&rec_full[d]));
+          }
+          if (lane == 0) {
+            if (p.trace && blockIdx.x == 0 && i < 1024) p.trace[i * 8] = clock64();
+            head += total;
+            in_flight += m;
+            ds += m;
+            if (ds >= kRecSlots) ds -= kRecSlots;
+          }
+          i += m;
+          __syncwarp();
+        }
+        boff += __shfl_sync(0xffffffffu, incl, cnt - 1);
       }
     }
   } else if (warp >= kWarpLoad0 && warp < kWarpLoad0 + 4 * kLoadGroups) {
-    // ------------------------------------------------------------ loaders: X gathers + metadata
+    // ------------------------------------------------------------ loaders: X gathers, record
+    // expansion (A tile) and metadata
     const int group = (warp - kWarpLoad0) >> 2;  // owns the stages s with s % kLoadGroups == group
     const int quarter = warp & 3;                               // TMEM lane quarter of this warp
     const int t = threadIdx.x - (kWarpLoad0 + 4 * group) * 32;  // 0..127 within the group
-    const int L = quarter * 32 + lane;                          // TMEM lane this thread writes
-    const int k = t >> 2;                                       // gathered row (logical K index)
-    const int sub = t & 3;
+    const int r = quarter * 32 + lane;                          // A row (= TMEM lane) this thread expands
     constexpr int kRowPieces = BN / 8;  // 16-byte pieces per gathered row
-    constexpr int kPer = kRowPieces / 4;  // pieces per thread
+    constexpr int kPer = kRowPieces / 4;  // pieces per thread (32 rows x kRowPieces / 128 threads)
+    // metadata lane word of TMEM lane (quarter*32 + lane): rows r0 and r0 + 8 of the quarter
+    const int mr0 = (lane & 7) + 16 * (lane >> 4), mk1 = (lane >> 3) & 1;
+    const uint32_t arow = (uint32_t)((r & 7) * 16 + (r >> 3) * 256);
     int64_t i = 0;
-    int s_next = 0;
-    uint32_t ph_next = 0;
+    int s_next = 0, rs_next = 0;
+    uint32_t ph_next = 0, rph_next = 0;
     int4 nxt = unit_entry(p, blockIdx.x);
     for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
       const int4 cur = nxt;
       nxt = unit_entry(p, u + ustep);
       const int ft = (int)(u % p.n_ftiles);
-      const int64_t c0 = entry_c0(cur), c1 = c0 + cur.y;
-      for (int64_t c = c0; c < c1; ++c, ++i) {
-        const int s = s_next;
-        const uint32_t ph = ph_next;
+      const int nch = cur.y;
+      for (int c = 0; c < nch; ++c, ++i) {
+        const int s = s_next, rs = rs_next;
+        const uint32_t ph = ph_next, rph = rph_next;
         if (++s_next == C::kStages) { s_next = 0; ph_next ^= 1; }
+        if (++rs_next == kRecSlots) { rs_next = 0; rph_next ^= 1; }
         // stage ownership (not chunk round-robin): a group that skipped ahead could otherwise
         // test the parity of a stage two phases ahead and pass on a stale record
         if (s % kLoadGroups != group) continue;
-        mbar_wait(smem_u32(&full_a[s]), ph);
+        mbar_wait(smem_u32(&empty[s]), ph ^ 1);      // the MMA has finished with stage s
+        mbar_wait(smem_u32(&rec_full[rs]), rph);     // the compressed record has landed
         if (t == 0) NM_TRACE(1);
-        const uint32_t rec = sRec + s * C::kRecBytes;
-        const uint32_t brow = sB + s * C::kBBytes + (k >> 3) * 1024 + (k & 7) * 128;
-        int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * k);
-        if (p.debug & 1) xr = -1;
-        const uint16_t* xsrc = p.X + (int64_t)(xr < 0 ? 0 : xr) * p.ldx;
+        const uint32_t rec = sRec + rec_off[rs];
+        // 8-row groups of consecutive X rows come in by TMA tile loads (one 8 x 64 box per
+        // 64-column slab, written into the SW128 atom); the other rows by cp.async gathers
+        const uint32_t cmask = (p.debug & 32) ? 0u : lds8(rec + kRecContOff);
+        if (t == 0 && cmask) {
+          constexpr int kSlabs = BN / 64;
+          asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(&full_b[s])),
+                       "r"((uint32_t)(__popc(cmask) * kSlabs * 1024))
+                       : "memory");
+#pragma unroll
+          for (int g8 = 0; g8 < 4; ++g8) {
+            if (!((cmask >> g8) & 1u)) continue;
+            const int32_t row0 = (int32_t)lds32(rec + 32 * g8);
+#pragma unroll
+            for (int h = 0; h < kSlabs; ++h)
+              asm volatile(
+                  "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+                  " [%0], [%1, {%2, %3}], [%4];" ::"r"(sB + s * C::kBBytes + h * 4096 + g8 * 1024),
+                  "l"(&tmX), "r"(ft * BN + 64 * h), "r"(row0), "r"(smem_u32(&full_b[s]))
+                  : "memory");
+          }
+        }
+        // cp.async gathers: 16-byte pieces of the 32 rows x BN columns; piece P = q * 128 + t
+        // is row P / kRowPieces, column piece P % kRowPieces, so a warp instruction covers
+        // whole 128-byte lines of consecutive pieces of one or more rows
 #pragma unroll
         for (int q = 0; q < kPer; ++q) {
-          const int c16 = sub + 4 * q;
+          const int P = q * kGroupThreads + t;
+          const int kk = P / kRowPieces, c16 = P % kRowPieces;
+          if ((cmask >> (kk >> 3)) & 1u) continue;  // this row arrives by TMA
+          int32_t xr = (int32_t)lds32(rec + 4 * kk);
+          if (p.debug & 1) xr = -1;
           const int col0 = ft * BN + c16 * 8;
           uint32_t bytes = 0;
           if (xr >= 0 && col0 < p.F) {
             const int rem = p.F - col0;
             bytes = rem >= 8 ? 16u : (uint32_t)(rem * 2);
           }
-          const uint32_t dst = brow + (c16 >> 3) * 4096 + ((((uint32_t)c16 & 7u) ^ ((uint32_t)k & 7u)) << 4);
-          cp_async16(dst, bytes ? (const void*)(xsrc + col0) : (const void*)p.X, bytes);
+          const uint16_t* src = bytes ? p.X + (int64_t)xr * p.ldx + col0 : p.X;
+          const uint32_t dst = sB + s * C::kBBytes + (kk >> 3) * 1024 + (kk & 7) * 128 + (c16 >> 3) * 4096 +
+                               ((((uint32_t)c16 & 7u) ^ ((uint32_t)kk & 7u)) << 4);
+          cp_async16(dst, src, bytes);
         }
         // the barrier tracks this thread's gathers asynchronously (arrival when they land)
         asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&full_b[s])) : "memory");
-        const uint32_t w = lds32(rec + kChunkValBytes + 4 * L);
+        if (t == 0) NM_TRACE(4);
+        // expand row r of the record (its non-empty (row, group) value pairs and nibble word)
+        // into the A tile and the stage's TMEM metadata column
+        const uint32_t mask = lds8(rec + kRecMaskOff + r);
+        const int ne = __popc(mask), nr = mask != 0u;
+        int ve = ne, vn = nr;  // inclusive scans over the quarter's 32 rows
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int a = __shfl_up_sync(0xffffffffu, ve, o), b = __shfl_up_sync(0xffffffffu, vn, o);
+          if (lane >= o) { ve += a; vn += b; }
+        }
+        const int NE = (int)lds16(rec + kRecTotOff);
+        int e = (int)lds16(rec + kRecQvOff + 2 * quarter) + ve - ne;
+        const int wn = (int)lds16(rec + kRecQnOff + 2 * quarter) + vn - 1;
+        uint32_t v[kChunkMB];
+#pragma unroll
+        for (int g = 0; g < kChunkMB; ++g) {
+          v[g] = 0u;
+          if (mask & (1u << g)) v[g] = lds32(rec + kRecHdrBytes + 4 * (e++));
+        }
+        const uint32_t W = nr ? lds32(rec + kRecHdrBytes + 4 * (NE + wn)) : kMetaNone;
+        mbar_arrive(smem_u32(&rec_empty[rs]));  // every read of the record is done
+        if (t == 0) NM_TRACE(5);
+        // metadata word of this thread's TMEM lane: asynchronous store, waited for below
+        const uint32_t Wa = __shfl_sync(0xffffffffu, W, mr0), Wb = __shfl_sync(0xffffffffu, W, mr0 + 8);
+        const uint32_t word = ((Wa >> (16 * mk1)) & 0xFFFFu) | (((Wb >> (16 * mk1)) & 0xFFFFu) << 16);
         const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + s;
-        asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(w) : "memory");
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(word) : "memory");
+        const uint32_t at = sA + s * C::kABytes + arow;
+        sts128(at, v[0], v[1], v[2], v[3]);          // physical k 0..7
+        sts128(at + 128, v[4], v[5], v[6], v[7]);    // physical k 8..15 (LBO = 128)
+        if (t == 0) NM_TRACE(6);
         asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        if (t == 0) NM_TRACE(7);
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         mbar_arrive(smem_u32(&full_b[s]));
         if (t == 0) NM_TRACE(2);
@@ -275,7 +437,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
       uint32_t ph = 0;
       int acc = 0;
       uint32_t aphase = 0;
-      const uint64_t adesc0 = sdesc(sRec, 128, 256, 0);
+      const uint64_t adesc0 = sdesc(sA, 128, 256, 0);
       const uint64_t bdesc0 = sdesc(sB, 4096, 1024, 2);
       int4 nxt = unit_entry(p, blockIdx.x);
       for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
@@ -289,12 +451,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p) {
         for (int c = 0; c < nch; ++c, ++i) {
           mbar_wait(smem_u32(&full_b[s]), ph);
           NM_TRACE(3);
-          // the gathers were written through the generic proxy (cp.async): make them visible
-          // to the tensor core's async-proxy operand reads (without this fence stale stage
-          // contents were observed on B200 -- tests/test_parity_fullsize.py)
-          if (!(p.debug & 16)) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          // the A tile (st.shared) and the gathers (cp.async) were written through the generic
+          // proxy: make them visible to the tensor core's async-proxy operand reads (without
+          // this fence stale stage contents were observed on B200 -- test_parity_fullsize.py)
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          const uint64_t ad = adesc0 + (uint64_t)((s * C::kRecBytes) >> 4);
+          const uint64_t ad = adesc0 + (uint64_t)((s * C::kABytes) >> 4);
           const uint64_t bd = bdesc0 + (uint64_t)((s * C::kBBytes) >> 4);
           const uint32_t mcol = C::kMeta0 + s;
           const uint32_t ecol = tbase + (mcol & ~1u);   // even column address ...
@@ -435,6 +597,7 @@ nm_status launch_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, 
   SpmmParams prm;
   prm.image = P->image;
   prm.unit_info = P->unit_info;
+  prm.rec_len16 = P->rec_len16;
   prm.row_map = P->row_map;
   prm.X = (const uint16_t*)PX;
   prm.ldx = ldx;
@@ -455,7 +618,24 @@ nm_status launch_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, 
   }
   int64_t grid = prm.n_units < sms ? prm.n_units : sms;
   if (grid < 1) return NM_OK;
-  k_spmm_sptc<BN><<<(unsigned)grid, kThreads, C::kSmem, s>>>(prm);
+  // X as a 2-D tensor (F columns x n rows, ldx pitch) for the TMA tile loads of consecutive
+  // gather rows: 64 x 8 boxes, SWIZZLE_128B (the B tile's atom), out-of-range columns zero
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  if (!encode) {
+    cudaDriverEntryPointQueryResult q;
+    NM_CUDA(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void**)&encode, cudaEnableDefault, &q));
+    if (!encode || q != cudaDriverEntryPointSuccess) return fail(NM_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  }
+  CUtensorMap tm;
+  const cuuint64_t dims[2] = {(cuuint64_t)F, (cuuint64_t)P->n};
+  const cuuint64_t strides[1] = {(cuuint64_t)ldx * 2};
+  const cuuint32_t box[2] = {64, 8};
+  const cuuint32_t es[2] = {1, 1};
+  const CUresult er = encode(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, const_cast<void*>(PX), dims, strides, box, es,
+                             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                             CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (er != CUDA_SUCCESS) return fail(NM_ERR_CUDA, "cuTensorMapEncodeTiled failed for X");
+  k_spmm_sptc<BN><<<(unsigned)grid, kThreads, C::kSmem, s>>>(prm, tm);
   NM_CUDA(cudaGetLastError());
   if (prm.trace) {  // profiling aid only: synchronous dump of CTA 0's timeline
     NM_CUDA(cudaStreamSynchronize(s));

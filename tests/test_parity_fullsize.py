@@ -20,7 +20,7 @@ def test_deterministic_repeats_no_pipeline_races():
         pytest.skip("no CUDA device")
     import bench
     from paper_conf_ppopp_chensz0s25_b200 import api, graphs
-    w = bench.WORKLOADS["c2-powerlaw-n262k-d16-f128-1:2:4"]
+    w = bench.parse_workload("c2-powerlaw-n262k-d16-f128-1:2:4")
     ip, ic, vals, X32 = bench.make_graph(w)
     perm, _ = api.reorder(ip, ic, w["V"], 2, w["M"], max_outer=1)
     P = api.pack(ip, ic, perm, w["V"], 2, w["M"], dtype=w["dtype"], val=vals, order="original")
@@ -42,7 +42,7 @@ def test_bench_config_sampled_rows(workload):
         pytest.skip("no CUDA device")
     import bench
     from paper_conf_ppopp_chensz0s25_b200 import api, graphs
-    w = bench.WORKLOADS[workload]
+    w = bench.parse_workload(workload)
     ip, ic, vals, X32 = bench.make_graph(w)
     perm, st = api.reorder(ip, ic, w["V"], 2, w["M"])
     P = api.pack(ip, ic, perm, w["V"], 2, w["M"], dtype=w["dtype"], val=vals, order="original")

@@ -280,3 +280,51 @@ def test_spmm_hybrid_parity(kind, seed, V, M, tau):
     torch.cuda.synchronize()
     err = np.abs(Y.cpu().numpy().astype(np.float64) - Y_ref)
     assert (err <= TOL * E).all(), err.max()
+
+
+def _star_plus_er(n=3000, hubs=(0, 17), m=6000, seed=51):
+    """ER graph plus hub vertices adjacent to every other vertex: hub rows of degree ~n split
+    into several residual work items (kResSeg = 256 entries each)."""
+    ip, ic = graphs.er_graph(n, m, seed)
+    A = set()
+    for i in range(n):
+        for k in range(ip[i], ip[i + 1]):
+            A.add((i, int(ic[k])))
+    for h in hubs:
+        for v in range(n):
+            if v != h:
+                A.add((h, v))
+                A.add((v, h))
+    rows = np.array(sorted(A), dtype=np.int64)
+    ip2 = np.concatenate([[0], np.cumsum(np.bincount(rows[:, 0], minlength=n))]).astype(np.int64)
+    return ip2, rows[:, 1].astype(np.int32)
+
+
+@pytest.mark.parametrize("F", [32, 128, 300])
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+def test_residual_split_hub_rows(F, dtype):
+    """Everything in the residual (tau = inf): hub rows are cut into several work items whose
+    partials are combined deterministically -- parity and bitwise-identical repeats."""
+    dev = _cuda()
+    ip, ic = _star_plus_er()
+    n = len(ip) - 1
+    perm = np.random.default_rng(2).permutation(n).astype(np.int32)
+    v32, bits, v64 = _values(ip, ic, dtype, 3)
+    xbits, x64 = graphs.round16(graphs.features(n, F, 4), dtype)
+    Y_ref, E, _ = oracle.spmm(ip, ic, v64, x64)
+    tdt = torch.float16 if dtype == "f16" else torch.bfloat16
+    ldx = (F + 7) // 8 * 8
+    X = torch.zeros((n, ldx), dtype=torch.int16, device=dev)
+    X[:, :F] = torch.from_numpy(xbits.view(np.int16)).to(dev)
+    X = X.view(tdt)
+    P = api.pack(ip, ic, perm, 1, 2, 4, dtype=dtype, val=v32, order="original", tau=10 ** 9)
+    assert P.info()["n_mb"] == 0 and P.info()["residual_nnz"] == ip[-1]
+    outs = []
+    for _ in range(3):
+        Y = torch.full((n, F), float("nan"), device=dev)
+        api.spmm(P, X, Y, F=F)
+        torch.cuda.synchronize()
+        outs.append(Y.cpu().numpy())
+    err = np.abs(outs[0].astype(np.float64) - Y_ref)
+    assert (err <= TOL * E).all(), err.max()
+    assert all(np.array_equal(outs[0], o) for o in outs[1:])

@@ -10,7 +10,7 @@ import oracle  # noqa: E402
 from paper_conf_ppopp_chensz0s25_b200 import api, graphs  # noqa: E402
 
 wl = sys.argv[1] if len(sys.argv) > 1 else "c2-powerlaw-n262k-d16-f128-1:2:4"
-w = bench.WORKLOADS[wl]
+w = bench.parse_workload(wl)
 ip, ic, vals, X32 = bench.make_graph(w)
 n = w["n"]
 perm, st = api.reorder(ip, ic, w["V"], 2, w["M"])

@@ -21,7 +21,7 @@ def main():
     import bench
     from paper_conf_ppopp_chensz0s25_b200 import api, graphs
     wl = sys.argv[1] if len(sys.argv) > 1 else bench.DEFAULT
-    w = bench.WORKLOADS[wl]
+    w = bench.parse_workload(wl)
     ip, ic, vals, X32 = bench.make_graph(w)
     perm, _ = api.reorder(ip, ic, w["V"], 2, w["M"])
     P = api.pack(ip, ic, perm, w["V"], 2, w["M"], dtype=w["dtype"], val=vals, order="original")
@@ -37,11 +37,23 @@ def main():
     torch.cuda.synchronize()
     del os.environ["NM_SPMM_TRACE"]
     t = np.fromfile(path, dtype=np.uint64).astype(np.int64)
-    ch = t[:8192].reshape(1024, 8)[:, :4]
+    full = t[:8192].reshape(1024, 8)
+    ch = full[:, :4]
     un = t[8192:].reshape(2048, 4)
-    n = int((ch[:, 0] > 0).sum())
+    n = int((ch[:, 3] > 0).sum())  # chunks the MMA issued (the producer marks sub-batches only)
     ch = ch[:n]
     base = ch[0, 0]
+    ch[:, 0] = np.where(ch[:, 0] > 0, ch[:, 0], 0)
+    ch[:, 0] = np.maximum.accumulate(ch[:, 0])  # issue time of the sub-batch holding the chunk
+    # loader sub-steps (slots 1 -> 4 -> 5 -> 6 -> 7 -> 2): sees record, gathers issued, record
+    # expanded + released, A tile + tcgen05.st issued, tcgen05.wait::st done, arrived
+    sub = full[:n][:, [1, 4, 5, 6, 7, 2]]
+    own = sub[:, 0] > 0
+    if own.any():
+        d = np.diff(sub[own], axis=1)
+        for name, v in zip(["gathers issue", "expand+release", "A sts + tcgen05.st", "tcgen05.wait::st",
+                            "fence+arrive"], d.T):
+            print("loader %-22s median %6d  p90 %6d cycles" % (name, np.median(v), np.percentile(v, 90)))
     ch = ch - base
     print("chunks traced:", n)
     d_rec_ld = ch[:, 1] - ch[:, 0]
