@@ -217,7 +217,7 @@ NM_API nm_status nm_unpermute_rows(const void* Yp, void* Y, const int32_t* perm_
  * fp32 accumulation in tensor memory) plus the residual CSR (CUDA cores), i.e. exactly
  * (P A P^T)(P X) for the packed rows (the aggregation SpMM of L182, L492).
  *   PX : device, n x F, leading dimension ldx (elements), dtype of the pack, permuted order.
- *        ldx must be a multiple of 8 (16-byte rows).
+ *        ldx must be a multiple of 8 (16-byte rows) and below 2^31.
  *   Yp : device fp32, (row_end-row_begin) x F, leading dimension ldy; overwritten.
  *   F  : 1 <= F <= 4096.
  * Stream-ordered, asynchronous.  Errors: INVALID_ARG, UNSUPPORTED, CUDA. */

@@ -201,6 +201,7 @@ nm_status check_spmm_args(const nm_packed* P, const void* PX, int64_t ldx, float
   if (!P || !PX || !Yp) return fail(NM_ERR_INVALID_ARG, "nm_spmm: NULL argument");
   if (F < 1 || F > 4096) return fail(NM_ERR_UNSUPPORTED, "nm_spmm: F must be in [1, 4096]");
   if (ldx < F || ldy < F) return fail(NM_ERR_INVALID_ARG, "nm_spmm: leading dimension < F");
+  if (ldx > INT32_MAX) return fail(NM_ERR_UNSUPPORTED, "nm_spmm: ldx must fit in 32 bits");
   if (ldx % 8 != 0 || ((uintptr_t)PX & 15) != 0)
     return fail(NM_ERR_INVALID_ARG, "nm_spmm: PX rows must be 16-byte aligned (ldx % 8 == 0)");
   return NM_OK;

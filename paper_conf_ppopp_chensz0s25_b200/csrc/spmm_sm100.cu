@@ -39,16 +39,25 @@ namespace {
 #define NM_LOAD_GROUPS 3
 #endif
 constexpr int kWarpRec = 0, kWarpLoad0 = 1, kLoadGroups = NM_LOAD_GROUPS;
-constexpr int kWarpMma = kWarpLoad0 + 4 * kLoadGroups, kWarpEpi0 = kWarpMma + 1, kEpiWarps = 8;
-constexpr int kThreads = (kWarpEpi0 + kEpiWarps) * 32;  // 576
+#ifndef NM_EPI_WARPS
+#define NM_EPI_WARPS 8
+#endif
+constexpr int kWarpMma = kWarpLoad0 + 4 * kLoadGroups, kWarpEpi0 = kWarpMma + 1, kEpiWarps = NM_EPI_WARPS;
+constexpr int kThreads = (kWarpEpi0 + kEpiWarps) * 32;
+static_assert(kEpiWarps == 4 || kEpiWarps == 8, "epilogue: one or two warps per TMEM lane quarter");
 constexpr int kGroupThreads = 128;                     // loader threads per group
 constexpr int kPrefetchUnits = 2;                      // record L2-prefetch distance (units)
 // compressed records land in a byte ring of kRecRing bytes (allocated in chunk order; a
 // record that runs past the end continues into a kRecMaxBytes pad, so every record is
 // contiguous without skipping) described by kRecSlots descriptors; descriptor i % kRecSlots
 // belongs to chunk i, so loader group g only ever waits on descriptors = g (mod 3)
-constexpr int kRecSlots = 10 * kLoadGroups;
-constexpr int kRecRing = 32 * 1024;  // power of two
+#ifndef NM_REC_CPASYNC
+#define NM_REC_CPASYNC 0             // records by warp-wide cp.async instead of one bulk copy each
+#endif
+#ifndef NM_REC_SLOTS_PER_GROUP
+#define NM_REC_SLOTS_PER_GROUP 16
+#endif
+constexpr int kRecSlots = NM_REC_SLOTS_PER_GROUP * kLoadGroups;
 constexpr int kIssueLanes = 8;       // records whose bulk copies are issued together
 
 struct SpmmParams {
@@ -65,17 +74,27 @@ struct SpmmParams {
   int64_t n_units;
   int n_ftiles;
   uint32_t idesc;
-  int debug;                  // profiling switches (NM_SPMM_DEBUG): 1 = no gather reads, 2 = no Y stores
+  int debug;                  // profiling switches (NM_SPMM_DEBUG, results invalid): 2 = no Y stores,
+                              // 32 = no TMA row tiles, 64 = no record expansion, 128 = no
+                              // X gathers, 512 = no record
+                              // L2 prefetch, 1024 = no records (with 32|64|128 only)
   unsigned long long* trace;  // NM_SPMM_TRACE: per-chunk clock64 timeline of CTA 0
 };
 
+// clock64 timeline of CTA 0 (tools/trace_spmm.py): compiled in only with -DNM_SPMM_TRACE_BUILD
+// (NM_NVCC_FLAGS), so the product kernel carries no trace instructions
+#ifdef NM_SPMM_TRACE_BUILD
+#define NM_TRACE_ON 1
+#else
+#define NM_TRACE_ON 0
+#endif
 #define NM_TRACE(slot)                                                                              \
   do {                                                                                              \
-    if (p.trace && blockIdx.x == 0 && i < 1024) p.trace[i * 8 + (slot)] = clock64();                \
+    if (NM_TRACE_ON && p.trace && blockIdx.x == 0 && i < 1024) p.trace[i * 8 + (slot)] = clock64(); \
   } while (0)
 #define NM_TRACE_U(slot)                                                                            \
   do {                                                                                              \
-    if (p.trace && blockIdx.x == 0 && lane == 0 && (u / ustep) < 1024)                               \
+    if (NM_TRACE_ON && p.trace && blockIdx.x == 0 && lane == 0 && (u / ustep) < 1024)               \
       p.trace[8192 + (u / ustep) * 4 + (slot)] = clock64();                                         \
   } while (0)
 
@@ -117,6 +136,23 @@ __device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) {
       : "memory");
 }
 
+// long waits (the epilogue waiting for a whole unit of MMAs): back off so the spinning warps
+// do not take issue slots from the loaders (ncu: 20% of executed instructions were this spin)
+__device__ __forceinline__ void mbar_wait_sleep(uint32_t a, uint32_t parity) {
+  uint32_t ok;
+  for (;;) {
+    asm volatile(
+        "{\n\t.reg .pred P;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, P;\n\t}"
+        : "=r"(ok)
+        : "r"(a), "r"(parity)
+        : "memory");
+    if (ok) return;
+    __nanosleep(200);
+  }
+}
+
 __device__ __forceinline__ void mbar_arrive(uint32_t a) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(a) : "memory");
 }
@@ -134,6 +170,15 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t
 
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, uint32_t src_bytes) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+
+// 16-byte cp.async whose source is ignored (destination zero-filled) when ign is true
+__device__ __forceinline__ void cp_async16_ign(uint32_t dst, const void* src, bool ign) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t"
+      "cp.async.cg.shared.global [%0], [%1], 16, q;\n\t}" ::"r"(dst),
+      "l"(src), "r"((int)ign)
+      : "memory");
 }
 
 __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t sbo, uint32_t layout) {
@@ -162,11 +207,14 @@ struct Cfg {
   static constexpr int kABytes = kChunkValBytes;                // 128 x 16 values (4096)
   static constexpr int kBBytes = 32 * BN * 2;                   // 32 K-rows x BN halves
   static constexpr int kStageBytes = kABytes + kBBytes;
-  static constexpr int kRecRegion = kRecRing + kRecMaxBytes;
-  static constexpr int kStagesRaw = (214 * 1024 - kRecRegion) / kStageBytes;
+  static constexpr int kStagesRaw = (214 * 1024 - 32 * 1024 - kRecMaxBytes) / kStageBytes;
   // a multiple of the loader-group count: group g owns stages s % kLoadGroups == g, so every
   // stage has one consumer group that visits it in chunk order (parity waits stay valid)
   static constexpr int kStages = ((kStagesRaw > 16 ? 16 : kStagesRaw) / kLoadGroups) * kLoadGroups;
+  // the record ring takes what the stages leave (largest power of two, >= 32 KB)
+  static constexpr int kRingAvail = 214 * 1024 - kStages * kStageBytes - kRecMaxBytes;
+  static constexpr int kRecRing = kRingAvail >= 128 * 1024 ? 128 * 1024 : kRingAvail >= 64 * 1024 ? 64 * 1024 : 32 * 1024;
+  static constexpr int kRecRegion = kRecRing + kRecMaxBytes;
   static constexpr int kNAcc = (2 * BN + kStages <= 512) ? 2 : 1;
   static constexpr int kMeta0 = kNAcc * BN;                     // metadata column of stage s: kMeta0 + s
   static constexpr int kBRegion = kStages * kBBytes;            // 1024-aligned tiles (SW128)
@@ -197,21 +245,26 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
   uint32_t* rec_off = tmem_slot + 4;        // [kRecSlots] ring offset of each descriptor's record
   uint32_t* rec_end = rec_off + kRecSlots;  // [kRecSlots] producer-private: cumulative end of each record
 
+  // shared-window addresses of the barrier arrays (index i at base + 8 i)
+  const uint32_t bRecFull = smem_u32(rec_full), bRecEmpty = smem_u32(rec_empty);
+  const uint32_t bFull = smem_u32(full_b), bEmpty = smem_u32(empty);
+  const uint32_t bTfull = smem_u32(tfull), bTempty = smem_u32(tempty);
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < kRecSlots; ++s) {
-      mbar_init(smem_u32(&rec_full[s]), 1);
-      mbar_init(smem_u32(&rec_empty[s]), kGroupThreads);
+      mbar_init(smem_u32(&rec_full[s]), NM_REC_CPASYNC ? 32 : 1);  // cp.async lanes / one expect_tx
+      mbar_init(smem_u32(&rec_empty[s]), kGroupThreads / 32);  // one arrival per loader warp
     }
     for (int s = 0; s < C::kStages; ++s) {
-      mbar_init(smem_u32(&full_b[s]), 2 * kGroupThreads);  // cp.async completions + A/metadata stores
+      // per-thread cp.async completions + one arrival per loader warp (A tile / metadata written)
+      mbar_init(smem_u32(&full_b[s]), kGroupThreads + kGroupThreads / 32);
       mbar_init(smem_u32(&empty[s]), 1);
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(smem_u32(&tfull[a]), 1);
-      mbar_init(smem_u32(&tempty[a]), kEpiWarps * 32);
+      mbar_init(smem_u32(&tempty[a]), kEpiWarps);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -236,9 +289,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
     uint32_t oph = 0;                  // use parity of the oldest descriptor
     int in_flight = 0;                 // records issued and not yet known to be released
     int64_t i = 0;                     // chunk counter (trace only)
+    int nsb = 0;                       // sub-batch counter (trace only)
     auto prefetch_unit = [&](int4 b) {  // the records of a panel are contiguous: one L2 prefetch
       const int64_t len = lo_hi(b.z, b.w);
-      if (lane == 0 && len > 0)
+      if (lane == 0 && len > 0 && !(p.debug & 512))
         asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p.image + lo_hi(b.x, b.y)),
                      "r"((uint32_t)len)
                      : "memory");
@@ -247,23 +301,31 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
       return lane < e.y ? 16u * __ldg(p.rec_len16 + entry_c0(e) + lane) : 0u;
     };
     for (int k = 0; k < kPrefetchUnits; ++k) prefetch_unit(unit_bytes(p, blockIdx.x + k * ustep));
-    int4 nxt = unit_entry(p, blockIdx.x), nxtb = unit_bytes(p, blockIdx.x);
+    // schedule lookahead: entries two units ahead, record sizes one unit ahead (from an entry
+    // that is already in registers), so no HBM round trip sits between two units' issues
+    int4 e1 = unit_entry(p, blockIdx.x), b1 = unit_bytes(p, blockIdx.x);
+    int4 e2 = unit_entry(p, blockIdx.x + ustep), b2 = unit_bytes(p, blockIdx.x + ustep);
     int4 pfb = unit_bytes(p, blockIdx.x + kPrefetchUnits * ustep);
-    uint32_t nlen = first_lens(nxt);
+    uint32_t nlen = first_lens(e1);
     for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
-      const int4 cur = nxt, curb = nxtb;
+      NM_TRACE_U(0);
+      const int4 cur = e1, curb = b1;
       uint32_t len = nlen;
-      nxt = unit_entry(p, u + ustep);
-      nxtb = unit_bytes(p, u + ustep);
+      e1 = e2;
+      b1 = b2;
+      e2 = unit_entry(p, u + 2 * ustep);
+      b2 = unit_bytes(p, u + 2 * ustep);
+      nlen = first_lens(e1);
       prefetch_unit(pfb);
       pfb = unit_bytes(p, u + (kPrefetchUnits + 1) * ustep);
       const int64_t c0 = entry_c0(cur);
       const int nch = cur.y;
       int64_t boff = lo_hi(curb.x, curb.y);
-      for (int b0 = 0; b0 < nch; b0 += 32) {
+      uint32_t blen = 0;  // sizes of the next batch of 32 records of this unit, one batch ahead
+      for (int b0 = 0; b0 < ((p.debug & 1024) ? 0 : nch); b0 += 32) {
         const int cnt = min(32, nch - b0);
-        if (b0 > 0) len = lane < cnt ? 16u * __ldg(p.rec_len16 + c0 + b0 + lane) : 0u;
-        if (b0 + 32 >= nch) nlen = first_lens(nxt);  // next unit's sizes, ahead of use
+        if (b0 > 0) len = blen;
+        if (b0 + 32 < nch) blen = lane < nch - b0 - 32 ? 16u * __ldg(p.rec_len16 + c0 + b0 + 32 + lane) : 0u;
         uint32_t incl = len;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -277,30 +339,61 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
           // the sub-batch: up to kIssueLanes records totalling at most half the ring
           const uint32_t e0 = __shfl_sync(0xffffffffu, excl, sb);
           m = __popc(__ballot_sync(0xffffffffu, lane >= sb && lane < sb + kIssueLanes && lane < cnt &&
-                                                    incl - e0 <= (uint32_t)(kRecRing / 2)));
+                                                    incl - e0 <= (uint32_t)(C::kRecRing / 2)));
           const uint32_t total = __shfl_sync(0xffffffffu, incl, sb + m - 1) - e0;
+          if (NM_TRACE_ON && p.trace && blockIdx.x == 0 && lane == 0 && nsb < 1024) {
+            p.trace[12288 + 4 * nsb] = clock64();
+            p.trace[12290 + 4 * nsb] = ((uint64_t)in_flight << 32) | (head - tail);
+          }
           if (lane == 0) {
-            while (head + total - tail > (uint32_t)kRecRing || in_flight + m > kRecSlots) {
-              mbar_wait(smem_u32(&rec_empty[os]), oph);
+            int nw = 0;
+            while (head + total - tail > (uint32_t)C::kRecRing || in_flight + m > kRecSlots) {
+              ++nw;
+              mbar_wait(bRecEmpty + 8 * os, oph);
               tail = rec_end[os];
               --in_flight;
               if (++os == kRecSlots) { os = 0; oph ^= 1; }
             }
+            if (NM_TRACE_ON && p.trace && blockIdx.x == 0 && nsb < 1024) {
+              p.trace[12289 + 4 * nsb] = clock64();
+              p.trace[12291 + 4 * nsb] = ((uint64_t)nw << 32) | (uint32_t)m;
+            }
           }
+          ++nsb;
           const uint32_t h0 = __shfl_sync(0xffffffffu, head, 0);
           const int d0 = __shfl_sync(0xffffffffu, ds, 0);
+#if NM_REC_CPASYNC
+          // records through the LSU: the warp copies each record with 16-byte cp.async (512 B
+          // per instruction) and every lane's cp.async.mbarrier.arrive.noinc marks it landed
+          for (int k = 0; k < m; ++k) {
+            int d = d0 + k;
+            if (d >= kRecSlots) d -= kRecSlots;
+            const uint32_t ek = __shfl_sync(0xffffffffu, excl, sb + k);
+            const uint32_t lk = __shfl_sync(0xffffffffu, len, sb + k);
+            const uint32_t start = h0 + (ek - e0);
+            const uint32_t pos = start & (uint32_t)(C::kRecRing - 1);
+            if (lane == 0) {
+              rec_end[d] = start + lk;
+              rec_off[d] = pos;
+            }
+            const uint8_t* src = p.image + boff + ek;
+            for (uint32_t o = 16u * lane; o < lk; o += 512u) cp_async16(sRec + pos + o, src + o, 16u);
+            asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bRecFull + 8 * d) : "memory");
+          }
+#else
           if (lane >= sb && lane < sb + m) {
             int d = d0 + (lane - sb);
             if (d >= kRecSlots) d -= kRecSlots;
             const uint32_t start = h0 + (excl - e0);
-            const uint32_t pos = start & (uint32_t)(kRecRing - 1);
+            const uint32_t pos = start & (uint32_t)(C::kRecRing - 1);
             rec_end[d] = start + len;
             rec_off[d] = pos;
-            mbar_arrive_tx(smem_u32(&rec_full[d]), len);
-            bulk_g2s(sRec + pos, p.image + boff + excl, len, smem_u32(&rec_full[d]));
+            mbar_arrive_tx(bRecFull + 8 * d, len);
+            bulk_g2s(sRec + pos, p.image + boff + excl, len, bRecFull + 8 * d);
           }
+#endif
           if (lane == 0) {
-            if (p.trace && blockIdx.x == 0 && i < 1024) p.trace[i * 8] = clock64();
+            if (NM_TRACE_ON && p.trace && blockIdx.x == 0 && i < 1024) p.trace[i * 8] = clock64();
             head += total;
             in_flight += m;
             ds += m;
@@ -321,96 +414,134 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
     const int r = quarter * 32 + lane;                          // A row (= TMEM lane) this thread expands
     constexpr int kRowPieces = BN / 8;  // 16-byte pieces per gathered row
     constexpr int kPer = kRowPieces / 4;  // pieces per thread (32 rows x kRowPieces / 128 threads)
+    constexpr bool kFixedCol = kGroupThreads % kRowPieces == 0;
+    constexpr int kRowsPerPass = kGroupThreads / kRowPieces;
+    const int c16f = t % kRowPieces, kk0 = t / kRowPieces;
+    const uint32_t dcol16 = (uint32_t)(c16f >> 3) * 4096u;
+    const int32_t ldx32 = (int32_t)p.ldx;
     // metadata lane word of TMEM lane (quarter*32 + lane): rows r0 and r0 + 8 of the quarter
     const int mr0 = (lane & 7) + 16 * (lane >> 4), mk1 = (lane >> 3) & 1;
     const uint32_t arow = (uint32_t)((r & 7) * 16 + (r >> 3) * 256);
-    int64_t i = 0;
-    int s_next = 0, rs_next = 0;
-    uint32_t ph_next = 0, rph_next = 0;
+    // the group walks only its own chunks j = group (mod kLoadGroups) of the CTA's chunk
+    // sequence; stage j % kStages and record descriptor j % kRecSlots (both multiples of
+    // kLoadGroups, so they advance by kLoadGroups with a phase flip on wrap-around)
+    int64_t i = group, i0 = 0;  // next own chunk, first chunk of the current unit
+    int s = group, rs = group;
+    uint32_t ph = 0, rph = 0;
     int4 nxt = unit_entry(p, blockIdx.x);
     for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
       const int4 cur = nxt;
       nxt = unit_entry(p, u + ustep);
       const int ft = (int)(u % p.n_ftiles);
-      const int nch = cur.y;
-      for (int c = 0; c < nch; ++c, ++i) {
-        const int s = s_next, rs = rs_next;
-        const uint32_t ph = ph_next, rph = rph_next;
-        if (++s_next == C::kStages) { s_next = 0; ph_next ^= 1; }
-        if (++rs_next == kRecSlots) { rs_next = 0; rph_next ^= 1; }
-        // stage ownership (not chunk round-robin): a group that skipped ahead could otherwise
-        // test the parity of a stage two phases ahead and pass on a stale record
-        if (s % kLoadGroups != group) continue;
-        mbar_wait(smem_u32(&empty[s]), ph ^ 1);      // the MMA has finished with stage s
-        mbar_wait(smem_u32(&rec_full[rs]), rph);     // the compressed record has landed
+      // this thread's gather column piece (kFixedCol): source offset and byte count
+      const int col0f = ft * BN + c16f * 8;
+      const uint32_t colbytes = col0f >= p.F ? 0u : (p.F - col0f >= 8 ? 16u : (uint32_t)(p.F - col0f) * 2u);
+      const uint16_t* xcol = p.X + (colbytes ? col0f : 0);
+      const int64_t i_end = i0 + cur.y;
+      i0 = i_end;
+      for (; i < i_end; i += kLoadGroups) {
+        mbar_wait(bEmpty + 8 * s, ph ^ 1);       // the MMA has finished with stage s
+        if (t == 0) NM_TRACE(7);
+        if (!(p.debug & 1024)) mbar_wait(bRecFull + 8 * rs, rph);  // the compressed record has landed
         if (t == 0) NM_TRACE(1);
-        const uint32_t rec = sRec + rec_off[rs];
+        const uint32_t rec = sRec + ((p.debug & 1024) ? 0u : rec_off[rs]);
         // 8-row groups of consecutive X rows come in by TMA tile loads (one 8 x 64 box per
         // 64-column slab, written into the SW128 atom); the other rows by cp.async gathers
         const uint32_t cmask = (p.debug & 32) ? 0u : lds8(rec + kRecContOff);
-        if (t == 0 && cmask) {
+        if (t < 32 && cmask) {  // first warp of the group: one TMA tile load per lane
           constexpr int kSlabs = BN / 64;
-          asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(&full_b[s])),
-                       "r"((uint32_t)(__popc(cmask) * kSlabs * 1024))
-                       : "memory");
-#pragma unroll
-          for (int g8 = 0; g8 < 4; ++g8) {
-            if (!((cmask >> g8) & 1u)) continue;
+          if (t == 0)
+            asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(bFull + 8 * s),
+                         "r"((uint32_t)(__popc(cmask) * kSlabs * 1024))
+                         : "memory");
+          __syncwarp();
+          const int g8 = t / kSlabs, h = t % kSlabs;
+          if (g8 < 4 && ((cmask >> g8) & 1u)) {
             const int32_t row0 = (int32_t)lds32(rec + 32 * g8);
-#pragma unroll
-            for (int h = 0; h < kSlabs; ++h)
-              asm volatile(
-                  "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
-                  " [%0], [%1, {%2, %3}], [%4];" ::"r"(sB + s * C::kBBytes + h * 4096 + g8 * 1024),
-                  "l"(&tmX), "r"(ft * BN + 64 * h), "r"(row0), "r"(smem_u32(&full_b[s]))
-                  : "memory");
+            asm volatile(
+                "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+                " [%0], [%1, {%2, %3}], [%4];" ::"r"(sB + s * C::kBBytes + h * 4096 + g8 * 1024),
+                "l"(&tmX), "r"(ft * BN + 64 * h), "r"(row0), "r"(bFull + 8 * s)
+                : "memory");
           }
         }
         // cp.async gathers: 16-byte pieces of the 32 rows x BN columns; piece P = q * 128 + t
         // is row P / kRowPieces, column piece P % kRowPieces, so a warp instruction covers
         // whole 128-byte lines of consecutive pieces of one or more rows
+        if constexpr (kFixedCol) {
+          // BN = 64 / 128 / 256: the thread's column piece is the same for every q, so the
+          // source column, byte count and swizzle term are per-unit constants
+          const uint32_t sbase = sB + s * C::kBBytes + dcol16;
+          if (p.debug & 128) {
+            // profiling: no gathers
+          } else if (colbytes == 16u) {  // unit-uniform: full pieces, a zero row is an ignore-src zero fill
 #pragma unroll
-        for (int q = 0; q < kPer; ++q) {
-          const int P = q * kGroupThreads + t;
-          const int kk = P / kRowPieces, c16 = P % kRowPieces;
-          if ((cmask >> (kk >> 3)) & 1u) continue;  // this row arrives by TMA
-          int32_t xr = (int32_t)lds32(rec + 4 * kk);
-          if (p.debug & 1) xr = -1;
-          const int col0 = ft * BN + c16 * 8;
-          uint32_t bytes = 0;
-          if (xr >= 0 && col0 < p.F) {
-            const int rem = p.F - col0;
-            bytes = rem >= 8 ? 16u : (uint32_t)(rem * 2);
+            for (int q = 0; q < kPer; ++q) {
+              const int kk = q * kRowsPerPass + kk0;
+              if ((cmask >> (kk >> 3)) & 1u) continue;  // this row arrives by TMA
+              const int32_t xr = (int32_t)lds32(rec + 4 * kk);
+              cp_async16_ign(sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16f ^ (uint32_t)kk) & 7u) << 4),
+                             xcol + (int64_t)max(xr, 0) * ldx32, xr < 0);
+            }
+          } else {  // the F tail
+#pragma unroll
+            for (int q = 0; q < kPer; ++q) {
+              const int kk = q * kRowsPerPass + kk0;
+              if ((cmask >> (kk >> 3)) & 1u) continue;
+              const int32_t xr = (int32_t)lds32(rec + 4 * kk);
+              cp_async16(sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16f ^ (uint32_t)kk) & 7u) << 4),
+                         xcol + (int64_t)max(xr, 0) * ldx32, xr >= 0 ? colbytes : 0u);
+            }
           }
-          const uint16_t* src = bytes ? p.X + (int64_t)xr * p.ldx + col0 : p.X;
-          const uint32_t dst = sB + s * C::kBBytes + (kk >> 3) * 1024 + (kk & 7) * 128 + (c16 >> 3) * 4096 +
-                               ((((uint32_t)c16 & 7u) ^ ((uint32_t)kk & 7u)) << 4);
-          cp_async16(dst, src, bytes);
+        } else {
+#pragma unroll
+          for (int q = 0; q < kPer; ++q) {
+            const int P = q * kGroupThreads + t;
+            const int kk = P / kRowPieces, c16 = P % kRowPieces;
+            if ((cmask >> (kk >> 3)) & 1u) continue;  // this row arrives by TMA
+            const int32_t xr = (int32_t)lds32(rec + 4 * kk);
+            const int col0 = ft * BN + c16 * 8;
+            uint32_t bytes = 0;
+            if (xr >= 0 && col0 < p.F) {
+              const int rem = p.F - col0;
+              bytes = rem >= 8 ? 16u : (uint32_t)(rem * 2);
+            }
+            const uint16_t* src = bytes ? p.X + (int64_t)xr * ldx32 + col0 : p.X;
+            const uint32_t dst = sB + s * C::kBBytes + (kk >> 3) * 1024 + (kk & 7) * 128 + (c16 >> 3) * 4096 +
+                                 ((((uint32_t)c16 & 7u) ^ ((uint32_t)kk & 7u)) << 4);
+            cp_async16(dst, src, bytes);
+          }
         }
         // the barrier tracks this thread's gathers asynchronously (arrival when they land)
-        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&full_b[s])) : "memory");
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bFull + 8 * s) : "memory");
         if (t == 0) NM_TRACE(4);
         // expand row r of the record (its non-empty (row, group) value pairs and nibble word)
         // into the A tile and the stage's TMEM metadata column
-        const uint32_t mask = lds8(rec + kRecMaskOff + r);
+        const uint32_t mask = (p.debug & 64) ? 0u : lds8(rec + kRecMaskOff + r);
         const int ne = __popc(mask), nr = mask != 0u;
-        int ve = ne, vn = nr;  // inclusive scans over the quarter's 32 rows
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const int a = __shfl_up_sync(0xffffffffu, ve, o), b = __shfl_up_sync(0xffffffffu, vn, o);
-          if (lane >= o) { ve += a; vn += b; }
-        }
+        // inclusive prefix sums over the quarter's 32 rows from ballots (no shuffle chain):
+        // ne = sum of its bits 2^k, each bit's prefix is a popc of the ballot below this lane
+        uint32_t le;
+        asm("mov.u32 %0, %%lanemask_le;" : "=r"(le));
+        const int ve = __popc(__ballot_sync(0xffffffffu, ne & 1) & le) +
+                       2 * __popc(__ballot_sync(0xffffffffu, ne & 2) & le) +
+                       4 * __popc(__ballot_sync(0xffffffffu, ne & 4) & le) +
+                       8 * __popc(__ballot_sync(0xffffffffu, ne & 8) & le);
+        const int vn = __popc(__ballot_sync(0xffffffffu, nr) & le);
         const int NE = (int)lds16(rec + kRecTotOff);
         int e = (int)lds16(rec + kRecQvOff + 2 * quarter) + ve - ne;
         const int wn = (int)lds16(rec + kRecQnOff + 2 * quarter) + vn - 1;
+        // entry of (r, g) = e + #set bits of mask below g: independent loads, no serial chain
         uint32_t v[kChunkMB];
+        const uint32_t vbase = rec + kRecHdrBytes + 4 * e;
 #pragma unroll
         for (int g = 0; g < kChunkMB; ++g) {
           v[g] = 0u;
-          if (mask & (1u << g)) v[g] = lds32(rec + kRecHdrBytes + 4 * (e++));
+          if (mask & (1u << g)) v[g] = lds32(vbase + 4 * __popc(mask & ((1u << g) - 1u)));
         }
         const uint32_t W = nr ? lds32(rec + kRecHdrBytes + 4 * (NE + wn)) : kMetaNone;
-        mbar_arrive(smem_u32(&rec_empty[rs]));  // every read of the record is done
+        __syncwarp();  // every read of the record by this warp is done
+        if (lane == 0) mbar_arrive(bRecEmpty + 8 * rs);
         if (t == 0) NM_TRACE(5);
         // metadata word of this thread's TMEM lane: asynchronous store, waited for below
         const uint32_t Wa = __shfl_sync(0xffffffffu, W, mr0), Wb = __shfl_sync(0xffffffffu, W, mr0 + 8);
@@ -422,75 +553,91 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
         sts128(at + 128, v[4], v[5], v[6], v[7]);    // physical k 8..15 (LBO = 128)
         if (t == 0) NM_TRACE(6);
         asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-        if (t == 0) NM_TRACE(7);
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-        mbar_arrive(smem_u32(&full_b[s]));
+        __syncwarp();  // the warp's A-tile rows and metadata lanes are written
+        if (lane == 0) mbar_arrive(bFull + 8 * s);
         if (t == 0) NM_TRACE(2);
+        s += kLoadGroups;
+        if (s >= C::kStages) { s -= C::kStages; ph ^= 1; }
+        rs += kLoadGroups;
+        if (rs >= kRecSlots) { rs -= kRecSlots; rph ^= 1; }
       }
     }
   } else if (warp == kWarpMma) {
-    // ------------------------------------------------------------ MMA issuer (one thread)
-    // The cp.async gathers are published through cp.async.mbarrier.arrive on full_b.
-    if (lane == 0) {
-      int64_t i = 0;  // chunk counter (trace only)
-      int s = 0;
-      uint32_t ph = 0;
-      int acc = 0;
-      uint32_t aphase = 0;
-      const uint64_t adesc0 = sdesc(sA, 128, 256, 0);
-      const uint64_t bdesc0 = sdesc(sB, 4096, 1024, 2);
-      int4 nxt = unit_entry(p, blockIdx.x);
-      for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
-        const int4 cur = nxt;
-        nxt = unit_entry(p, u + ustep);
-        const int nch = cur.y;
-        mbar_wait(smem_u32(&tempty[acc]), aphase ^ 1);
-        NM_TRACE_U(1);
+    // ------------------------------------------------------------ MMA issuer
+    // The loop is warp-uniform (all lanes wait and advance the stage state, so descriptors
+    // and TMEM addresses stay in uniform registers) and one elected lane issues the MMA and
+    // its commit: the per-chunk issue path is ~20 instructions (a single divergent lane
+    // needed ~56 with register moves into the uniform datapath -- the kernel's skeleton was
+    // bound by it).  The cp.async gathers are published through
+    // cp.async.mbarrier.arrive on full_b.
+    int64_t i = 0;  // chunk counter (trace only)
+    int s = 0;
+    uint32_t ph = 0;
+    int acc = 0;
+    uint32_t aphase = 0;
+    const uint64_t adesc0 = sdesc(sA, 128, 256, 0);
+    const uint64_t bdesc0 = sdesc(sB, 4096, 1024, 2);
+    uint64_t ad = adesc0, bd = bdesc0;          // descriptors of stage s
+    uint32_t mcol = C::kMeta0;                  // metadata column of stage s
+    int4 nxt = unit_entry(p, blockIdx.x);
+    for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
+      const int4 cur = nxt;
+      nxt = unit_entry(p, u + ustep);
+      const int nch = cur.y;
+      mbar_wait(bTempty + 8 * acc, aphase ^ 1);
+      NM_TRACE_U(1);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      const uint32_t dcol = tbase + acc * BN;
+      for (int c = 0; c < nch; ++c, ++i) {
+        mbar_wait(bFull + 8 * s, ph);
+        NM_TRACE(3);
+        // the A tile (st.shared) and the gathers (cp.async) were written through the generic
+        // proxy: make them visible to the tensor core's async-proxy operand reads (without
+        // this fence stale stage contents were observed on B200 -- test_parity_fullsize.py)
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        const uint32_t dcol = tbase + acc * BN;
-        for (int c = 0; c < nch; ++c, ++i) {
-          mbar_wait(smem_u32(&full_b[s]), ph);
-          NM_TRACE(3);
-          // the A tile (st.shared) and the gathers (cp.async) were written through the generic
-          // proxy: make them visible to the tensor core's async-proxy operand reads (without
-          // this fence stale stage contents were observed on B200 -- test_parity_fullsize.py)
-          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          const uint64_t ad = adesc0 + (uint64_t)((s * C::kABytes) >> 4);
-          const uint64_t bd = bdesc0 + (uint64_t)((s * C::kBBytes) >> 4);
-          const uint32_t mcol = C::kMeta0 + s;
-          const uint32_t ecol = tbase + (mcol & ~1u);   // even column address ...
-          const uint32_t idesc = p.idesc | (mcol & 1u);  // ... + sparse_id2 selects the odd one
-          const uint32_t accum = c > 0 ? 1u : 0u;
-          asm volatile(
-              "{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %5, 0;\n\t"
-              "tcgen05.mma.sp.cta_group::1.kind::f16 [%0], %1, %2, [%3], %4, q;\n\t}" ::"r"(dcol),
-              "l"(ad), "l"(bd), "r"(ecol), "r"(idesc), "r"(accum)
-              : "memory");
-          asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-                           smem_u32(&empty[s]))
-                       : "memory");
-          if (++s == C::kStages) { s = 0; ph ^= 1; }
+        // metadata column: even column address + sparse_id2 selects the odd one
+        asm volatile(
+            "{\n\t.reg .pred e, q;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "setp.ne.b32 q, %5, 0;\n\t"
+            "@e tcgen05.mma.sp.cta_group::1.kind::f16 [%0], %1, %2, [%3], %4, q;\n\t"
+            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%6];\n\t}" ::"r"(dcol),
+            "l"(ad), "l"(bd), "r"(tbase + (mcol & ~1u)), "r"(p.idesc | (mcol & 1u)), "r"(c), "r"(bEmpty + 8 * s)
+            : "memory");
+        if (++s == C::kStages) {
+          s = 0;
+          ph ^= 1;
+          ad = adesc0;
+          bd = bdesc0;
+          mcol = C::kMeta0;
+        } else {
+          ad += (uint64_t)(C::kABytes >> 4);
+          bd += (uint64_t)(C::kBBytes >> 4);
+          ++mcol;
         }
-        if (nch > 0)
-          asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-                           smem_u32(&tfull[acc]))
-                       : "memory");
-        else
-          mbar_arrive(smem_u32(&tfull[acc]));
-        if (++acc == C::kNAcc) { acc = 0; aphase ^= 1; }
       }
+      if (nch > 0)
+        asm volatile(
+            "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(bTfull +
+                                                                                                          8 * acc)
+            : "memory");
+      else if (lane == 0)
+        mbar_arrive(bTfull + 8 * acc);
+      __syncwarp();
+      if (++acc == C::kNAcc) { acc = 0; aphase ^= 1; }
     }
-    __syncwarp();
   } else {
     // ------------------------------------------------------------ epilogue
-    // tcgen05.ld 16x256b: thread t holds rows (t/4) and (t/4 + 8) of its 16-lane block,
-    // columns 2*(t%4) + {0,1} of every 8-column repetition -> 8-byte stores, four threads
-    // complete a 32-byte sector of a Y row.
+    // tcgen05.ld 16x256b: thread t holds rows (t/4) and (t/4 + 8) of a 16-lane block, columns
+    // 2*(t%4) + {0,1} of every 8-column repetition -> 8-byte stores, four threads complete a
+    // 32-byte sector of a Y row.  kEpiWarps = 8: two warps per TMEM lane quarter, one 16-lane
+    // block each; kEpiWarps = 4: one warp per quarter does both blocks.
+    constexpr int kBlocks = 8 / kEpiWarps;               // 16-lane blocks per warp
     const int quarter = warp & 3;                        // TMEM lane quarter this warp may access
-    const int half = (warp - kWarpEpi0) >> 2;            // which 16 lanes of the quarter
-    const int lane0 = quarter * 32 + half * 16;          // first TMEM lane of this warp's block
-    const int rlo = lane0 + (lane >> 2), rhi = rlo + 8;  // rows (within the panel) of this thread
+    const int blk0 = ((warp - kWarpEpi0) >> 2) * kBlocks;
     const int cpair = 2 * (lane & 3);
     int acc = 0;
     uint32_t aphase = 0;
@@ -499,65 +646,95 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
       const int64_t g = (int64_t)e.x * kPanelRows + r;
       return g < p.rows ? (p.row_map ? (int64_t)__ldg(p.row_map + g) : g) : -1;
     };
+    auto row_of = [&](int b, int hi) { return quarter * 32 + (blk0 + b) * 16 + (lane >> 2) + 8 * hi; };
     int4 nxt = unit_entry(p, blockIdx.x);
-    int64_t nlo = blockIdx.x < p.n_units ? out_row(nxt, rlo) : -1;
-    int64_t nhi = blockIdx.x < p.n_units ? out_row(nxt, rhi) : -1;
+    int64_t nrow[kBlocks][2];  // output rows of the next unit (prefetched one unit ahead)
+#pragma unroll
+    for (int b = 0; b < kBlocks; ++b)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) nrow[b][h] = blockIdx.x < p.n_units ? out_row(nxt, row_of(b, h)) : -1;
     for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
       const int4 cur = nxt;
-      const int64_t olo = nlo, ohi = nhi;
+      int64_t orow[kBlocks][2];
+#pragma unroll
+      for (int b = 0; b < kBlocks; ++b)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) orow[b][h] = nrow[b][h];
       nxt = unit_entry(p, u + ustep);
       if (u + ustep < p.n_units) {
-        nlo = out_row(nxt, rlo);
-        nhi = out_row(nxt, rhi);
+#pragma unroll
+        for (int b = 0; b < kBlocks; ++b)
+#pragma unroll
+          for (int h = 0; h < 2; ++h) nrow[b][h] = out_row(nxt, row_of(b, h));
       }
       const int ft = (int)(u % p.n_ftiles);
       const bool has = cur.y > 0;
-      mbar_wait(smem_u32(&tfull[acc]), aphase);
+      const bool full_tile = vec_ok && ft * BN + BN <= p.F;
+      mbar_wait_sleep(bTfull + 8 * acc, aphase);
       NM_TRACE_U(2);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+#pragma unroll
+      for (int b = 0; b < kBlocks; ++b) {
+        const int64_t olo = orow[b][0], ohi = orow[b][1];
+        const uint32_t lane0 = (uint32_t)(quarter * 32 + (blk0 + b) * 16);
 #pragma unroll 1
-      for (int cc = 0; cc < BN; cc += 64) {
-        uint32_t v[32];
-        if (has) {
-          const uint32_t taddr = tbase + ((uint32_t)lane0 << 16) + acc * BN + cc;
-          asm volatile(
-              "tcgen05.ld.sync.aligned.16x256b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-              "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-              : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-                "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
-                "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
-                "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
-                "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
-              : "r"(taddr));
-          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-        } else {
-#pragma unroll
-          for (int j = 0; j < 32; ++j) v[j] = 0u;
-        }
-        if (p.debug & 2) continue;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          const int col = ft * BN + cc + 8 * j + cpair;
-          if (col >= p.F) continue;
-          const float2 lo = make_float2(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]));
-          const float2 hi = make_float2(__uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3]));
-          if (vec_ok && col + 2 <= p.F) {
-            if (olo >= 0) __stcs((float2*)(p.Y + olo * p.ldy + col), lo);
-            if (ohi >= 0) __stcs((float2*)(p.Y + ohi * p.ldy + col), hi);
+        for (int cc = 0; cc < BN; cc += 64) {
+          uint32_t v[32];
+          if (has) {
+            const uint32_t taddr = tbase + (lane0 << 16) + acc * BN + cc;
+            asm volatile(
+                "tcgen05.ld.sync.aligned.16x256b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+                "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+                : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+                  "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+                  "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
+                  "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
+                  "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+                : "r"(taddr));
+            asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
           } else {
-            if (olo >= 0) {
-              p.Y[olo * p.ldy + col] = lo.x;
-              if (col + 1 < p.F) p.Y[olo * p.ldy + col + 1] = lo.y;
+#pragma unroll
+            for (int j = 0; j < 32; ++j) v[j] = 0u;
+          }
+          if (p.debug & 2) continue;
+          if (full_tile) {  // unit-uniform fast path: every column in range, 8-byte stores
+            float* ylo = p.Y + olo * p.ldy + ft * BN + cc + cpair;
+            float* yhi = p.Y + ohi * p.ldy + ft * BN + cc + cpair;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              if (olo >= 0)
+                __stcs((float2*)(ylo + 8 * j), make_float2(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1])));
+              if (ohi >= 0)
+                __stcs((float2*)(yhi + 8 * j),
+                       make_float2(__uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3])));
             }
-            if (ohi >= 0) {
-              p.Y[ohi * p.ldy + col] = hi.x;
-              if (col + 1 < p.F) p.Y[ohi * p.ldy + col + 1] = hi.y;
+            continue;
+          }
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const int col = ft * BN + cc + 8 * j + cpair;
+            if (col >= p.F) continue;
+            const float2 lo = make_float2(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]));
+            const float2 hi = make_float2(__uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3]));
+            if (vec_ok && col + 2 <= p.F) {
+              if (olo >= 0) __stcs((float2*)(p.Y + olo * p.ldy + col), lo);
+              if (ohi >= 0) __stcs((float2*)(p.Y + ohi * p.ldy + col), hi);
+            } else {
+              if (olo >= 0) {
+                p.Y[olo * p.ldy + col] = lo.x;
+                if (col + 1 < p.F) p.Y[olo * p.ldy + col + 1] = lo.y;
+              }
+              if (ohi >= 0) {
+                p.Y[ohi * p.ldy + col] = hi.x;
+                if (col + 1 < p.F) p.Y[ohi * p.ldy + col + 1] = hi.y;
+              }
             }
           }
         }
       }
       asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-      mbar_arrive(smem_u32(&tempty[acc]));
+      __syncwarp();
+      if (lane == 0) mbar_arrive(bTempty + 8 * acc);
       NM_TRACE_U(3);
       if (++acc == C::kNAcc) { acc = 0; aphase ^= 1; }
     }

@@ -1,0 +1,6 @@
+# one ncu --set full capture of k_spmm_sptc on a workload: prof1.sh <workload> <tag>
+WL=${1:-c2-banded-n1m-d16-f128-1:2:4}; TAG=${2:-cur}
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout 1200 ncu --set full --clock-control none --import-source on -k regex:k_spmm_sptc -s 3 -c 1 -o gpurun_out/prof_$TAG -f \
+  python bench.py --steps 2 --warmup 3 --no-cpu --no-cusparse --workload $WL > gpurun_out/prof_bench_$TAG.log 2>&1
+echo done

@@ -24,7 +24,8 @@ def main():
     w = bench.parse_workload(wl)
     ip, ic, vals, X32 = bench.make_graph(w)
     perm, _ = api.reorder(ip, ic, w["V"], 2, w["M"])
-    P = api.pack(ip, ic, perm, w["V"], 2, w["M"], dtype=w["dtype"], val=vals, order="original")
+    tau = w["tau"] if w["tau"] is not None else api.hybrid_tau(w["F"])
+    P = api.pack(ip, ic, perm, w["V"], 2, w["M"], dtype=w["dtype"], val=vals, order="original", tau=tau)
     xb, _ = graphs.round16(X32, w["dtype"])
     X = torch.from_numpy(xb.view(np.int16)).cuda().view(torch.float16)
     Y = torch.empty((w["n"], w["F"]), device="cuda")
@@ -37,6 +38,8 @@ def main():
     torch.cuda.synchronize()
     del os.environ["NM_SPMM_TRACE"]
     t = np.fromfile(path, dtype=np.uint64).astype(np.int64)
+    if os.environ.get("NM_TRACE_SAVE"):
+        np.save(os.environ["NM_TRACE_SAVE"], t)
     full = t[:8192].reshape(1024, 8)
     ch = full[:, :4]
     un = t[8192:].reshape(2048, 4)
@@ -47,13 +50,34 @@ def main():
     ch[:, 0] = np.maximum.accumulate(ch[:, 0])  # issue time of the sub-batch holding the chunk
     # loader sub-steps (slots 1 -> 4 -> 5 -> 6 -> 7 -> 2): sees record, gathers issued, record
     # expanded + released, A tile + tcgen05.st issued, tcgen05.wait::st done, arrived
-    sub = full[:n][:, [1, 4, 5, 6, 7, 2]]
+    sub = full[:n][:, [7, 1, 4, 5, 6, 2]]
     own = sub[:, 0] > 0
     if own.any():
         d = np.diff(sub[own], axis=1)
-        for name, v in zip(["gathers issue", "expand+release", "A sts + tcgen05.st", "tcgen05.wait::st",
-                            "fence+arrive"], d.T):
+        for name, v in zip(["stage free -> record seen", "gathers issue", "expand+release",
+                            "A sts + tcgen05.st", "wait::st+fence+arrive"], d.T):
             print("loader %-22s median %6d  p90 %6d cycles" % (name, np.median(v), np.percentile(v, 90)))
+    G = int(os.environ.get("NM_TRACE_GROUPS", "3"))
+    f = full[:n].astype(np.int64)
+    if n > 2 * G:
+        ws = f[G:, 7] - f[:-G, 2]   # own previous chunk arrived -> this chunk's stage free
+        wr = f[G:, 1] - f[G:, 7]    # stage free -> record landed
+        busy = f[G:, 2] - f[G:, 1]  # record landed -> arrive (loader work)
+        for name, v in [("loader wait for stage", ws), ("loader wait for record", wr), ("loader busy", busy)]:
+            print("%-30s mean %6.0f median %6d p90 %6d cycles" % (name, v.mean(), np.median(v), np.percentile(v, 90)))
+    sbt = t[12288:].reshape(1024, 4)
+    nsb = int((sbt[:, 0] > 0).sum())
+    if nsb > 1:
+        sbt = sbt[:nsb]
+        wait_space = sbt[:, 1] - sbt[:, 0]
+        other = sbt[1:, 0] - sbt[:-1, 1]
+        infl, ringb = sbt[:, 2] >> 32, sbt[:, 2] & 0xFFFFFFFF
+        nw, m = sbt[:, 3] >> 32, sbt[:, 3] & 0xFFFFFFFF
+        print("producer: %d sub-batches (mean %.1f records), ring-space wait mean %.0f (p90 %.0f), other work "
+              "between waits mean %.0f (p90 %.0f) cycles; at entry: descriptors in flight mean %.1f, ring bytes "
+              "mean %.0f; descriptor waits per sub-batch mean %.2f" %
+              (nsb, m.mean(), wait_space.mean(), np.percentile(wait_space, 90), other.mean(),
+               np.percentile(other, 90), infl.mean(), ringb.mean(), nw.mean()))
     ch = ch - base
     print("chunks traced:", n)
     d_rec_ld = ch[:, 1] - ch[:, 0]
