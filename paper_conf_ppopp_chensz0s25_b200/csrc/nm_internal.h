@@ -64,7 +64,10 @@ struct ResSeg {
   int32_t slot;      // first workspace slot of the row's partials, -1 = single-segment row
   int32_t split_id;  // arrival counter of the row (split rows only)
   int32_t nseg, idx; // segments of the row, index of this one
+  int32_t yrow;      // output row of Y (row_map applied in NM_PACK_ORIGINAL_ORDER)
+  int32_t pad;
 };
+static_assert(sizeof(ResSeg) == 40, "ResSeg layout");
 
 }  // namespace nm
 

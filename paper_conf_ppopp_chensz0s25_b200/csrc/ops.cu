@@ -22,21 +22,22 @@ __device__ __forceinline__ float fma16(unsigned short a, unsigned short b, float
 }
 
 // Yp[l][f] += sum_k res_val[k] * PX[res_col[k]][f]  (the residual CSR, lossless remainder).
-// One warp per work item (<= kResSeg nonzeros of one row, ResSeg), features [f0, f0 + LPR*8)
-// of this launch's slab.  The warp's lanes form SUB = 32 / LPR subgroups of LPR lanes; a
-// subgroup covers LPR * 8 features with one 16-byte X load per lane and the subgroups take
-// alternate nonzeros (so F = 128 keeps all 32 lanes busy with 16-byte loads).  The item's
-// (col, val) pairs are fetched 32 at a time with one coalesced load and broadcast with
-// shuffles; the loop is unrolled so several X rows are in flight per lane.  Subgroup partial
-// sums are combined with xor-shuffles.  A row with one item adds its sum into Y; the items of
-// a split row (hub rows) write partials to their workspace slots and the last one to arrive
-// (per-row counter) adds the partials in item order -- deterministic, no float atomics.
-// F tail: the 16-byte vector at column f < F is inside the row (ldx % 8 == 0), only the
-// accumulate/store is masked.
+// Work items (ResSeg) hold <= kResSeg nonzeros of one row.  A warp is SUB = 32 / LPR
+// subgroups of LPR lanes and every subgroup runs its own items (items w*SUB + sub, ...), so a
+// warp has SUB independent items -- each a chain of dependent memory round trips -- in
+// flight; a lane owns 8 consecutive features of the launch's slab [f_base, f_base + LPR*8)
+// and reads them with one 16-byte load per nonzero.  The item's (col, val) pairs are fetched
+// LPR at a time with one coalesced load and broadcast within the subgroup by shuffles; the
+// loop is unrolled so kUnroll X rows are in flight per lane.  The next item's descriptor is
+// prefetched, and the Y row (addressed by the item's output row, row_map applied at pack
+// time) is read next to the first (col, val) batch.  A row with one item adds its sum into Y;
+// the items of a split row (hub rows) write partials to their workspace slots and the last
+// one to arrive (per-row counter) adds the partials in item order -- deterministic, no float
+// atomics.  F tail: the 16-byte vector at column f < F is inside the row (ldx % 8 == 0), only
+// the accumulate/store is masked.
 template <int BF, int LPR>
 __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ segs, int64_t n_segs,
                                                   const int32_t* __restrict__ rc, const uint16_t* __restrict__ rv,
-                                                  const int32_t* __restrict__ row_map,
                                                   const uint16_t* __restrict__ X, int64_t ldx,
                                                   float* __restrict__ Y, int64_t ldy, int F, int f_base,
                                                   float* __restrict__ ws, int32_t* __restrict__ cnt) {
@@ -44,30 +45,43 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
   constexpr int kUnroll = 4;
   const int lane = threadIdx.x & 31;
   const int sub = lane / LPR, li = lane % LPR;
+  const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (sub * LPR));
   const int f = f_base + li * 8;  // first feature of this lane
-  const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
-  const bool vec_y = ((ldy & 3) == 0) && ((((uintptr_t)Y) & 15) == 0);
-  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < n_segs; w += nw) {
-    const ResSeg g = segs[w];
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5) * SUB;  // subgroups in the grid
+  const bool vec_y = ((ldy & 3) == 0) && ((((uintptr_t)Y) & 15) == 0) && f + 8 <= F;
+  int64_t w = ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5) * SUB + sub;
+  ResSeg gn;
+  if (w < n_segs) gn = segs[w];
+  for (; w < n_segs; w += nw) {
+    const ResSeg g = gn;
+    if (w + nw < n_segs) gn = segs[w + nw];  // next item's descriptor, ahead of use
+    float* y = Y + (int64_t)g.yrow * ldy + f;
+    // single-item rows: the Y row comes in with the first (col, val) batch
+    float4 y0 = make_float4(0.f, 0.f, 0.f, 0.f), y1 = y0;
+    const bool early_y = g.slot < 0 && vec_y;
+    if (early_y) {
+      y0 = __ldcs((const float4*)y);
+      y1 = __ldcs((const float4*)(y + 4));
+    }
     float acc[8];
 #pragma unroll
     for (int q = 0; q < 8; ++q) acc[q] = 0.f;
-    for (int base = 0; base < g.len; base += 32) {
-      const int cnt_ = min(32, g.len - base);
+    for (int base = 0; base < g.len; base += LPR) {
+      const int cnt_ = min(LPR, g.len - base);
       int32_t c = 0;
       uint32_t v = 0u;  // 16-bit value bits (a zero value adds exact zeros)
-      if (lane < cnt_) {
-        c = __ldg(rc + g.kb + base + lane);
-        v = __ldg(rv + g.kb + base + lane);
+      if (li < cnt_) {
+        c = __ldg(rc + g.kb + base + li);
+        v = __ldg(rv + g.kb + base + li);
       }
-      for (int j = 0; j < cnt_; j += SUB * kUnroll) {
+      for (int j = 0; j < cnt_; j += kUnroll) {
         uint4 xv[kUnroll];
         uint32_t vv[kUnroll];
 #pragma unroll
         for (int u = 0; u < kUnroll; ++u) {
-          const int idx = j + u * SUB + sub;
-          const int32_t cc = __shfl_sync(0xffffffffu, c, idx & 31);
-          vv[u] = __shfl_sync(0xffffffffu, v, idx & 31);
+          const int idx = j + u;
+          const int32_t cc = __shfl_sync(gmask, c, idx & (LPR - 1), LPR);
+          vv[u] = __shfl_sync(gmask, v, idx & (LPR - 1), LPR);
           if (idx < cnt_ && f < F) {
             xv[u] = __ldg((const uint4*)(X + (int64_t)cc * ldx + f));
           } else {
@@ -87,34 +101,33 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
         }
       }
     }
-#pragma unroll
-    for (int o = LPR; o < 32; o <<= 1)
-#pragma unroll
-      for (int q = 0; q < 8; ++q) acc[q] += __shfl_xor_sync(0xffffffffu, acc[q], o);
-    float* y = Y + (row_map ? (int64_t)row_map[g.row] : (int64_t)g.row) * ldy + f;
+    if (early_y) {
+      y0.x += acc[0]; y0.y += acc[1]; y0.z += acc[2]; y0.w += acc[3];
+      y1.x += acc[4]; y1.y += acc[5]; y1.z += acc[6]; y1.w += acc[7];
+      __stcs((float4*)y, y0);
+      __stcs((float4*)(y + 4), y1);
+      continue;
+    }
     if (g.slot >= 0) {
       // split row: publish this item's partial, the last arrival reduces in item order
       float* part = ws + ((int64_t)(g.slot + g.idx) * kResSlab) + li * 8;
-      if (sub == 0) {
-        *(float4*)part = make_float4(acc[0], acc[1], acc[2], acc[3]);
-        *(float4*)(part + 4) = make_float4(acc[4], acc[5], acc[6], acc[7]);
-      }
+      *(float4*)part = make_float4(acc[0], acc[1], acc[2], acc[3]);
+      *(float4*)(part + 4) = make_float4(acc[4], acc[5], acc[6], acc[7]);
       __threadfence();
-      __syncwarp();
+      __syncwarp(gmask);
       int last = 0;
-      if (lane == 0) last = atomicAdd(cnt + g.split_id, 1) == g.nseg - 1;
-      last = __shfl_sync(0xffffffffu, last, 0);
+      if (li == 0) last = atomicAdd(cnt + g.split_id, 1) == g.nseg - 1;
+      last = __shfl_sync(gmask, last, 0, LPR);
       if (!last) continue;
       __threadfence();
 #pragma unroll
       for (int q = 0; q < 8; ++q) acc[q] = 0.f;
-      // subgroup j sums the partials i = j (mod SUB), kUnroll loads in flight per lane; the
-      // assignment is fixed, so the summation order is too
-      for (int i0 = 0; i0 < g.nseg; i0 += SUB * kUnroll) {
+      // the partials in item order, kUnroll loads in flight per lane
+      for (int i0 = 0; i0 < g.nseg; i0 += kUnroll) {
         float4 pa[kUnroll], pb[kUnroll];
 #pragma unroll
         for (int u = 0; u < kUnroll; ++u) {
-          const int i = i0 + u * SUB + sub;
+          const int i = i0 + u;
           pa[u] = pb[u] = make_float4(0.f, 0.f, 0.f, 0.f);
           if (i < g.nseg) {
             const float* pi = ws + ((int64_t)(g.slot + i) * kResSlab) + li * 8;
@@ -128,19 +141,15 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
           acc[4] += pb[u].x; acc[5] += pb[u].y; acc[6] += pb[u].z; acc[7] += pb[u].w;
         }
       }
-#pragma unroll
-      for (int o = LPR; o < 32; o <<= 1)
-#pragma unroll
-        for (int q = 0; q < 8; ++q) acc[q] += __shfl_xor_sync(0xffffffffu, acc[q], o);
-      if (lane == 0) cnt[g.split_id] = 0;  // ready for the next launch
+      if (li == 0) cnt[g.split_id] = 0;  // ready for the next launch
     }
-    if (sub == 0 && f < F) {
-      if (vec_y && f + 8 <= F) {
-        float4 y0 = *(float4*)y, y1 = *(float4*)(y + 4);
-        y0.x += acc[0]; y0.y += acc[1]; y0.z += acc[2]; y0.w += acc[3];
-        y1.x += acc[4]; y1.y += acc[5]; y1.z += acc[6]; y1.w += acc[7];
-        *(float4*)y = y0;
-        *(float4*)(y + 4) = y1;
+    if (f < F) {
+      if (vec_y) {
+        float4 a0 = *(float4*)y, a1 = *(float4*)(y + 4);
+        a0.x += acc[0]; a0.y += acc[1]; a0.z += acc[2]; a0.w += acc[3];
+        a1.x += acc[4]; a1.y += acc[5]; a1.z += acc[6]; a1.w += acc[7];
+        *(float4*)y = a0;
+        *(float4*)(y + 4) = a1;
       } else {
 #pragma unroll
         for (int q = 0; q < 8; ++q)
@@ -217,10 +226,11 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
   // lanes per item: 8 features per lane; one launch per slab of LPR * 8 features
   const int lpr = F <= 32 ? 4 : F <= 64 ? 8 : F <= 128 ? 16 : 32;
   const int bf = P->dtype == NM_BF16;
-  int64_t g = (P->n_res_segs + 7) / 8;
+  const int sub_per_warp = 32 / lpr;
+  int64_t g = (P->n_res_segs + 8 * sub_per_warp - 1) / (8 * sub_per_warp);
   if (g > 148 * 16) g = 148 * 16;
 #define NM_RES_LAUNCH(BF, LPR)                                                                            \
-  k_residual<BF, LPR><<<(unsigned)g, 256, 0, s>>>(P->res_segs, P->n_res_segs, rcol, P->res_val, P->row_map, \
+  k_residual<BF, LPR><<<(unsigned)g, 256, 0, s>>>(P->res_segs, P->n_res_segs, rcol, P->res_val, \
                                                   (const uint16_t*)PX, ldx, Yp, ldy, F, f_base, P->res_ws,      \
                                                   P->res_cnt)
   for (int f_base = 0; f_base < F; f_base += lpr * 8) {

@@ -462,11 +462,13 @@ __global__ void k_seg_fill(const int64_t* __restrict__ rrp, int64_t rows, const 
       ResSeg g;
       g.kb = b + i * kResSeg;
       g.row = (int32_t)l;
+      g.yrow = (int32_t)l;  // NM_PACK_ORIGINAL_ORDER: replaced by row_map[l] (k_seg_yrow)
       g.len = (int32_t)min((int64_t)kResSeg, len - i * kResSeg);
       g.slot = k > 1 ? (int32_t)slot_ptr[l] : -1;
       g.split_id = k > 1 ? (int32_t)split_ptr[l] : -1;
       g.nseg = (int32_t)k;
       g.idx = (int32_t)i;
+      g.pad = 0;
       segs[seg_ptr[l] + i] = g;
     }
   }
@@ -527,6 +529,11 @@ nm_status scan_excl(const int64_t* in, int64_t* out, int64_t n, cudaStream_t s) 
 }
 
 // identity == 1: a[i] = perm[i] (perm already offset); else a[i] = a[i] >= 0 ? perm[a[i]] : -1
+__global__ void k_seg_yrow(const int32_t* __restrict__ row_map, ResSeg* __restrict__ segs, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    segs[i].yrow = row_map[segs[i].row];
+}
+
 __global__ void k_map(const int32_t* __restrict__ perm, int32_t* __restrict__ a, int64_t m, int identity) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
     if (identity) a[i] = perm[i];
@@ -820,6 +827,8 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     NM_TRY(palloc((void**)&Pk->res_gather, sizeof(int32_t) * res_nnz));
     const int32_t* pm = d_perm.as<int32_t>();
     k_map<<<grid_for(rows, 256), 256, 0, s>>>(pm + rb, Pk->row_map, rows, 1);
+    if (Pk->n_res_segs)  // residual work items address Y by output row
+      k_seg_yrow<<<grid_for(Pk->n_res_segs, 256), 256, 0, s>>>(Pk->row_map, Pk->res_segs, Pk->n_res_segs);
     if (n_chunks) k_xrow_map<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(pm, full, n_chunks);
     if (res_nnz) {
       NM_CUDA(cudaMemcpyAsync(Pk->res_gather, Pk->res_col, sizeof(int32_t) * res_nnz, cudaMemcpyDeviceToDevice, s));
