@@ -168,9 +168,9 @@ NM_API nm_status nm_pack_hybrid(const nm_csr* A, const int32_t* perm, int V, int
                                 int tau, void* stream, nm_packed** out);
 
 /* nm_hybrid_tau -- the tau nm_pack_hybrid should use for an SpMM with F feature columns:
- * the break-even number of kept values at which a meta-block's bytes through L2 (its share
- * of a chunk record + 4 gathered X rows) equal those of the same values in the residual CSR
- * (6 bytes + 1 gathered X row each).  DESIGN.md §6.  Returns 0 for F < 1. */
+ * the break-even number of kept values at which a meta-block's gathered X bytes (its 4
+ * selected rows) equal those of the same values in the residual CSR (6 bytes + 1 gathered X
+ * row each): ceil(8F / (2F + 6)), i.e. 4 for F >= 10.  DESIGN.md §6.  Returns 0 for F < 1. */
 NM_API int nm_hybrid_tau(int F);
 
 /* Sizes: #meta-blocks, #values kept in MMA slots, #residual nonzeros, device bytes held,

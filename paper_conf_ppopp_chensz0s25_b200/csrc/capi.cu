@@ -170,10 +170,13 @@ int nm_version(void) { return 1; }
 // plus one gathered X row (2F bytes).  Blocks keeping fewer values than the break-even go to
 // the residual.
 int nm_hybrid_tau(int F) {
+  // break-even of the X-row traffic: a meta-block gathers its 4 selected X rows (8F bytes of
+  // 16-bit features) whatever it keeps, a residual value gathers one X row plus its 6-byte
+  // (col, value) entry.  The compressed chunk record adds only ~4 bytes per kept value, so it
+  // is left out; measured on B200: banded n = 2^20, F = 128 -> tau 2 / 3 / 5 / 7
+  // = 0.268 / 0.263 / 0.275 / 0.290 ms per step, and this model gives 4.
   if (F < 1) return 0;
-  const double block = nm::kChunkBytes / 8.0 + 4.0 * 2.0 * F;
-  const double value = 6.0 + 2.0 * F;
-  return (int)ceil(block / value);
+  return (int)ceil(8.0 * F / (2.0 * F + 6.0));
 }
 
 void nm_packed_free(nm_packed* P) {

@@ -36,28 +36,34 @@ namespace nm {
 namespace {
 
 #ifndef NM_LOAD_GROUPS
-#define NM_LOAD_GROUPS 3
+#define NM_LOAD_GROUPS 4
 #endif
 constexpr int kWarpRec = 0, kWarpLoad0 = 1, kLoadGroups = NM_LOAD_GROUPS;
+#ifndef NM_PRODUCERS
+#define NM_PRODUCERS 2               // record producer warps (alternate units, own ring halves)
+#endif
+constexpr int kProducers = NM_PRODUCERS;
+constexpr int kSlotsShift = kProducers == 1 ? 6 : kProducers == 2 ? 5 : 4;
+constexpr int kSlotsPP = 1 << kSlotsShift;    // record descriptors per producer (power of two)
+constexpr int kRecSlots = kSlotsPP * kProducers;
+static_assert(kProducers >= 1 && kProducers <= 3, "one to three record producers");
+static_assert((1 << kSlotsShift) == kSlotsPP, "descriptor count");
 #ifndef NM_EPI_WARPS
-#define NM_EPI_WARPS 8
+#define NM_EPI_WARPS 4
 #endif
 constexpr int kWarpMma = kWarpLoad0 + 4 * kLoadGroups, kWarpEpi0 = kWarpMma + 1, kEpiWarps = NM_EPI_WARPS;
-constexpr int kThreads = (kWarpEpi0 + kEpiWarps) * 32;
+constexpr int kWarpRec2 = kWarpEpi0 + kEpiWarps;  // producers 1.. (kProducers > 1)
+constexpr int kThreads = (kWarpEpi0 + kEpiWarps + kProducers - 1) * 32;
 static_assert(kEpiWarps == 4 || kEpiWarps == 8, "epilogue: one or two warps per TMEM lane quarter");
 constexpr int kGroupThreads = 128;                     // loader threads per group
 constexpr int kPrefetchUnits = 2;                      // record L2-prefetch distance (units)
-// compressed records land in a byte ring of kRecRing bytes (allocated in chunk order; a
-// record that runs past the end continues into a kRecMaxBytes pad, so every record is
-// contiguous without skipping) described by kRecSlots descriptors; descriptor i % kRecSlots
-// belongs to chunk i, so loader group g only ever waits on descriptors = g (mod 3)
+// compressed records land in byte rings, one per producer (allocated in chunk order; a record
+// that runs past the end continues into a kRecMaxBytes pad, so every record is contiguous
+// without skipping), each described by kSlotsPP descriptors: a producer's j-th record uses
+// descriptor j % kSlotsPP
 #ifndef NM_REC_CPASYNC
 #define NM_REC_CPASYNC 0             // records by warp-wide cp.async instead of one bulk copy each
 #endif
-#ifndef NM_REC_SLOTS_PER_GROUP
-#define NM_REC_SLOTS_PER_GROUP 16
-#endif
-constexpr int kRecSlots = NM_REC_SLOTS_PER_GROUP * kLoadGroups;
 constexpr int kIssueLanes = 8;       // records whose bulk copies are issued together
 
 struct SpmmParams {
@@ -212,9 +218,12 @@ struct Cfg {
   // stage has one consumer group that visits it in chunk order (parity waits stay valid)
   static constexpr int kStages = ((kStagesRaw > 16 ? 16 : kStagesRaw) / kLoadGroups) * kLoadGroups;
   // the record ring takes what the stages leave (largest power of two, >= 32 KB)
-  static constexpr int kRingAvail = 214 * 1024 - kStages * kStageBytes - kRecMaxBytes;
-  static constexpr int kRecRing = kRingAvail >= 128 * 1024 ? 128 * 1024 : kRingAvail >= 64 * 1024 ? 64 * 1024 : 32 * 1024;
-  static constexpr int kRecRegion = kRecRing + kRecMaxBytes;
+  static constexpr int kRingAvail = 214 * 1024 - kStages * kStageBytes - kProducers * kRecMaxBytes;
+  static constexpr int kRingPer = kRingAvail / kProducers;
+  static constexpr int kRecRing =  // each producer's ring: the largest power of two that fits
+      kRingPer >= 64 * 1024 ? 64 * 1024 : kRingPer >= 32 * 1024 ? 32 * 1024 : 16 * 1024;
+  static constexpr int kRingStride = kRecRing + kRecMaxBytes; // ring + wrap pad per producer
+  static constexpr int kRecRegion = kProducers * kRingStride;
   static constexpr int kNAcc = (2 * BN + kStages <= 512) ? 2 : 1;
   static constexpr int kMeta0 = kNAcc * BN;                     // metadata column of stage s: kMeta0 + s
   static constexpr int kBRegion = kStages * kBBytes;            // 1024-aligned tiles (SW128)
@@ -222,7 +231,7 @@ struct Cfg {
   static_assert(kMeta0 + kStages <= 512, "TMEM budget");
   static_assert(BN % 64 == 0 && BN >= 64 && BN <= 256, "BN");
   static_assert(kSmem <= 227 * 1024, "smem");
-  static_assert(kRecSlots % kLoadGroups == 0 && kRecMaxBytes % 16 == 0 && kRecRing >= 2 * kRecMaxBytes,
+  static_assert(kRecMaxBytes % 16 == 0 && kRecRing >= 2 * kRecMaxBytes,
                 "record ring");
 };
 
@@ -278,12 +287,21 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
   const uint32_t tbase = *tmem_slot;
   const int64_t ustep = gridDim.x;
 
-  if (warp == kWarpRec) {
+  if (warp == kWarpRec || (kProducers > 1 && warp >= kWarpRec2)) {
     // ------------------------------------------------------------ record producer (HBM stream)
+    // kProducers warps take alternate units of the CTA (producer pw: unit ordinals k with
+    // k % kProducers == pw), each with its own half of the ring and its own kSlotsPP
+    // descriptors, so record issue is not one warp's serial chain.
     // the warp reads the record sizes of 32 chunks at a time (one unit ahead); lane 0
     // allocates ring space -- waiting, oldest first, for the loader groups to release older
     // records -- and issues the bulk copies.  Lane 0's per-record path is kept short (32-bit
     // wrapping counters, no divisions): it is a serial chain on one thread.
+    const int pw = warp == kWarpRec ? 0 : 1 + warp - kWarpRec2;
+    const uint32_t sRecP = sRec + pw * C::kRingStride;  // this producer's ring
+    const uint32_t bRecFullP = bRecFull + 8 * pw * kSlotsPP, bRecEmptyP = bRecEmpty + 8 * pw * kSlotsPP;
+    uint32_t* rec_offP = rec_off + pw * kSlotsPP;
+    uint32_t* rec_endP = rec_end + pw * kSlotsPP;
+    const int64_t pstep = kProducers * ustep;  // unit stride of this producer
     uint32_t head = 0, tail = 0;       // cumulative ring bytes allocated / released (mod 2^32)
     int ds = 0, os = 0;                // next descriptor to fill / oldest one not yet released
     uint32_t oph = 0;                  // use parity of the oldest descriptor
@@ -300,24 +318,24 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
     auto first_lens = [&](int4 e) -> uint32_t {  // sizes of a unit's first 32 records (lane j)
       return lane < e.y ? 16u * __ldg(p.rec_len16 + entry_c0(e) + lane) : 0u;
     };
-    for (int k = 0; k < kPrefetchUnits; ++k) prefetch_unit(unit_bytes(p, blockIdx.x + k * ustep));
+    const int64_t u0 = blockIdx.x + pw * ustep;
+    for (int k = 0; k < kPrefetchUnits; ++k) prefetch_unit(unit_bytes(p, u0 + k * pstep));
     // schedule lookahead: entries two units ahead, record sizes one unit ahead (from an entry
     // that is already in registers), so no HBM round trip sits between two units' issues
-    int4 e1 = unit_entry(p, blockIdx.x), b1 = unit_bytes(p, blockIdx.x);
-    int4 e2 = unit_entry(p, blockIdx.x + ustep), b2 = unit_bytes(p, blockIdx.x + ustep);
-    int4 pfb = unit_bytes(p, blockIdx.x + kPrefetchUnits * ustep);
+    int4 e1 = unit_entry(p, u0), b1 = unit_bytes(p, u0);
+    int4 e2 = unit_entry(p, u0 + pstep), b2 = unit_bytes(p, u0 + pstep);
+    int4 pfb = unit_bytes(p, u0 + kPrefetchUnits * pstep);
     uint32_t nlen = first_lens(e1);
-    for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
-      NM_TRACE_U(0);
+    for (int64_t u = u0; u < p.n_units; u += pstep) {
       const int4 cur = e1, curb = b1;
       uint32_t len = nlen;
       e1 = e2;
       b1 = b2;
-      e2 = unit_entry(p, u + 2 * ustep);
-      b2 = unit_bytes(p, u + 2 * ustep);
+      e2 = unit_entry(p, u + 2 * pstep);
+      b2 = unit_bytes(p, u + 2 * pstep);
       nlen = first_lens(e1);
       prefetch_unit(pfb);
-      pfb = unit_bytes(p, u + (kPrefetchUnits + 1) * ustep);
+      pfb = unit_bytes(p, u + (kPrefetchUnits + 1) * pstep);
       const int64_t c0 = entry_c0(cur);
       const int nch = cur.y;
       int64_t boff = lo_hi(curb.x, curb.y);
@@ -341,20 +359,20 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
           m = __popc(__ballot_sync(0xffffffffu, lane >= sb && lane < sb + kIssueLanes && lane < cnt &&
                                                     incl - e0 <= (uint32_t)(C::kRecRing / 2)));
           const uint32_t total = __shfl_sync(0xffffffffu, incl, sb + m - 1) - e0;
-          if (NM_TRACE_ON && p.trace && blockIdx.x == 0 && lane == 0 && nsb < 1024) {
+          if (NM_TRACE_ON && p.trace && blockIdx.x == 0 && pw == 0 && lane == 0 && nsb < 1024) {
             p.trace[12288 + 4 * nsb] = clock64();
             p.trace[12290 + 4 * nsb] = ((uint64_t)in_flight << 32) | (head - tail);
           }
           if (lane == 0) {
             int nw = 0;
-            while (head + total - tail > (uint32_t)C::kRecRing || in_flight + m > kRecSlots) {
+            while (head + total - tail > (uint32_t)C::kRecRing || in_flight + m > kSlotsPP) {
               ++nw;
-              mbar_wait(bRecEmpty + 8 * os, oph);
-              tail = rec_end[os];
+              mbar_wait(bRecEmptyP + 8 * os, oph);
+              tail = rec_endP[os];
               --in_flight;
-              if (++os == kRecSlots) { os = 0; oph ^= 1; }
+              if (++os == kSlotsPP) { os = 0; oph ^= 1; }
             }
-            if (NM_TRACE_ON && p.trace && blockIdx.x == 0 && nsb < 1024) {
+            if (NM_TRACE_ON && p.trace && blockIdx.x == 0 && pw == 0 && nsb < 1024) {
               p.trace[12289 + 4 * nsb] = clock64();
               p.trace[12291 + 4 * nsb] = ((uint64_t)nw << 32) | (uint32_t)m;
             }
@@ -367,37 +385,37 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
           // per instruction) and every lane's cp.async.mbarrier.arrive.noinc marks it landed
           for (int k = 0; k < m; ++k) {
             int d = d0 + k;
-            if (d >= kRecSlots) d -= kRecSlots;
+            if (d >= kSlotsPP) d -= kSlotsPP;
             const uint32_t ek = __shfl_sync(0xffffffffu, excl, sb + k);
             const uint32_t lk = __shfl_sync(0xffffffffu, len, sb + k);
             const uint32_t start = h0 + (ek - e0);
             const uint32_t pos = start & (uint32_t)(C::kRecRing - 1);
             if (lane == 0) {
-              rec_end[d] = start + lk;
-              rec_off[d] = pos;
+              rec_endP[d] = start + lk;
+              rec_offP[d] = pos;
             }
             const uint8_t* src = p.image + boff + ek;
-            for (uint32_t o = 16u * lane; o < lk; o += 512u) cp_async16(sRec + pos + o, src + o, 16u);
-            asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bRecFull + 8 * d) : "memory");
+            for (uint32_t o = 16u * lane; o < lk; o += 512u) cp_async16(sRecP + pos + o, src + o, 16u);
+            asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bRecFullP + 8 * d) : "memory");
           }
 #else
           if (lane >= sb && lane < sb + m) {
             int d = d0 + (lane - sb);
-            if (d >= kRecSlots) d -= kRecSlots;
+            if (d >= kSlotsPP) d -= kSlotsPP;
             const uint32_t start = h0 + (excl - e0);
             const uint32_t pos = start & (uint32_t)(C::kRecRing - 1);
-            rec_end[d] = start + len;
-            rec_off[d] = pos;
-            mbar_arrive_tx(bRecFull + 8 * d, len);
-            bulk_g2s(sRec + pos, p.image + boff + excl, len, bRecFull + 8 * d);
+            rec_endP[d] = start + len;
+            rec_offP[d] = pos;
+            mbar_arrive_tx(bRecFullP + 8 * d, len);
+            bulk_g2s(sRecP + pos, p.image + boff + excl, len, bRecFullP + 8 * d);
           }
 #endif
           if (lane == 0) {
-            if (NM_TRACE_ON && p.trace && blockIdx.x == 0 && i < 1024) p.trace[i * 8] = clock64();
+            if (NM_TRACE_ON && kProducers == 1 && p.trace && blockIdx.x == 0 && i < 1024) p.trace[i * 8] = clock64();
             head += total;
             in_flight += m;
             ds += m;
-            if (ds >= kRecSlots) ds -= kRecSlots;
+            if (ds >= kSlotsPP) ds -= kSlotsPP;
           }
           i += m;
           __syncwarp();
@@ -425,11 +443,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
     // the group walks only its own chunks j = group (mod kLoadGroups) of the CTA's chunk
     // sequence; stage j % kStages and record descriptor j % kRecSlots (both multiples of
     // kLoadGroups, so they advance by kLoadGroups with a phase flip on wrap-around)
+    // records: unit ordinal k comes from producer k % kProducers; a chunk's descriptor is its
+    // index among that producer's chunks (mod kSlotsPP), its use parity the quotient's bit 0
     int64_t i = group, i0 = 0;  // next own chunk, first chunk of the current unit
-    int s = group, rs = group;
-    uint32_t ph = 0, rph = 0;
+    int s = group;
+    uint32_t ph = 0;
+    int64_t pc0 = 0, pc1 = 0, pc2 = 0;  // chunks of producer 0 / 1 / 2 before the current unit
+    int pw = 0;                 // producer of the current unit
     int4 nxt = unit_entry(p, blockIdx.x);
-    for (int64_t u = blockIdx.x; u < p.n_units; u += ustep) {
+    for (int64_t u = blockIdx.x; u < p.n_units; u += ustep, pw = (pw + 1 == kProducers) ? 0 : pw + 1) {
       const int4 cur = nxt;
       nxt = unit_entry(p, u + ustep);
       const int ft = (int)(u % p.n_ftiles);
@@ -437,14 +459,19 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
       const int col0f = ft * BN + c16f * 8;
       const uint32_t colbytes = col0f >= p.F ? 0u : (p.F - col0f >= 8 ? 16u : (uint32_t)(p.F - col0f) * 2u);
       const uint16_t* xcol = p.X + (colbytes ? col0f : 0);
-      const int64_t i_end = i0 + cur.y;
+      const int64_t i_first = i0, i_end = i0 + cur.y;
       i0 = i_end;
+      const int64_t lbase = (pw == 0 ? pc0 : pw == 1 ? pc1 : pc2) - i_first;  // producer-local index = lbase + i
+      if (pw == 0) pc0 += cur.y; else if (pw == 1) pc1 += cur.y; else pc2 += cur.y;
       for (; i < i_end; i += kLoadGroups) {
+        const int64_t li = lbase + i;
+        const int rs = pw * kSlotsPP + (int)(li & (kSlotsPP - 1));
+        const uint32_t rph = (uint32_t)(li >> kSlotsShift) & 1u;
         mbar_wait(bEmpty + 8 * s, ph ^ 1);       // the MMA has finished with stage s
         if (t == 0) NM_TRACE(7);
         if (!(p.debug & 1024)) mbar_wait(bRecFull + 8 * rs, rph);  // the compressed record has landed
         if (t == 0) NM_TRACE(1);
-        const uint32_t rec = sRec + ((p.debug & 1024) ? 0u : rec_off[rs]);
+        const uint32_t rec = sRec + pw * C::kRingStride + ((p.debug & 1024) ? 0u : rec_off[rs]);
         // 8-row groups of consecutive X rows come in by TMA tile loads (one 8 x 64 box per
         // 64-column slab, written into the SW128 atom); the other rows by cp.async gathers
         const uint32_t cmask = (p.debug & 32) ? 0u : lds8(rec + kRecContOff);
@@ -559,8 +586,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
         if (t == 0) NM_TRACE(2);
         s += kLoadGroups;
         if (s >= C::kStages) { s -= C::kStages; ph ^= 1; }
-        rs += kLoadGroups;
-        if (rs >= kRecSlots) { rs -= kRecSlots; rph ^= 1; }
       }
     }
   } else if (warp == kWarpMma) {
