@@ -145,17 +145,18 @@ __device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) {
 // long waits (the epilogue waiting for a whole unit of MMAs): back off so the spinning warps
 // do not take issue slots from the loaders (ncu: 20% of executed instructions were this spin)
 __device__ __forceinline__ void mbar_wait_sleep(uint32_t a, uint32_t parity) {
+  // try_wait with a suspend-time hint: the warp is descheduled until the phase completes (or
+  // ~1 ms passes), so it neither spins nor oversleeps the hand-off
   uint32_t ok;
   for (;;) {
     asm volatile(
         "{\n\t.reg .pred P;\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2, %3;\n\t"
         "selp.u32 %0, 1, 0, P;\n\t}"
         : "=r"(ok)
-        : "r"(a), "r"(parity)
+        : "r"(a), "r"(parity), "r"(1000000)
         : "memory");
     if (ok) return;
-    __nanosleep(200);
   }
 }
 
@@ -197,13 +198,21 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t
   return d;
 }
 
+// unit u = (scheduled panel u / n_ftiles, F tile u % n_ftiles); n_units < 2^31 (host check),
+// so 32-bit division -- a 64-bit one is a ~70-instruction sequence on every role's unit step
+__device__ __forceinline__ uint32_t unit_panel(const SpmmParams& p, int64_t u) {
+  return p.n_ftiles == 1 ? (uint32_t)u : (uint32_t)u / (uint32_t)p.n_ftiles;
+}
+__device__ __forceinline__ int unit_ft(const SpmmParams& p, int64_t u) {
+  return p.n_ftiles == 1 ? 0 : (int)((uint32_t)u % (uint32_t)p.n_ftiles);
+}
 // schedule entry of unit u (prefetched one unit ahead by every role): {panel, #chunks, c0}
 __device__ __forceinline__ int4 unit_entry(const SpmmParams& p, int64_t u) {
-  return u < p.n_units ? __ldg(p.unit_info + 2 * (u / p.n_ftiles)) : make_int4(0, 0, 0, 0);
+  return u < p.n_units ? __ldg(p.unit_info + 2 * unit_panel(p, u)) : make_int4(0, 0, 0, 0);
 }
 // {record byte offset lo, hi, record bytes lo, hi} of unit u
 __device__ __forceinline__ int4 unit_bytes(const SpmmParams& p, int64_t u) {
-  return u < p.n_units ? __ldg(p.unit_info + 2 * (u / p.n_ftiles) + 1) : make_int4(0, 0, 0, 0);
+  return u < p.n_units ? __ldg(p.unit_info + 2 * unit_panel(p, u) + 1) : make_int4(0, 0, 0, 0);
 }
 __device__ __forceinline__ int64_t entry_c0(int4 e) { return (int64_t)(uint32_t)e.z | ((int64_t)e.w << 32); }
 __device__ __forceinline__ int64_t lo_hi(int a, int b) { return (int64_t)(uint32_t)a | ((int64_t)b << 32); }
@@ -224,7 +233,8 @@ struct Cfg {
       kRingPer >= 64 * 1024 ? 64 * 1024 : kRingPer >= 32 * 1024 ? 32 * 1024 : 16 * 1024;
   static constexpr int kRingStride = kRecRing + kRecMaxBytes; // ring + wrap pad per producer
   static constexpr int kRecRegion = kProducers * kRingStride;
-  static constexpr int kNAcc = (2 * BN + kStages <= 512) ? 2 : 1;
+  // accumulators in TMEM (units in flight between the MMA issuer and the epilogue)
+  static constexpr int kNAcc = (3 * BN + kStages <= 512) ? 3 : (2 * BN + kStages <= 512) ? 2 : 1;
   static constexpr int kMeta0 = kNAcc * BN;                     // metadata column of stage s: kMeta0 + s
   static constexpr int kBRegion = kStages * kBBytes;            // 1024-aligned tiles (SW128)
   static constexpr int kSmem = 1024 + kBRegion + kStages * kABytes + kRecRegion + 2048;
@@ -249,8 +259,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
   uint64_t* full_b = rec_empty + kRecSlots; // A tile + gathers + metadata ready
   uint64_t* empty = full_b + C::kStages;    // MMA done with the stage (tcgen05.commit)
   uint64_t* tfull = empty + C::kStages;     // accumulator ready (2)
-  uint64_t* tempty = tfull + 2;             // accumulator drained (2)
-  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  uint64_t* tempty = tfull + 4;             // accumulator drained (kNAcc <= 4)
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 4);
   uint32_t* rec_off = tmem_slot + 4;        // [kRecSlots] ring offset of each descriptor's record
   uint32_t* rec_end = rec_off + kRecSlots;  // [kRecSlots] producer-private: cumulative end of each record
 
@@ -271,7 +281,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
       mbar_init(smem_u32(&full_b[s]), kGroupThreads + kGroupThreads / 32);
       mbar_init(smem_u32(&empty[s]), 1);
     }
-    for (int a = 0; a < 2; ++a) {
+    for (int a = 0; a < 4; ++a) {
       mbar_init(smem_u32(&tfull[a]), 1);
       mbar_init(smem_u32(&tempty[a]), kEpiWarps);
     }
@@ -454,7 +464,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
     for (int64_t u = blockIdx.x; u < p.n_units; u += ustep, pw = (pw + 1 == kProducers) ? 0 : pw + 1) {
       const int4 cur = nxt;
       nxt = unit_entry(p, u + ustep);
-      const int ft = (int)(u % p.n_ftiles);
+      const int ft = unit_ft(p, u);
       // this thread's gather column piece (kFixedCol): source offset and byte count
       const int col0f = ft * BN + c16f * 8;
       const uint32_t colbytes = col0f >= p.F ? 0u : (p.F - col0f >= 8 ? 16u : (uint32_t)(p.F - col0f) * 2u);
@@ -620,7 +630,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
         // the A tile (st.shared) and the gathers (cp.async) were written through the generic
         // proxy: make them visible to the tensor core's async-proxy operand reads (without
         // this fence stale stage contents were observed on B200 -- test_parity_fullsize.py)
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        if (!(p.debug & 16)) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         // metadata column: even column address + sparse_id2 selects the odd one
         asm volatile(
@@ -692,7 +702,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
 #pragma unroll
           for (int h = 0; h < 2; ++h) nrow[b][h] = out_row(nxt, row_of(b, h));
       }
-      const int ft = (int)(u % p.n_ftiles);
+      const int ft = unit_ft(p, u);
       const bool has = cur.y > 0;
       const bool full_tile = vec_ok && ft * BN + BN <= p.F;
       mbar_wait_sleep(bTfull + 8 * acc, aphase);
@@ -809,6 +819,8 @@ nm_status launch_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, 
   prm.rows = P->row_end - P->row_begin;
   prm.n_ftiles = (F + BN - 1) / BN;
   prm.n_units = P->n_panels * prm.n_ftiles;
+  if (prm.n_units + 4 * (int64_t)sms >= ((int64_t)1 << 31))
+    return fail(NM_ERR_UNSUPPORTED, "nm_spmm: too many work units for one launch (row-shard the matrix)");
   prm.idesc = make_idesc(P->dtype, BN);
   const char* dbg = getenv("NM_SPMM_DEBUG");
   prm.debug = dbg ? atoi(dbg) : 0;
