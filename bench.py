@@ -10,7 +10,8 @@ a5-a8), with the permutations folded into the SpMM's gather/scatter indices
 packing (a4) are offline preprocessing -- run and reported, not timed.
 
 Multi-GPU (torchrun, N > 1): the rows of B = P A P^T are split into contiguous,
-panel-aligned blocks, one per rank, X replicated; the SpMM needs no exchange
+panel-aligned blocks of balanced cost (stored entries + Y rows), one per rank, X replicated
+(SURVEY §8(e)); the SpMM needs no exchange
 (the GCN driver in paper_conf_ppopp_chensz0s25_b200/dist.py all-gathers).  Total work is
 fixed: "scaling": "strong".  Time = max over ranks of the device-timed region.
 """
@@ -265,8 +266,9 @@ def main():
         hb = buf.cpu().numpy()
         perm = hb[:n].astype(np.int32)
         rst = {k: (float(v) if k == "seconds" else int(v)) for k, v in zip(keys, hb[n:])}
-    from paper_conf_ppopp_chensz0s25_b200.dist import shard_rows
-    rb, re = shard_rows(n, world, rank)
+    # contiguous panel-aligned row blocks balanced by stored entries + Y rows
+    from paper_conf_ppopp_chensz0s25_b200.dist import balanced_bounds, panel_costs
+    rb, re = balanced_bounds(panel_costs(ip, perm), n, world)[rank]
     t0 = time.perf_counter()
     tau = w["tau"] if w["tau"] is not None else api.hybrid_tau(F)
     P = api.pack(ip, ic, perm, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order=args.order, tau=tau)

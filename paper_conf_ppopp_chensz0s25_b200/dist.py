@@ -3,6 +3,10 @@
 
 * ``shard_rows``: contiguous, panel-aligned (128-row) blocks of B = P A P^T, one per rank,
   equal panel counts (the last rank takes the remainder).
+* ``balanced_bounds`` / ``panel_costs``: contiguous, panel-aligned blocks
+  whose summed per-panel cost (stored entries of the panel's rows + a per-row term for the
+  Y writes) is as equal as the panel granularity allows -- power-law rows make equal-row
+  shards unequal in work.
 * ``gcn_forward``: a K-layer GCN forward (Eq. 1) in the permuted vertex order with
   X replicated: per layer each rank computes its row block of Ahat (H W) with libnm
   (nm_gcn_layer) and the next layer's full operand is assembled with one NCCL
@@ -31,13 +35,57 @@ def padded_rows(n: int, world: int, panel: int = PANEL) -> int:
     return ((P + world - 1) // world) * panel
 
 
-def gcn_forward(H, layers, local_layer, group=None):
+def panel_costs(ip, perm, panel: int = PANEL, row_weight: float = 8.0):
+    """Per-panel cost of B = P A P^T: sum over the panel's rows p of deg(perm[p]) +
+    row_weight (the Y row write, in units of one stored entry).  ip: CSR row pointer of A."""
+    import numpy as np
+    deg = np.diff(np.asarray(ip, dtype=np.int64))[np.asarray(perm, dtype=np.int64)]
+    n = deg.shape[0]
+    P = (n + panel - 1) // panel
+    pad = np.zeros(P * panel, dtype=np.float64)
+    pad[:n] = deg + row_weight
+    return pad.reshape(P, panel).sum(axis=1)
+
+
+def balanced_bounds(costs, n: int, world: int, panel: int = PANEL):
+    """[(row_begin, row_end)] per rank: contiguous panel ranges minimising the largest summed
+    cost (the linear-partition bottleneck: bisection on the bound, greedy packing decides
+    feasibility), so no contiguous panel-aligned split -- equal rows included -- has a smaller
+    maximum.  Trailing ranks may be empty."""
+    import numpy as np
+    costs = np.asarray(costs, dtype=np.float64)
+    P = costs.shape[0]
+
+    def pack(T):  # greedy: start a new block when the next panel would exceed T
+        cuts, acc = [0], 0.0
+        for i, c in enumerate(costs):
+            if acc + c > T and acc > 0:
+                cuts.append(i)
+                acc = 0.0
+            acc += c
+        return cuts
+
+    lo, hi = (float(costs.max()) if P else 0.0), float(costs.sum())
+    for _ in range(64):
+        mid = 0.5 * (lo + hi)
+        if len(pack(mid)) <= world:
+            hi = mid
+        else:
+            lo = mid
+    cuts = pack(hi)
+    cuts = cuts + [P] * (world + 1 - len(cuts))
+    return [(min(n, a * panel), min(n, b * panel)) for a, b in zip(cuts[:-1], cuts[1:])]
+
+
+def gcn_forward(H, layers, local_layer, group=None, bounds=None):
     """Multi-layer GCN forward with one all-gather per layer.
 
     H: full [n x F0] input (permuted order, replicated on every rank).
     layers: list of (W, bias, relu) per layer.
     local_layer(l, H_full, W, bias, relu, rb, re) -> this rank's rows [re-rb x F_out] of
         act(Ahat (H_full W) + bias) for layer l.
+    bounds: optional [(row_begin, row_end)] per rank (e.g. balanced_bounds); default equal
+        panel counts (shard_rows).  Shards are padded to the largest one for the collective.
     Returns the full [n x F_L] output on every rank.
     """
     import torch
@@ -46,8 +94,11 @@ def gcn_forward(H, layers, local_layer, group=None):
     world = dist.get_world_size(group) if dist.is_initialized() else 1
     rank = dist.get_rank(group) if dist.is_initialized() else 0
     n = H.shape[0]
-    rb, re = shard_rows(n, world, rank)
-    rows_pad = padded_rows(n, world)
+    if bounds is None:
+        bounds = [shard_rows(n, world, r) for r in range(world)]
+    assert len(bounds) == world and bounds[0][0] == 0 and bounds[-1][1] == n
+    rb, re = bounds[rank]
+    rows_pad = max(1, max(b - a for a, b in bounds))
     cur = H
     for li, (W, bias, relu) in enumerate(layers):
         out_loc = local_layer(li, cur, W, bias, relu, rb, re)
@@ -61,8 +112,7 @@ def gcn_forward(H, layers, local_layer, group=None):
         dist.all_gather_into_tensor(full, send, group=group)
         # drop each rank's padding rows
         parts = []
-        for r in range(world):
-            a, b = shard_rows(n, world, r)
+        for r, (a, b) in enumerate(bounds):
             parts.append(full[r * rows_pad: r * rows_pad + (b - a)])
         cur = torch.cat(parts, dim=0)
     return cur

@@ -27,6 +27,31 @@ def test_shard_rows_partition(n, world):
         assert b - a <= nmdist.padded_rows(n, world)
 
 
+@pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
+@pytest.mark.parametrize("seed", [0, 1])
+def test_balanced_bounds_partition_and_balance(world, seed):
+    """Cost-balanced shards: a contiguous panel-aligned partition of all rows,
+    and no rank exceeds the ideal share by more than one panel's cost -- on a power-law graph
+    where equal-row shards are clearly unbalanced."""
+    n = 5000
+    ip, ic = graphs.lmcl_graph(n, 30000, 2.1, 1, 0.0, seed, scramble=False)
+    perm = np.arange(n, dtype=np.int32)
+    costs = nmdist.panel_costs(ip, perm)
+    assert costs.shape[0] == (n + 127) // 128
+    assert costs.sum() == pytest.approx(ip[-1] + 8.0 * n)
+    bounds = nmdist.balanced_bounds(costs, n, world)
+    assert bounds[0][0] == 0 and bounds[-1][1] == n
+    for (a, b), (c, d) in zip(bounds[:-1], bounds[1:]):
+        assert b == c
+    for a, b in bounds:
+        assert a <= b and (a % 128 == 0 or a == n)
+    share = [costs[a // 128:(b + 127) // 128].sum() for a, b in bounds]
+    assert max(share) <= costs.sum() / world + costs.max() + 1e-9
+    if world > 1:
+        eq = [costs[a // 128:(b + 127) // 128].sum() for a, b in (nmdist.shard_rows(n, world, r) for r in range(world))]
+        assert max(share) <= max(eq) + 1e-9
+
+
 def _free_port():
     s = socket.socket()
     s.bind(("127.0.0.1", 0))
@@ -61,26 +86,35 @@ def _local_layer_factory(ip, ic, vals):
     return local_layer
 
 
-def _worker(rank, world, port, q):
+def _bounds(ip, world, balanced):
+    if not balanced:
+        return None
+    n = len(ip) - 1
+    return nmdist.balanced_bounds(nmdist.panel_costs(ip, np.arange(n)), n, world)
+
+
+def _worker(rank, world, port, q, balanced=False):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     ip, ic, vals, H, Ws, bs = _problem()
     layers = [(Ws[0], bs[0], True), (Ws[1], bs[1], False)]
-    out = nmdist.gcn_forward(torch.from_numpy(H), layers, _local_layer_factory(ip, ic, vals))
+    out = nmdist.gcn_forward(torch.from_numpy(H), layers, _local_layer_factory(ip, ic, vals),
+                             bounds=_bounds(ip, world, balanced))
     q.put((rank, out.numpy()))
     dist.barrier()
     dist.destroy_process_group()
 
 
-def test_gcn_forward_gloo_world2_matches_single_process():
+@pytest.mark.parametrize("balanced", [False, True])
+def test_gcn_forward_gloo_world2_matches_single_process(balanced):
     ip, ic, vals, H, Ws, bs = _problem()
     layers = [(Ws[0], bs[0], True), (Ws[1], bs[1], False)]
     ref = nmdist.gcn_forward(torch.from_numpy(H), layers, _local_layer_factory(ip, ic, vals)).numpy()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, balanced)) for r in range(2)]
     for p in procs:
         p.start()
     got = dict(q.get(timeout=120) for _ in range(2))
