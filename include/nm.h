@@ -253,6 +253,25 @@ NM_API nm_status nm_gcn_layer(const nm_packed* Ahat, const void* H, const void* 
                        void* Hout, int F_in, int F_out, int flags, void* ws, size_t ws_bytes,
                        void* stream);
 
+/* nm_gcn_layer_backward -- gradients of nm_gcn_layer (linear-first or aggregate-first give the
+ * same Z = Ahat (H W) + b), SURVEY §8(f) item 4:
+ *   dZ = dHout * act'(Z) (ReLU: Hout > 0), db = column sums of dZ, dT = Ahat^T dZ = Ahat dZ
+ *   (Ahat symmetric: the reorder keeps the adjacency symmetric, PAPER.md L69-79 / L725, so the
+ *   same pack serves the backward aggregation), dW = H^T dT, dH = dT W^T.
+ *   Ahat : the whole matrix (row_begin 0, row_end n) packed in permuted order (flags 0).
+ *   H    : n x F_in, W : F_in x F_out, Hout / dHout : n x F_out -- device, row-major, dtype of
+ *          the pack (16-bit), permuted vertex order.
+ *   dH   : n x F_in 16-bit (nullable: skipped), dW : F_in x F_out fp32, db : F_out fp32
+ *          (nullable).  dT is rounded to 16-bit once before the two GEMMs (cuBLASLt, fp32
+ *          accumulation).
+ *   flags: NM_RELU or 0.  ws: nm_gcn_backward_workspace_bytes(n, F_in, F_out) bytes.
+ *   Stream-ordered.  Errors: INVALID_ARG, UNSUPPORTED (row shard, fused-order pack, F not a
+ *   multiple of 8), CUDA. */
+NM_API size_t nm_gcn_backward_workspace_bytes(int64_t n, int F_in, int F_out);
+NM_API nm_status nm_gcn_layer_backward(const nm_packed* Ahat, const void* H, const void* W, const void* Hout,
+                                       const void* dHout, void* dH, float* dW, float* db, int F_in, int F_out,
+                                       int flags, void* ws, size_t ws_bytes, void* stream);
+
 /* ------------------------------------------------------------------------------------- */
 NM_API const char* nm_status_string(nm_status s);
 NM_API const char* nm_last_error(void);   /* thread-local detail of the last failure on this thread */

@@ -281,3 +281,37 @@ def unpack(pk: dict, n: int):
             Bd[i, rc[k]] = rv[k]
             present[i, rc[k]] = True
     return Bd, present
+
+
+def csr_transpose(indptr, indices, val):
+    """A^T of a CSR matrix (plain counting sort; no symmetry assumed)."""
+    indptr = np.asarray(indptr, dtype=np.int64)
+    indices = np.asarray(indices, dtype=np.int64)
+    val = np.asarray(val, dtype=np.float64)
+    n = indptr.shape[0] - 1
+    rows = np.repeat(np.arange(n), np.diff(indptr))
+    order = np.lexsort((rows, indices))  # by column, then row
+    tp = np.concatenate([[0], np.cumsum(np.bincount(indices, minlength=n))]).astype(np.int64)
+    return tp, rows[order].astype(np.int32), val[order]
+
+
+def gcn_layer(indptr, indices, val, H, W, b, relu: bool):
+    """Eq. 1 in fp64: Hout = act(A (H W) + b); returns (Hout, Z)."""
+    XW = np.asarray(H, dtype=np.float64) @ np.asarray(W, dtype=np.float64)
+    Z, _, _ = spmm(indptr, indices, val, XW)
+    Z = Z + np.asarray(b, dtype=np.float64)
+    return (np.maximum(Z, 0.0) if relu else Z), Z
+
+
+def gcn_layer_backward(indptr, indices, val, H, W, Z, dHout, relu: bool):
+    """Gradients of gcn_layer for the upstream gradient dHout, step by step in fp64 (SURVEY
+    §8(f) item 4): dZ = dHout * act'(Z); db = sum over rows of dZ; dT = A^T dZ (the transpose
+    is formed explicitly -- the oracle does not assume A symmetric); dW = H^T dT; dH = dT W^T.
+    Pinned by central finite differences (tests/test_oracle_gcn_backward.py)."""
+    dZ = np.asarray(dHout, dtype=np.float64) * ((np.asarray(Z) > 0) if relu else 1.0)
+    db = dZ.sum(axis=0)
+    tp, ti, tv = csr_transpose(indptr, indices, val)
+    dT, _, _ = spmm(tp, ti, tv, dZ)
+    dW = np.asarray(H, dtype=np.float64).T @ dT
+    dH = dT @ np.asarray(W, dtype=np.float64).T
+    return dH, dW, db, dT

@@ -227,3 +227,17 @@ def gcn_layer(P: Packed, H, W, bias, Hout, ws, relu=True, order="linear", stream
     L.check(L.load().nm_gcn_layer(P.handle, _ptr(H), _ptr(W), _ptr(bias), _ptr(Hout), H.shape[1],
                                   W.shape[1], flags, _ptr(ws), ws.numel(), _stream_ptr(stream)),
             "nm_gcn_layer")
+
+
+def gcn_backward_workspace_bytes(n, F_in, F_out):
+    return int(L.load().nm_gcn_backward_workspace_bytes(n, F_in, F_out))
+
+
+def gcn_layer_backward(P: Packed, H, W, Hout, dHout, dH, dW, db, ws, relu=True, stream=None):
+    """nm_gcn_layer_backward: dW (fp32), db (fp32, optional) and dH (16-bit, optional) of
+    Hout = act(Ahat (H W) + b) for the upstream gradient dHout (Ahat^T = Ahat)."""
+    L.check(L.load().nm_gcn_layer_backward(P.handle, _ptr(H), _ptr(W), _ptr(Hout), _ptr(dHout), _ptr(dH),
+                                           _ptr(dW), _ptr(db), H.shape[1], W.shape[1],
+                                           L.NM_RELU if relu else 0, _ptr(ws), ws.numel(),
+                                           _stream_ptr(stream)),
+            "nm_gcn_layer_backward")

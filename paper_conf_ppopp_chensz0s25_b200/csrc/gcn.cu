@@ -116,6 +116,78 @@ nm_status dense_gemm(const void* A, const void* W, void* C, int64_t m, int k, in
   return st;
 }
 
+// General column-major product C[m x nn] = op(A)[m x k] op(B)[k x nn] (cuBLASLt, fp32
+// accumulation); A/B 16-bit, C 16-bit or fp32; lda/ldb/ldc are column-major leading dims.
+nm_status lt_gemm(bool ta, bool tb, int64_t m, int64_t nn, int64_t k, const void* A, int64_t lda, const void* B,
+                  int64_t ldb, void* C, int64_t ldc, nm_dtype dt, bool c_f32, void* ws, cudaStream_t s) {
+  static thread_local LtHandle lt;
+  if (!lt.h) {
+    cublasStatus_t r = cublasLtCreate(&lt.h);
+    if (r != CUBLAS_STATUS_SUCCESS) return lt_fail(r, "cublasLtCreate");
+  }
+  if (m == 0 || nn == 0) return NM_OK;
+  const cudaDataType_t ty = dt == NM_BF16 ? CUDA_R_16BF : CUDA_R_16F;
+  const cudaDataType_t cty = c_f32 ? CUDA_R_32F : ty;
+  cublasLtMatmulDesc_t op = nullptr;
+  cublasLtMatrixLayout_t la = nullptr, lb = nullptr, lc = nullptr;
+  cublasLtMatmulPreference_t pref = nullptr;
+  nm_status st = NM_OK;
+  do {
+    if (cublasLtMatmulDescCreate(&op, CUBLAS_COMPUTE_32F, CUDA_R_32F) != CUBLAS_STATUS_SUCCESS) {
+      st = fail(NM_ERR_CUDA, "cublasLtMatmulDescCreate");
+      break;
+    }
+    const cublasOperation_t opa = ta ? CUBLAS_OP_T : CUBLAS_OP_N, opb = tb ? CUBLAS_OP_T : CUBLAS_OP_N;
+    cublasLtMatmulDescSetAttribute(op, CUBLASLT_MATMUL_DESC_TRANSA, &opa, sizeof(opa));
+    cublasLtMatmulDescSetAttribute(op, CUBLASLT_MATMUL_DESC_TRANSB, &opb, sizeof(opb));
+    if (cublasLtMatrixLayoutCreate(&la, ty, ta ? k : m, ta ? m : k, lda) != CUBLAS_STATUS_SUCCESS ||
+        cublasLtMatrixLayoutCreate(&lb, ty, tb ? nn : k, tb ? k : nn, ldb) != CUBLAS_STATUS_SUCCESS ||
+        cublasLtMatrixLayoutCreate(&lc, cty, m, nn, ldc) != CUBLAS_STATUS_SUCCESS) {
+      st = fail(NM_ERR_CUDA, "cublasLtMatrixLayoutCreate");
+      break;
+    }
+    if (cublasLtMatmulPreferenceCreate(&pref) != CUBLAS_STATUS_SUCCESS) {
+      st = fail(NM_ERR_CUDA, "cublasLtMatmulPreferenceCreate");
+      break;
+    }
+    size_t wsb = kLtWorkspace;
+    cublasLtMatmulPreferenceSetAttribute(pref, CUBLASLT_MATMUL_PREF_MAX_WORKSPACE_BYTES, &wsb, sizeof(wsb));
+    cublasLtMatmulHeuristicResult_t heur;
+    int nres = 0;
+    if (cublasLtMatmulAlgoGetHeuristic(lt.h, op, la, lb, lc, lc, pref, 1, &heur, &nres) != CUBLAS_STATUS_SUCCESS ||
+        nres == 0) {
+      st = fail(NM_ERR_CUDA, "cublasLt: no algorithm");
+      break;
+    }
+    const float one = 1.f, zero = 0.f;
+    cublasStatus_t r = cublasLtMatmul(lt.h, op, &one, A, la, B, lb, &zero, C, lc, C, lc, &heur.algo, ws, wsb, s);
+    if (r != CUBLAS_STATUS_SUCCESS) st = lt_fail(r, "cublasLtMatmul");
+  } while (0);
+  if (pref) cublasLtMatmulPreferenceDestroy(pref);
+  if (la) cublasLtMatrixLayoutDestroy(la);
+  if (lb) cublasLtMatrixLayoutDestroy(lb);
+  if (lc) cublasLtMatrixLayoutDestroy(lc);
+  if (op) cublasLtMatmulDescDestroy(op);
+  return st;
+}
+
+// dZ = relu ? dHout * [Hout > 0] : dHout (16-bit in and out, exact), and a 16-bit ones
+// vector (the column sums of dZ are a GEMM with it)
+__global__ void k_relu_grad(const uint16_t* __restrict__ dHout, const uint16_t* __restrict__ Hout, int64_t total,
+                            int relu, uint16_t* __restrict__ dZ) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint16_t h = Hout[i];
+    // fp16 and bf16 share the sign bit; h > 0 <=> sign clear and not (+0)
+    const bool pos = !(h & 0x8000u) && (h & 0x7FFFu);
+    dZ[i] = (!relu || pos) ? dHout[i] : (uint16_t)0;
+  }
+}
+
+__global__ void k_fill16(uint16_t* __restrict__ a, int64_t n, uint16_t v) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    a[i] = v;
+}
+
 inline int grid_for(int64_t total) {
   int64_t g = (total + 255) / 256;
   if (g > 148 * 16) g = 148 * 16;
@@ -174,5 +246,64 @@ extern "C" nm_status nm_gcn_layer(const nm_packed* Ahat, const void* H, const vo
   if (bf) k_bias_act<1><<<grid_for(rows * F_out), 256, 0, s>>>(pre, rows, F_out, bias, flags & NM_RELU, (uint16_t*)Hout);
   else k_bias_act<0><<<grid_for(rows * F_out), 256, 0, s>>>(pre, rows, F_out, bias, flags & NM_RELU, (uint16_t*)Hout);
   NM_CUDA(cudaGetLastError());
+  return NM_OK;
+}
+
+// ---- backward ----------------------------------------------------------
+// Z = Ahat (H W) + b, Hout = act(Z).  With dZ = dHout * act'(Z) (act' from Hout > 0 for ReLU):
+//   db = 1^T dZ,   dT = Ahat^T dZ = Ahat dZ   (Ahat is symmetric -- the reorder keeps the
+//   adjacency symmetric, PAPER.md L69-79 / L725 -- so the same packed matrix serves the
+//   backward aggregation),   dW = H^T dT,   dH = dT W^T.
+extern "C" size_t nm_gcn_backward_workspace_bytes(int64_t n, int F_in, int F_out) {
+  (void)F_in;
+  return align256((size_t)n * 2) + 2 * align256((size_t)n * F_out * 2) + align256((size_t)n * F_out * 4) +
+         kLtWorkspace;
+}
+
+extern "C" nm_status nm_gcn_layer_backward(const nm_packed* Ahat, const void* H, const void* W, const void* Hout,
+                                           const void* dHout, void* dH, float* dW, float* db, int F_in, int F_out,
+                                           int flags, void* ws, size_t ws_bytes, void* stream) {
+  if (!Ahat || !H || !W || !Hout || !dHout || !dW || !ws)
+    return fail(NM_ERR_INVALID_ARG, "nm_gcn_layer_backward: NULL argument");
+  if (F_in < 1 || F_out < 1 || F_out % 8 != 0 || F_in % 8 != 0)
+    return fail(NM_ERR_UNSUPPORTED, "nm_gcn_layer_backward: F_in and F_out must be positive multiples of 8");
+  if (flags & ~NM_RELU) return fail(NM_ERR_INVALID_ARG, "nm_gcn_layer_backward: unknown flags");
+  if (Ahat->row_map) return fail(NM_ERR_UNSUPPORTED, "nm_gcn_layer_backward: needs a pack in permuted order");
+  const int64_t n = Ahat->n;
+  if (Ahat->row_begin != 0 || Ahat->row_end != n)
+    return fail(NM_ERR_UNSUPPORTED, "nm_gcn_layer_backward: needs the whole matrix (Ahat^T = Ahat), not a row shard");
+  if (ws_bytes < nm_gcn_backward_workspace_bytes(n, F_in, F_out))
+    return fail(NM_ERR_INVALID_ARG, "nm_gcn_layer_backward: workspace too small");
+  if (n == 0) return NM_OK;
+  cudaStream_t s = (cudaStream_t)stream;
+  const nm_dtype dt = Ahat->dtype;
+  uint8_t* w8 = (uint8_t*)ws;
+  uint16_t* ones = (uint16_t*)w8;
+  uint16_t* dZ = (uint16_t*)(w8 + align256((size_t)n * 2));
+  float* dT32 = (float*)((uint8_t*)dZ + align256((size_t)n * F_out * 2));
+  uint16_t* dT16 = (uint16_t*)((uint8_t*)dT32 + align256((size_t)n * F_out * 4));
+  void* lt_ws = (uint8_t*)dT16 + align256((size_t)n * F_out * 2);
+  const int64_t tot = n * F_out;
+  k_relu_grad<<<grid_for(tot), 256, 0, s>>>((const uint16_t*)dHout, (const uint16_t*)Hout, tot, flags & NM_RELU, dZ);
+  NM_CUDA(cudaGetLastError());
+  nm_status st;
+  if (db) {  // db[1 x F_out] = ones[1 x n] dZ[n x F_out]
+    k_fill16<<<grid_for(n), 256, 0, s>>>(ones, n, dt == NM_BF16 ? (uint16_t)0x3F80u : (uint16_t)0x3C00u);
+    NM_CUDA(cudaGetLastError());
+    st = dense_gemm(ones, dZ, db, 1, (int)n, F_out, dt, true, lt_ws, s);
+    if (st != NM_OK) return st;
+  }
+  st = nm_spmm(Ahat, dZ, F_out, dT32, F_out, F_out, stream);  // dT = Ahat dZ
+  if (st != NM_OK) return st;
+  if (dt == NM_BF16) k_to16<1><<<grid_for(tot), 256, 0, s>>>(dT32, tot, dT16);
+  else k_to16<0><<<grid_for(tot), 256, 0, s>>>(dT32, tot, dT16);
+  NM_CUDA(cudaGetLastError());
+  // column-major views: row-major X[r x c] is X^c[c x r].  dW^c[F_out x F_in] = dT^c H^c^T
+  st = lt_gemm(false, true, F_out, F_in, n, dT16, F_out, H, F_in, dW, F_out, dt, true, lt_ws, s);
+  if (st != NM_OK) return st;
+  if (dH) {  // dH^c[F_in x n] = W^c^T dT^c
+    st = lt_gemm(true, false, F_in, n, F_out, W, F_out, dT16, F_out, dH, F_in, dt, false, lt_ws, s);
+    if (st != NM_OK) return st;
+  }
   return NM_OK;
 }

@@ -107,3 +107,52 @@ def test_gcn_layer_aggregate_first_and_row_shards(n, fin, fout, V, M, shards):
     ref = np.maximum(Ya @ w64 + b, 0.0)
     bound = 3e-3 * (Ea @ np.abs(w64)) + 2.0 ** -8 * np.abs(ref) + 1e-30
     assert (np.abs(got - ref) <= bound).all(), np.abs(got - ref).max()
+
+
+@pytest.mark.parametrize("n,fin,fout,V,M", [(2048, 64, 32, 1, 4), (1500, 96, 128, 8, 8)])
+@pytest.mark.parametrize("relu", [True, False])
+def test_gcn_layer_backward(n, fin, fout, V, M, relu):
+    """nm_gcn_layer_backward vs the oracle's fp64 backward, which forms
+    Ahat^T explicitly (the GPU reuses the same pack: Ahat^T = Ahat).  The ReLU mask is the
+    GPU's Hout > 0 on both sides; db within 1e-3 of sum |dZ|; dW, dH (dT rounded to bf16 once)
+    within a relative Frobenius error of 1e-2."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    dev = torch.device("cuda:0")
+    ip, ic = graphs.er_graph(n, 6 * n, 7, self_loops=True)
+    vals = _gcn_norm(ip, ic)
+    vbits, v64 = graphs.round16(vals, "bf16")
+    perm, _ = api.reorder(ip, ic, V, 2, M)
+    P = api.pack(ip, ic, perm, V, 2, M, dtype="bf16", val=vals)
+    rng = np.random.default_rng(2)
+    hb, h64 = graphs.round16(rng.standard_normal((n, fin)).astype(np.float32), "bf16")
+    wb, w64 = graphs.round16((rng.standard_normal((fin, fout)) / np.sqrt(fin)).astype(np.float32), "bf16")
+    gb, g64 = graphs.round16(rng.standard_normal((n, fout)).astype(np.float32), "bf16")
+    b = rng.standard_normal(fout).astype(np.float32)
+    tb = lambda a: torch.from_numpy(a.view(np.int16)).to(dev).view(torch.bfloat16)
+    pd = torch.from_numpy(perm).to(dev)
+    H, W, G = tb(hb), tb(wb), tb(gb)
+    PH, PG = torch.empty_like(H), torch.empty_like(G)
+    api.permute_rows(H, PH, pd, "bf16")
+    api.permute_rows(G, PG, pd, "bf16")
+    ws = torch.empty(api.gcn_workspace_bytes(n, fin, fout), dtype=torch.uint8, device=dev)
+    Hout = torch.empty((n, fout), dtype=torch.bfloat16, device=dev)
+    api.gcn_layer(P, PH, W, torch.from_numpy(b).to(dev), Hout, ws, relu=relu)
+    wsb = torch.empty(api.gcn_backward_workspace_bytes(n, fin, fout), dtype=torch.uint8, device=dev)
+    dH = torch.empty((n, fin), dtype=torch.bfloat16, device=dev)
+    dW = torch.empty((fin, fout), dtype=torch.float32, device=dev)
+    db = torch.empty(fout, dtype=torch.float32, device=dev)
+    api.gcn_layer_backward(P, PH, W, Hout, PG, dH, dW, db, wsb, relu=relu)
+    torch.cuda.synchronize()
+    hout_p = graphs.bf16_bits_to_f64(Hout.view(torch.int16).cpu().numpy().view(np.uint16))
+    hout = np.empty_like(hout_p)
+    hout[perm] = hout_p
+    dH_ref, dW_ref, db_ref, _ = oracle.gcn_layer_backward(ip, ic, v64, h64, w64, hout, g64, relu)
+    dZ = g64 * ((hout > 0) if relu else 1.0)
+    assert np.all(np.abs(db.cpu().numpy() - db_ref) <= 1e-3 * np.abs(dZ).sum(0) + 1e-6)
+    got_dw = dW.cpu().numpy().astype(np.float64)
+    assert np.linalg.norm(got_dw - dW_ref) <= 1e-2 * np.linalg.norm(dW_ref)
+    dh_p = graphs.bf16_bits_to_f64(dH.view(torch.int16).cpu().numpy().view(np.uint16))
+    got_dh = np.empty_like(dh_p)
+    got_dh[perm] = dh_p
+    assert np.linalg.norm(got_dh - dH_ref) <= 1e-2 * np.linalg.norm(dH_ref)
