@@ -5,6 +5,10 @@
 
 #include "nm_internal.h"
 
+#ifndef NM_RES_UNROLL
+#define NM_RES_UNROLL 2  // X rows in flight per lane in k_residual (measured: 2 >= 4 >> 8)
+#endif
+
 namespace nm {
 namespace {
 
@@ -28,7 +32,7 @@ __device__ __forceinline__ float fma16(unsigned short a, unsigned short b, float
 // flight; a lane owns 8 consecutive features of the launch's slab [f_base, f_base + LPR*8)
 // and reads them with one 16-byte load per nonzero.  The item's (col, val) pairs are fetched
 // LPR at a time with one coalesced load and broadcast within the subgroup by shuffles; the
-// loop is unrolled so kUnroll X rows are in flight per lane.  The next item's descriptor is
+// loop is unrolled so kUnroll X rows are in flight per lane (2: more costs occupancy).  The next item's descriptor is
 // prefetched, and the Y row (addressed by the item's output row, row_map applied at pack
 // time) is read next to the first (col, val) batch.  A row with one item adds its sum into Y;
 // the items of a split row (hub rows) write partials to their workspace slots and the last
@@ -42,7 +46,7 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
                                                   float* __restrict__ Y, int64_t ldy, int F, int f_base,
                                                   float* __restrict__ ws, int32_t* __restrict__ cnt) {
   constexpr int SUB = 32 / LPR;
-  constexpr int kUnroll = 4;
+  constexpr int kUnroll = NM_RES_UNROLL;
   const int lane = threadIdx.x & 31;
   const int sub = lane / LPR, li = lane % LPR;
   const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (sub * LPR));

@@ -65,6 +65,12 @@ constexpr int kPrefetchUnits = 2;                      // record L2-prefetch dis
 #define NM_REC_CPASYNC 0             // records by warp-wide cp.async instead of one bulk copy each
 #endif
 constexpr int kIssueLanes = 8;       // records whose bulk copies are issued together
+#ifndef NM_SMEM_BUDGET
+#define NM_SMEM_BUDGET (214 * 1024)  // stages + record rings (barriers and alignment on top)
+#endif
+#ifndef NM_MIN_RING
+#define NM_MIN_RING (32 * 1024)      // ring bytes reserved before the stage count is chosen
+#endif
 
 struct SpmmParams {
   const uint8_t* image;
@@ -222,12 +228,12 @@ struct Cfg {
   static constexpr int kABytes = kChunkValBytes;                // 128 x 16 values (4096)
   static constexpr int kBBytes = 32 * BN * 2;                   // 32 K-rows x BN halves
   static constexpr int kStageBytes = kABytes + kBBytes;
-  static constexpr int kStagesRaw = (214 * 1024 - 32 * 1024 - kRecMaxBytes) / kStageBytes;
+  static constexpr int kStagesRaw = (NM_SMEM_BUDGET - NM_MIN_RING - kRecMaxBytes) / kStageBytes;
   // a multiple of the loader-group count: group g owns stages s % kLoadGroups == g, so every
   // stage has one consumer group that visits it in chunk order (parity waits stay valid)
   static constexpr int kStages = ((kStagesRaw > 16 ? 16 : kStagesRaw) / kLoadGroups) * kLoadGroups;
   // the record ring takes what the stages leave (largest power of two, >= 32 KB)
-  static constexpr int kRingAvail = 214 * 1024 - kStages * kStageBytes - kProducers * kRecMaxBytes;
+  static constexpr int kRingAvail = NM_SMEM_BUDGET - kStages * kStageBytes - kProducers * kRecMaxBytes;
   static constexpr int kRingPer = kRingAvail / kProducers;
   static constexpr int kRecRing =  // each producer's ring: the largest power of two that fits
       kRingPer >= 64 * 1024 ? 64 * 1024 : kRingPer >= 32 * 1024 ? 32 * 1024 : 16 * 1024;
