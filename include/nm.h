@@ -101,6 +101,19 @@ typedef struct {
 NM_API nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
                      int32_t* perm_out, nm_reorder_stats* st);
 
+/* nm_reorder_gpu -- nm_reorder with Stage-1 (Alg. 2 lines 4-13: Hamming position codes of
+ * every (row, segment) of B, L339-346 / Listing 1, and the stable lexicographic row
+ * sort, L366-384) and the omega / MBscore counts (L203, L382) run on the current CUDA device
+ * (the paper's SOGRE is a GPU library, L484).  Stage-2 (Alg. 3) stays on
+ * the host: its greedy is sequential in the recorded pairs.  The permutation is bit-identical
+ * to nm_reorder's and to the CPU oracle's.
+ *   A, V, N, M, opts, perm_out, st : as nm_reorder (A host or device CSR; perm_out host).
+ *   stream : cudaStream_t the device work is ordered on (NULL = legacy default stream).
+ * Synchronous on return.  Device scratch: ~ 40 bytes per stored entry + 40 per vertex,
+ * allocated and freed inside the call.  Errors: as nm_reorder, plus CUDA / OOM. */
+NM_API nm_status nm_reorder_gpu(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
+                                int32_t* perm_out, nm_reorder_stats* st, void* stream);
+
 /* nm_select_pattern -- the paper's best-V:N:M search (§5): reorder for 1:2:M
  * with M = 4, 8, ... (<= max_M) while the reordered graph conforms (omega = MBscore = 0),
  * then for V:2:M with V = 2, 4, ... (<= max_V, "V going from 1 to 32 in a similar manner")

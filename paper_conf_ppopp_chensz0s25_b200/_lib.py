@@ -57,6 +57,9 @@ SIGNATURES = {
     "nm_reorder": (ctypes.c_int, [ctypes.POINTER(nm_csr), ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                   ctypes.POINTER(nm_reorder_opts), P32,
                                   ctypes.POINTER(nm_reorder_stats)]),
+    "nm_reorder_gpu": (ctypes.c_int, [ctypes.POINTER(nm_csr), ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                      ctypes.POINTER(nm_reorder_opts), P32,
+                                      ctypes.POINTER(nm_reorder_stats), ctypes.c_void_p]),
     "nm_select_pattern": (ctypes.c_int, [ctypes.POINTER(nm_csr), ctypes.c_int, ctypes.c_int,
                                          ctypes.POINTER(nm_reorder_opts), P32,
                                          ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.c_int),

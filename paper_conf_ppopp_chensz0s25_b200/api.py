@@ -49,14 +49,20 @@ def _stream_ptr(stream=None):
 
 
 def reorder(indptr, indices, V: int, N: int, M: int, max_outer=10, max_stage1=10, max_stage2=10,
-            gain_rule=0, keep_best=1):
-    """nm_reorder: returns (perm int32[n], stats dict)."""
+            gain_rule=0, keep_best=1, device=False, stream=None):
+    """nm_reorder (host) or, with device=True, nm_reorder_gpu (Stage-1 sort and the counts on
+    the current CUDA device): returns (perm int32[n], stats dict)."""
     c, keep = _csr_struct(indptr, indices)
     perm = np.zeros(c.n, np.int32)
     o = L.nm_reorder_opts(max_outer, max_stage1, max_stage2, gain_rule, keep_best)
     st = L.nm_reorder_stats()
-    L.check(L.load().nm_reorder(ctypes.byref(c), V, N, M, ctypes.byref(o),
-                                perm.ctypes.data_as(L.P32), ctypes.byref(st)), "nm_reorder")
+    if device:
+        L.check(L.load().nm_reorder_gpu(ctypes.byref(c), V, N, M, ctypes.byref(o),
+                                        perm.ctypes.data_as(L.P32), ctypes.byref(st),
+                                        _stream_ptr(stream)), "nm_reorder_gpu")
+    else:
+        L.check(L.load().nm_reorder(ctypes.byref(c), V, N, M, ctypes.byref(o),
+                                    perm.ctypes.data_as(L.P32), ctypes.byref(st)), "nm_reorder")
     return perm, {f: getattr(st, f) for f, _ in L.nm_reorder_stats._fields_}
 
 

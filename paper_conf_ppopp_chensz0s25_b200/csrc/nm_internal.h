@@ -145,5 +145,6 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
 nm_status count_violations_dev(const DevCsr& A, const int32_t* perm_dev, int V, int N, int M,
                                int64_t* omega, int64_t* mb, int32_t* pscore_host,
                                cudaStream_t s);
+nm_status stage1_sort_dev(const DevCsr& A, int32_t* perm_dev, int N, int M, cudaStream_t s);
 
 }  // namespace nm

@@ -336,9 +336,68 @@ using namespace nm;
 namespace nm {
 namespace {
 
+// The two steps of Alg. 1 that have a GPU version (Stage-1 sort and the counts); Stage-2
+// stays on the host (its greedy is sequential in the recorded pairs).
+struct Backend {
+  virtual ~Backend() {}
+  virtual nm_status stage1(std::vector<int32_t>& perm, std::vector<int32_t>& iperm, int N, int M) = 0;
+  virtual nm_status counts(const std::vector<int32_t>& perm, const std::vector<int32_t>& iperm, int V, int N,
+                           int M, int64_t* w, int64_t* mb) = 0;
+};
+
+struct HostBackend : Backend {
+  const Graph& g;
+  explicit HostBackend(const Graph& g_) : g(g_) {}
+  nm_status stage1(std::vector<int32_t>& perm, std::vector<int32_t>& iperm, int N, int M) override {
+    stage1_sort(g, perm, iperm, N, M);
+    return NM_OK;
+  }
+  nm_status counts(const std::vector<int32_t>& perm, const std::vector<int32_t>& iperm, int V, int N, int M,
+                   int64_t* w, int64_t* mb) override {
+    *w = omega_pscore(g, perm, iperm, N, M, nullptr);
+    *mb = mbscore(g, perm, iperm, V, M);
+    return NM_OK;
+  }
+};
+
+// Stage-1 sort (reorder_gpu.cu) and omega / MBscore (counts.cu) on the device
+struct DeviceBackend : Backend {
+  const DevCsr& d;
+  cudaStream_t s;
+  int32_t* dperm = nullptr;
+  DeviceBackend(const DevCsr& d_, cudaStream_t s_) : d(d_), s(s_) {}
+  ~DeviceBackend() override { if (dperm) cudaFree(dperm); }
+  nm_status upload(const std::vector<int32_t>& perm) {
+    if (!dperm) NM_CUDA(cudaMalloc(&dperm, sizeof(int32_t) * d.n));
+    NM_CUDA(cudaMemcpyAsync(dperm, perm.data(), sizeof(int32_t) * d.n, cudaMemcpyHostToDevice, s));
+    return NM_OK;
+  }
+  nm_status stage1(std::vector<int32_t>& perm, std::vector<int32_t>& iperm, int N, int M) override {
+    nm_status st = upload(perm);
+    if (st == NM_OK) st = stage1_sort_dev(d, dperm, N, M, s);
+    if (st != NM_OK) return st;
+    NM_CUDA(cudaMemcpyAsync(perm.data(), dperm, sizeof(int32_t) * d.n, cudaMemcpyDeviceToHost, s));
+    NM_CUDA(cudaStreamSynchronize(s));
+    invert(perm, iperm);
+    return NM_OK;
+  }
+  nm_status counts(const std::vector<int32_t>& perm, const std::vector<int32_t>&, int V, int N, int M,
+                   int64_t* w, int64_t* mb) override {
+    nm_status st = upload(perm);
+    if (st != NM_OK) return st;
+    return count_violations_dev(d, dperm, V, N, M, w, mb, nullptr, s);
+  }
+};
+
+#define NM_TRY(x)                   \
+  do {                              \
+    nm_status s_ = (x);             \
+    if (s_ != NM_OK) return s_;     \
+  } while (0)
+
 // Alg. 1 on a validated host graph: perm_out receives the (keep-best) order.
-void reorder_core(const Graph& g, int V, int N, int M, const nm_reorder_opts& o, int32_t* perm_out,
-                  nm_reorder_stats* st) {
+nm_status reorder_core(const Graph& g, Backend& be, int V, int N, int M, const nm_reorder_opts& o,
+                       int32_t* perm_out, nm_reorder_stats* st) {
   auto t0 = std::chrono::steady_clock::now();
   const int64_t n = g.n;
   std::vector<int32_t> perm(n), iperm(n), best;
@@ -346,24 +405,23 @@ void reorder_core(const Graph& g, int V, int N, int M, const nm_reorder_opts& o,
   iperm = perm;
   nm_reorder_stats stats;
   memset(&stats, 0, sizeof(stats));
-  int64_t w = omega_pscore(g, perm, iperm, N, M, nullptr);
-  int64_t mb = mbscore(g, perm, iperm, V, M);
+  int64_t w = 0, mb = 0;
+  NM_TRY(be.counts(perm, iperm, V, N, M, &w, &mb));
   stats.omega_init = w;
   stats.mb_init = mb;
   int64_t best_score = w + mb;
   best = perm;
   int64_t it = 0;
   while ((w > 0 || mb > 0) && it <= o.max_outer) {
-    int64_t mb1 = mb;
+    int64_t mb1 = mb, w1 = 0;
     for (int i1 = 0; mb1 > 0 && i1 <= o.max_stage1; ++i1) {  // Alg. 2
-      stage1_sort(g, perm, iperm, N, M);
+      NM_TRY(be.stage1(perm, iperm, N, M));
       stats.stage1_iters++;
-      mb1 = mbscore(g, perm, iperm, V, M);
+      NM_TRY(be.counts(perm, iperm, V, N, M, &w1, &mb1));
     }
     stats.stage2_passes += stage2(g, perm, iperm, N, M, o.max_stage2, o.gain_rule, &stats.max_pairs_per_primary);
     ++it;
-    w = omega_pscore(g, perm, iperm, N, M, nullptr);
-    mb = mbscore(g, perm, iperm, V, M);
+    NM_TRY(be.counts(perm, iperm, V, N, M, &w, &mb));
     if (o.keep_best && w + mb < best_score) {
       best_score = w + mb;
       best = perm;
@@ -373,10 +431,10 @@ void reorder_core(const Graph& g, int V, int N, int M, const nm_reorder_opts& o,
   const std::vector<int32_t>& res = o.keep_best ? best : perm;
   memcpy(perm_out, res.data(), sizeof(int32_t) * n);
   invert(res, iperm);
-  stats.omega_final = omega_pscore(g, res, iperm, N, M, nullptr);
-  stats.mb_final = mbscore(g, res, iperm, V, M);
+  NM_TRY(be.counts(res, iperm, V, N, M, &stats.omega_final, &stats.mb_final));
   stats.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
   if (st) *st = stats;
+  return NM_OK;
 }
 
 struct HostGraph {
@@ -417,8 +475,30 @@ extern "C" nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_r
   HostGraph hg;
   s = hg.load(A);
   if (s != NM_OK) return s;
-  reorder_core(hg.g, V, N, M, o, perm_out, st);
-  return NM_OK;
+  HostBackend be(hg.g);
+  return reorder_core(hg.g, be, V, N, M, o, perm_out, st);
+}
+
+extern "C" nm_status nm_reorder_gpu(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
+                                    int32_t* perm_out, nm_reorder_stats* st, void* stream) {
+  if (!A || !perm_out) return fail(NM_ERR_INVALID_ARG, "nm_reorder_gpu: NULL argument");
+  if (V < 1 || N < 1 || M <= N) return fail(NM_ERR_INVALID_ARG, "nm_reorder_gpu: need V >= 1, 1 <= N < M");
+  if (M > 32) return fail(NM_ERR_UNSUPPORTED, "nm_reorder_gpu: M > 32");
+  nm_status s = check_graph_arg(A);
+  if (s != NM_OK) return s;
+  nm_reorder_opts o = {10, 10, 10, 0, 1};
+  if (opts) o = *opts;
+  HostGraph hg;  // Stage-2 walks the host copy
+  s = hg.load(A);
+  if (s != NM_OK) return s;
+  cudaStream_t cs = (cudaStream_t)stream;
+  DevCsr d;
+  nm_csr pattern = *A;
+  pattern.val = nullptr;  // the reorder needs the pattern only
+  s = upload_csr(&pattern, NM_F16, &d, cs);
+  if (s != NM_OK) return s;
+  DeviceBackend be(d, cs);
+  return reorder_core(hg.g, be, V, N, M, o, perm_out, st);
 }
 
 extern "C" nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, const nm_reorder_opts* opts,
@@ -438,11 +518,12 @@ extern "C" nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, co
   // 1:2:M with M = 4, 8, ... while the graph can be reordered to conform ...
   int bestV = 1, bestM = 4;
   nm_reorder_stats first;
-  reorder_core(hg.g, 1, 2, 4, o, perm_out, &first);
+  HostBackend be(hg.g);
+  NM_TRY(reorder_core(hg.g, be, 1, 2, 4, o, perm_out, &first));
   if (st) *st = first;
   if (first.omega_final == 0 && first.mb_final == 0) {
     for (int M = 8; M <= max_M; M *= 2) {
-      reorder_core(hg.g, 1, 2, M, o, cand.data(), &cst);
+      NM_TRY(reorder_core(hg.g, be, 1, 2, M, o, cand.data(), &cst));
       if (cst.omega_final != 0 || cst.mb_final != 0) break;
       bestM = M;
       memcpy(perm_out, cand.data(), sizeof(int32_t) * n);
@@ -450,7 +531,7 @@ extern "C" nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, co
     }
     // ... then V:2:M with V = 2, 4, ..., max_V "in a similar manner" (doubling)
     for (int V = 2; V <= max_V; V *= 2) {
-      reorder_core(hg.g, V, 2, bestM, o, cand.data(), &cst);
+      NM_TRY(reorder_core(hg.g, be, V, 2, bestM, o, cand.data(), &cst));
       if (cst.omega_final != 0 || cst.mb_final != 0) break;
       bestV = V;
       memcpy(perm_out, cand.data(), sizeof(int32_t) * n);
