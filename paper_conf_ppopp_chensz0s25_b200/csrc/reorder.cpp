@@ -6,6 +6,8 @@
 #include <algorithm>
 #include <chrono>
 #include <cstdint>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <numeric>
 #include <vector>
@@ -210,34 +212,50 @@ inline void gains(const Graph& g, const std::vector<int32_t>& perm, const SegCou
   *gt = st;
 }
 
-Pair freshtop(const Graph& g, const std::vector<int32_t>& perm, const SegCount& cp, const SegCount& ct, int N,
-              int M, int64_t p, int64_t t, const std::vector<uint8_t>& used, bool need_positive) {
-  Pair best;
-  for (int64_t u = p * M; u < std::min<int64_t>(g.n, p * M + M); ++u) {
-    if (used[u]) continue;
+bool all_used(const std::vector<uint8_t>& used, int64_t seg, int M, int64_t n) {
+  for (int64_t q = seg * M; q < std::min<int64_t>(n, seg * M + M); ++q)
+    if (!used[q]) return false;
+  return true;
+}
+
+// Gain table of a (primary p, target t) pair: (gp, gt) of every position pair (u, v) of the
+// two segments w.r.t. the pass-start order (the M x M table of).  The gains do not
+// depend on which positions are already used, so a table can be computed ahead of the
+// sequential pick (and in parallel with other targets' tables) without changing the result.
+void gain_table(const Graph& g, const std::vector<int32_t>& perm, const SegCount& cp, const SegCount& ct, int N,
+                int M, int64_t p, int64_t t, const std::vector<uint8_t>& used, int64_t* tab /* [M*M*2] */) {
+  // positions already used are never picked again (used only grows): their entries are skipped
+  for (int64_t u = p * M; u < std::min<int64_t>(g.n, p * M + M); ++u)
     for (int64_t v = t * M; v < std::min<int64_t>(g.n, t * M + M); ++v) {
+      if (used[u] || used[v]) continue;
+      int64_t* e = tab + 2 * ((u - p * M) * M + (v - t * M));
+      gains(g, perm, cp, ct, N, u, v, &e[0], &e[1]);
+    }
+}
+
+// freshtop (Alg. 3): the best fresh (u, v) pair over a precomputed table; scan u-major in
+// position order, strict ">" so ties keep the smallest (u, v) (reading #18)
+Pair pick_from_table(const int64_t* tab, int64_t n, int M, int64_t p, int64_t t, const std::vector<uint8_t>& used,
+                     bool need_positive) {
+  Pair best;
+  for (int64_t u = p * M; u < std::min<int64_t>(n, p * M + M); ++u) {
+    if (used[u]) continue;
+    for (int64_t v = t * M; v < std::min<int64_t>(n, t * M + M); ++v) {
       if (used[v]) continue;
-      int64_t gp, gt;
-      gains(g, perm, cp, ct, N, u, v, &gp, &gt);
-      const int64_t gg = gp + gt;
+      const int64_t* e = tab + 2 * ((u - p * M) * M + (v - t * M));
+      const int64_t gg = e[0] + e[1];
       if (need_positive && gg <= 0) continue;
-      if (!best.found || gg > best.g) {  // ties keep the smallest (u, v) (reading #18)
+      if (!best.found || gg > best.g) {
         best.found = true;
         best.g = gg;
-        best.gp = gp;
-        best.gt = gt;
+        best.gp = e[0];
+        best.gt = e[1];
         best.u = u;
         best.v = v;
       }
     }
   }
   return best;
-}
-
-bool all_used(const std::vector<uint8_t>& used, int64_t seg, int M, int64_t n) {
-  for (int64_t q = seg * M; q < std::min<int64_t>(n, seg * M + M); ++q)
-    if (!used[q]) return false;
-  return true;
 }
 
 int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>& iperm, int N, int M,
@@ -250,7 +268,14 @@ int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>&
   SegCount cp, ct;
   cp.init(n);
   ct.init(n);
-  std::vector<int64_t> su, sv;
+  std::vector<int64_t> su, sv, tb, tabs;
+#ifdef _OPENMP
+  const int nthr = std::max(1, std::min(omp_get_max_threads(), 16));
+#else
+  const int nthr = 1;
+#endif
+  std::vector<SegCount> cts(nthr);  // per-thread target counters for the parallel tables
+  for (SegCount& c : cts) c.init(n);
   for (int it = 0; it <= maxiter; ++it) {
     omega_pscore(g, perm, iperm, N, M, &pscore);
     std::vector<int64_t> I;
@@ -275,9 +300,11 @@ int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>&
       }
       cp.build(g, perm, p, M);
       ct.build(g, perm, t, M);
+      std::vector<int64_t> tab(2 * (size_t)M * M);
+      gain_table(g, perm, cp, ct, N, M, p, t, used, tab.data());
       int64_t npairs = 0;
       for (;;) {
-        Pair pr = freshtop(g, perm, cp, ct, N, M, p, t, used, true);  // "beneficial" swaps
+        Pair pr = pick_from_table(tab.data(), n, M, p, t, used, true);  // "beneficial" swaps
         if (!pr.found) break;
         su.push_back(pr.u);
         sv.push_back(pr.v);
@@ -301,19 +328,41 @@ int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>&
           if (inI[I[k]]) snap.push_back(I[k]);
         cp.build(g, perm, p, M);
         int64_t npairs = 0;
-        for (int64_t t : snap) {
-          if (!inI[t]) continue;
-          ct.build(g, perm, t, M);
-          Pair pr = freshtop(g, perm, cp, ct, N, M, p, t, used, gain_rule == 1);
-          if (!pr.found) continue;
-          su.push_back(pr.u);
-          sv.push_back(pr.v);
-          ++npairs;
-          used[pr.u] = used[pr.v] = 1;
-          est[p] -= pr.gp;
-          est[t] -= pr.gt;
-          if (est[t] <= 0) { inI[t] = 0; --live; }
-          if (est[p] <= 0 || all_used(used, p, M, n)) break;
+        // targets in batches: their gain tables in parallel, the picks in target order.  Only
+        // the target being picked can leave I, so the batch's membership filter is final.
+        size_t k = 0, batch = 4;
+        bool stop = false;
+        while (!stop && k < snap.size()) {
+          tb.clear();
+          for (; k < snap.size() && tb.size() < batch; ++k)
+            if (inI[snap[k]]) tb.push_back(snap[k]);
+          batch = std::min<size_t>(batch * 2, 256);
+          if (tabs.size() < tb.size() * 2 * M * M) tabs.resize(tb.size() * 2 * M * M);
+          const int64_t nb = (int64_t)tb.size();
+#pragma omp parallel for schedule(dynamic, 1) num_threads(nthr) if (nb > 1)
+          for (int64_t b = 0; b < nb; ++b) {
+#ifdef _OPENMP
+            SegCount& c = cts[omp_get_thread_num()];
+#else
+            SegCount& c = cts[0];
+#endif
+            c.build(g, perm, tb[b], M);
+            gain_table(g, perm, cp, c, N, M, p, tb[b], used, tabs.data() + (size_t)b * 2 * M * M);
+            c.clear();
+          }
+          for (int64_t b = 0; b < nb; ++b) {
+            const int64_t t = tb[b];
+            Pair pr = pick_from_table(tabs.data() + (size_t)b * 2 * M * M, n, M, p, t, used, gain_rule == 1);
+            if (!pr.found) continue;
+            su.push_back(pr.u);
+            sv.push_back(pr.v);
+            ++npairs;
+            used[pr.u] = used[pr.v] = 1;
+            est[p] -= pr.gp;
+            est[t] -= pr.gt;
+            if (est[t] <= 0) { inI[t] = 0; --live; }
+            if (est[p] <= 0 || all_used(used, p, M, n)) { stop = true; break; }
+          }
         }
         *max_pairs = std::max(*max_pairs, npairs);
       }
@@ -412,14 +461,23 @@ nm_status reorder_core(const Graph& g, Backend& be, int V, int N, int M, const n
   int64_t best_score = w + mb;
   best = perm;
   int64_t it = 0;
+  double t_s1 = 0, t_s2 = 0;  // NM_REORDER_TRACE=1: per-stage wall time on stderr
+  auto now = [] { return std::chrono::steady_clock::now(); };
+  auto secs = [](std::chrono::steady_clock::time_point a, std::chrono::steady_clock::time_point b) {
+    return std::chrono::duration<double>(b - a).count();
+  };
   while ((w > 0 || mb > 0) && it <= o.max_outer) {
     int64_t mb1 = mb, w1 = 0;
+    auto ta = now();
     for (int i1 = 0; mb1 > 0 && i1 <= o.max_stage1; ++i1) {  // Alg. 2
       NM_TRY(be.stage1(perm, iperm, N, M));
       stats.stage1_iters++;
       NM_TRY(be.counts(perm, iperm, V, N, M, &w1, &mb1));
     }
+    auto tb = now();
     stats.stage2_passes += stage2(g, perm, iperm, N, M, o.max_stage2, o.gain_rule, &stats.max_pairs_per_primary);
+    t_s1 += secs(ta, tb);
+    t_s2 += secs(tb, now());
     ++it;
     NM_TRY(be.counts(perm, iperm, V, N, M, &w, &mb));
     if (o.keep_best && w + mb < best_score) {
@@ -433,6 +491,10 @@ nm_status reorder_core(const Graph& g, Backend& be, int V, int N, int M, const n
   invert(res, iperm);
   NM_TRY(be.counts(res, iperm, V, N, M, &stats.omega_final, &stats.mb_final));
   stats.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+  if (const char* tr = getenv("NM_REORDER_TRACE"))
+    if (tr[0] == '1')
+      fprintf(stderr, "nm_reorder trace: stage1(+MB counts) %.3f s, stage2 %.3f s, total %.3f s\n", t_s1, t_s2,
+              stats.seconds);
   if (st) *st = stats;
   return NM_OK;
 }
