@@ -63,10 +63,13 @@ __global__ void k_groups(const uint64_t* __restrict__ key, int64_t m, int M, int
 
 template <typename T>
 struct Buf {
+  // stream-ordered pool allocations: the reorder calls these once per Stage-1 iteration
   T* p = nullptr;
-  ~Buf() { if (p) cudaFree(p); }
-  nm_status alloc(size_t n) {
-    NM_CUDA(cudaMalloc(&p, sizeof(T) * (n > 0 ? n : 1)));
+  cudaStream_t st = 0;
+  ~Buf() { if (p) cudaFreeAsync(p, st); }
+  nm_status alloc(size_t n, cudaStream_t s) {
+    st = s;
+    NM_CUDA(cudaMallocAsync(&p, sizeof(T) * (n > 0 ? n : 1), s));
     return NM_OK;
   }
 };
@@ -87,9 +90,9 @@ nm_status count_violations_dev(const DevCsr& A, const int32_t* perm_dev, int V, 
   Buf<int32_t> pscore;
   Buf<unsigned long long> tot;
   nm_status st;
-  if ((st = iperm.alloc(n)) || (st = pid.alloc(n)) || (st = deg.alloc(n + 1)) || (st = Brp.alloc(n + 1)) ||
-      (st = k1.alloc(nnz)) || (st = k2.alloc(nnz)) || (st = k3.alloc(nnz)) || (st = k4.alloc(nnz)) ||
-      (st = pscore.alloc(S)) || (st = tot.alloc(2)))
+  if ((st = iperm.alloc(n, s)) || (st = pid.alloc(n, s)) || (st = deg.alloc(n + 1, s)) || (st = Brp.alloc(n + 1, s)) ||
+      (st = k1.alloc(nnz, s)) || (st = k2.alloc(nnz, s)) || (st = k3.alloc(nnz, s)) || (st = k4.alloc(nnz, s)) ||
+      (st = pscore.alloc(S, s)) || (st = tot.alloc(2, s)))
     return st;
   const int32_t* perm = perm_dev;
   if (!perm) {
@@ -103,7 +106,7 @@ nm_status count_violations_dev(const DevCsr& A, const int32_t* perm_dev, int V, 
     size_t bytes = 0;
     NM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, bytes, deg.p, Brp.p, n + 1, s));
     Buf<uint8_t> tmp;
-    if ((st = tmp.alloc(bytes))) return st;
+    if ((st = tmp.alloc(bytes, s))) return st;
     NM_CUDA(cub::DeviceScan::ExclusiveSum(tmp.p, bytes, deg.p, Brp.p, n + 1, s));
   }
   k_keys<<<g256(n * 32), 256, 0, s>>>(A.rp, A.ci, perm, iperm.p, n, Brp.p, V, k1.p, k2.p);
@@ -112,18 +115,18 @@ nm_status count_violations_dev(const DevCsr& A, const int32_t* perm_dev, int V, 
     NM_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, bytes, k1.p, k3.p, nnz, 0, 64, s));
     NM_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, b2, k2.p, k4.p, nnz, 0, 64, s));
     Buf<uint8_t> tmp;
-    if ((st = tmp.alloc(bytes > b2 ? bytes : b2))) return st;
+    if ((st = tmp.alloc(bytes > b2 ? bytes : b2, s))) return st;
     NM_CUDA(cub::DeviceRadixSort::SortKeys(tmp.p, bytes, k1.p, k3.p, nnz, 0, 64, s));
     NM_CUDA(cub::DeviceRadixSort::SortKeys(tmp.p, b2, k2.p, k4.p, nnz, 0, 64, s));
   }
   // distinct (panel, column) keys for the vertical constraint
   Buf<int64_t> nsel;
-  if ((st = nsel.alloc(1))) return st;
+  if ((st = nsel.alloc(1, s))) return st;
   {
     size_t bytes = 0;
     NM_CUDA(cub::DeviceSelect::Unique(nullptr, bytes, k4.p, k2.p, nsel.p, nnz, s));
     Buf<uint8_t> tmp;
-    if ((st = tmp.alloc(bytes))) return st;
+    if ((st = tmp.alloc(bytes, s))) return st;
     NM_CUDA(cub::DeviceSelect::Unique(tmp.p, bytes, k4.p, k2.p, nsel.p, nnz, s));
   }
   int64_t nuniq = 0;

@@ -114,10 +114,13 @@ struct RowKeyLess {
 
 template <typename T>
 struct DBuf {
+  // stream-ordered pool allocations: the reorder calls these once per Stage-1 iteration
   T* p = nullptr;
-  ~DBuf() { if (p) cudaFree(p); }
-  nm_status alloc(size_t n) {
-    NM_CUDA(cudaMalloc(&p, sizeof(T) * (n > 0 ? n : 1)));
+  cudaStream_t st = 0;
+  ~DBuf() { if (p) cudaFreeAsync(p, st); }
+  nm_status alloc(size_t n, cudaStream_t s) {
+    st = s;
+    NM_CUDA(cudaMallocAsync(&p, sizeof(T) * (n > 0 ? n : 1), s));
     return NM_OK;
   }
 };
@@ -127,7 +130,7 @@ nm_status with_temp(F&& f, cudaStream_t s) {
   size_t bytes = 0;
   NM_CUDA(f((void*)nullptr, bytes));
   DBuf<uint8_t> tmp;
-  nm_status st = tmp.alloc(bytes);
+  nm_status st = tmp.alloc(bytes, s);
   if (st != NM_OK) return st;
   NM_CUDA(f((void*)tmp.p, bytes));
   (void)s;
@@ -144,9 +147,9 @@ nm_status stage1_sort_dev(const DevCsr& A, int32_t* perm_dev, int N, int M, cuda
   DBuf<int64_t> deg, Brp, gid, goff, gx, gc;
   DBuf<uint64_t> k1, k2;
   nm_status st;
-  if ((st = iperm.alloc(n)) || (st = order.alloc(n)) || (st = nperm.alloc(n)) || (st = ngr.alloc(n + 1)) ||
-      (st = deg.alloc(n + 1)) || (st = Brp.alloc(n + 1)) || (st = goff.alloc(n + 1)) || (st = k1.alloc(nnz)) ||
-      (st = k2.alloc(nnz)) || (st = flag.alloc(nnz)) || (st = gid.alloc(nnz)))
+  if ((st = iperm.alloc(n, s)) || (st = order.alloc(n, s)) || (st = nperm.alloc(n, s)) || (st = ngr.alloc(n + 1, s)) ||
+      (st = deg.alloc(n + 1, s)) || (st = Brp.alloc(n + 1, s)) || (st = goff.alloc(n + 1, s)) || (st = k1.alloc(nnz, s)) ||
+      (st = k2.alloc(nnz, s)) || (st = flag.alloc(nnz, s)) || (st = gid.alloc(nnz, s)))
     return st;
   k_s1_inv<<<grid_for(n, B), B, 0, s>>>(perm_dev, iperm.p, n);
   NM_CUDA(cudaMemsetAsync(deg.p, 0, sizeof(int64_t) * (n + 1), s));
@@ -156,9 +159,11 @@ nm_status stage1_sort_dev(const DevCsr& A, int32_t* perm_dev, int N, int M, cuda
   if ((st = with_temp([&](void* t, size_t& b) { return cub::DeviceScan::ExclusiveSum(t, b, dp, bp, n + 1, s); }, s)))
     return st;
   k_s1_keys<<<grid_for(n * 32, B), B, 0, s>>>(A.rp, A.ci, perm_dev, iperm.p, n, Brp.p, k1.p);
+  int hb = 32;  // key bits: 32 column bits + enough row bits for n
+  while (hb < 64 && ((int64_t)1 << (hb - 32)) < n) ++hb;
   uint64_t* a1 = k1.p;
   uint64_t* a2 = k2.p;
-  if ((st = with_temp([&](void* t, size_t& b) { return cub::DeviceRadixSort::SortKeys(t, b, a1, a2, nnz, 0, 64, s); }, s)))
+  if ((st = with_temp([&](void* t, size_t& b) { return cub::DeviceRadixSort::SortKeys(t, b, a1, a2, nnz, 0, hb, s); }, s)))
     return st;
   // group ids = exclusive scan of the group-start flags
   int64_t ngroups = 0;
@@ -175,7 +180,7 @@ nm_status stage1_sort_dev(const DevCsr& A, int32_t* perm_dev, int N, int M, cuda
     NM_CUDA(cudaStreamSynchronize(s));
     ngroups = last + lastf;
   }
-  if ((st = gx.alloc(ngroups)) || (st = gc.alloc(ngroups))) return st;
+  if ((st = gx.alloc(ngroups, s)) || (st = gc.alloc(ngroups, s))) return st;
   NM_CUDA(cudaMemsetAsync(ngr.p, 0, sizeof(int32_t) * (n + 1), s));
   if (nnz > 0)
     k_s1_codes<<<grid_for(nnz, B), B, 0, s>>>(k2.p, nnz, (uint32_t)M, N, S, gid.p, gx.p, gc.p, ngr.p);
