@@ -317,25 +317,23 @@ int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>&
     } else {
       size_t head = 0;
       int64_t live = (int64_t)I.size();
-      std::vector<int64_t> snap;
       while (live > 1) {
         while (!inI[I[head]]) ++head;
         const int64_t p = I[head++];
         inI[p] = 0;
         --live;
-        snap.clear();
-        for (size_t k = head; k < I.size(); ++k)
-          if (inI[I[k]]) snap.push_back(I[k]);
+        // the targets are the live entries of I after the primary, walked lazily: only the
+        // target being picked can leave I, so this equals a snapshot taken when p is popped
         cp.build(g, perm, p, M);
         int64_t npairs = 0;
         // targets in batches: their gain tables in parallel, the picks in target order.  Only
         // the target being picked can leave I, so the batch's membership filter is final.
-        size_t k = 0, batch = 4;
+        size_t k = head, batch = 4;
         bool stop = false;
-        while (!stop && k < snap.size()) {
+        while (!stop && k < I.size()) {
           tb.clear();
-          for (; k < snap.size() && tb.size() < batch; ++k)
-            if (inI[snap[k]]) tb.push_back(snap[k]);
+          for (; k < I.size() && tb.size() < batch; ++k)
+            if (inI[I[k]]) tb.push_back(I[k]);
           batch = std::min<size_t>(batch * 2, 256);
           if (tabs.size() < tb.size() * 2 * M * M) tabs.resize(tb.size() * 2 * M * M);
           const int64_t nb = (int64_t)tb.size();
