@@ -6,6 +6,7 @@
 #include <algorithm>
 #include <chrono>
 #include <cstdint>
+#include <climits>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -169,7 +170,13 @@ struct SegCount {
   // dense per-vertex counters with a touched list: cnt[w] = #vertices of the segment adjacent to w
   std::vector<int32_t> cnt;
   std::vector<int32_t> touched;
-  void init(int64_t n) { cnt.assign(n, 0); }
+  std::vector<int32_t> mark;  // gain_table's N(x) marker (stamped, per counter owner)
+  int32_t stamp = 0;
+  void init(int64_t n) {
+    cnt.assign(n, 0);
+    mark.assign(n, 0);
+    stamp = 0;
+  }
   void build(const Graph& g, const std::vector<int32_t>& perm, int64_t seg, int M) {
     clear();
     for (int64_t q = seg * M; q < std::min<int64_t>(g.n, seg * M + M); ++q) {
@@ -222,15 +229,50 @@ bool all_used(const std::vector<uint8_t>& used, int64_t seg, int M, int64_t n) {
 // two segments w.r.t. the pass-start order (the M x M table of).  The gains do not
 // depend on which positions are already used, so a table can be computed ahead of the
 // sequential pick (and in parallel with other targets' tables) without changing the result.
-void gain_table(const Graph& g, const std::vector<int32_t>& perm, const SegCount& cp, const SegCount& ct, int N,
+void gain_table(const Graph& g, const std::vector<int32_t>& perm, const SegCount& cp, SegCount& ct, int N,
                 int M, int64_t p, int64_t t, const std::vector<uint8_t>& used, int64_t* tab /* [M*M*2] */) {
-  // positions already used are never picked again (used only grows): their entries are skipped
-  for (int64_t u = p * M; u < std::min<int64_t>(g.n, p * M + M); ++u)
-    for (int64_t v = t * M; v < std::min<int64_t>(g.n, t * M + M); ++v) {
-      if (used[u] || used[v]) continue;
-      int64_t* e = tab + 2 * ((u - p * M) * M + (v - t * M));
-      gains(g, perm, cp, ct, N, u, v, &e[0], &e[1]);
+  // Same sums as gains(): a column w adjacent to x only contributes the d = -1 terms, one
+  // adjacent to y only the d = +1 terms, a common one nothing.  Per u the x-only sums over
+  // N(x) are formed once with N(x) marked; per v a walk of N(y) moves the common columns out
+  // of them and adds the y-only ones (one pass over N(y) instead of a merge per pair).
+  // Positions already used are never picked again (used only grows): their entries are skipped.
+  const int64_t ue = std::min<int64_t>(g.n, p * M + M), ve = std::min<int64_t>(g.n, t * M + M);
+  for (int64_t u = p * M; u < ue; ++u) {
+    if (used[u]) continue;
+    const int32_t x = perm[u];
+    if (++ct.stamp == INT32_MAX) {
+      std::fill(ct.mark.begin(), ct.mark.end(), 0);
+      ct.stamp = 1;
     }
+    const int32_t sx = ct.stamp;
+    int64_t Sp = 0, St = 0;
+    for (int64_t k = g.rp[x]; k < g.rp[x + 1]; ++k) {
+      const int32_t w = g.ci[k];
+      ct.mark[w] = sx;
+      const int c1 = cp.cnt[w], c2 = ct.cnt[w];
+      Sp += (c1 > N) - (c1 - 1 > N);
+      St += (c2 > N) - (c2 + 1 > N);
+    }
+    for (int64_t v = t * M; v < ve; ++v) {
+      if (used[v]) continue;
+      const int32_t y = perm[v];
+      int64_t sp = Sp, st = St;
+      for (int64_t k = g.rp[y]; k < g.rp[y + 1]; ++k) {
+        const int32_t w = g.ci[k];
+        const int c1 = cp.cnt[w], c2 = ct.cnt[w];
+        if (ct.mark[w] == sx) {
+          sp -= (c1 > N) - (c1 - 1 > N);
+          st -= (c2 > N) - (c2 + 1 > N);
+        } else {
+          sp += (c1 > N) - (c1 + 1 > N);
+          st += (c2 > N) - (c2 - 1 > N);
+        }
+      }
+      int64_t* e = tab + 2 * ((u - p * M) * M + (v - t * M));
+      e[0] = sp;
+      e[1] = st;
+    }
+  }
 }
 
 // freshtop (Alg. 3): the best fresh (u, v) pair over a precomputed table; scan u-major in
