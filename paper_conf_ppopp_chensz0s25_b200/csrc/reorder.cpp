@@ -599,8 +599,23 @@ extern "C" nm_status nm_reorder_gpu(const nm_csr* A, int V, int N, int M, const 
   pattern.val = nullptr;  // the reorder needs the pattern only
   s = upload_csr(&pattern, NM_F16, &d, cs);
   if (s != NM_OK) return s;
-  DeviceBackend be(d, cs);
-  return reorder_core(hg.g, be, V, N, M, o, perm_out, st);
+  // the per-iteration scratch of Stage-1 and the counts comes from the device's default
+  // stream-ordered pool: keep it reserved between iterations, give it back at the end
+  int dev = 0;
+  cudaMemPool_t pool;
+  NM_CUDA(cudaGetDevice(&dev));
+  NM_CUDA(cudaDeviceGetDefaultMemPool(&pool, dev));
+  uint64_t keep = UINT64_MAX, thr0 = 0;
+  NM_CUDA(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr0));
+  NM_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep));
+  {
+    DeviceBackend be(d, cs);
+    s = reorder_core(hg.g, be, V, N, M, o, perm_out, st);
+  }
+  cudaStreamSynchronize(cs);
+  cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr0);
+  cudaMemPoolTrimTo(pool, 0);
+  return s;
 }
 
 extern "C" nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, const nm_reorder_opts* opts,
