@@ -109,8 +109,8 @@ NM_API nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reord
  * to nm_reorder's and to the CPU oracle's.
  *   A, V, N, M, opts, perm_out, st : as nm_reorder (A host or device CSR; perm_out host).
  *   stream : cudaStream_t the device work is ordered on (NULL = legacy default stream).
- * Synchronous on return.  Device scratch: ~ 40 bytes per stored entry + 40 per vertex,
- * allocated and freed inside the call.  Errors: as nm_reorder, plus CUDA / OOM. */
+ * Synchronous on return.  Device memory: ~ 60 bytes per stored entry + 60 per vertex,
+ * from the default stream-ordered pool, trimmed on return.  Errors: as nm_reorder, plus CUDA / OOM. */
 NM_API nm_status nm_reorder_gpu(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
                                 int32_t* perm_out, nm_reorder_stats* st, void* stream);
 

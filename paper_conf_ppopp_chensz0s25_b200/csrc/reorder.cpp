@@ -370,7 +370,7 @@ int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>&
         int64_t npairs = 0;
         // targets in batches: their gain tables in parallel, the picks in target order.  Only
         // the target being picked can leave I, so the batch's membership filter is final.
-        size_t k = head, batch = 4;
+        size_t k = head, batch = (size_t)std::max(4, M);  // about the targets a primary needs (<= M pairs)
         bool stop = false;
         while (!stop && k < I.size()) {
           tb.clear();
