@@ -226,7 +226,7 @@ bool all_used(const std::vector<uint8_t>& used, int64_t seg, int M, int64_t n) {
 }
 
 // Gain table of a (primary p, target t) pair: (gp, gt) of every position pair (u, v) of the
-// two segments w.r.t. the pass-start order (the M x M table of).  The gains do not
+// two segments w.r.t. the pass-start order (swap_cands = GetCandidates(prim, targ), Alg. 3 lines 11-14, L459-462).  The gains do not
 // depend on which positions are already used, so a table can be computed ahead of the
 // sequential pick (and in parallel with other targets' tables) without changing the result.
 void gain_table(const Graph& g, const std::vector<int32_t>& perm, const SegCount& cp, SegCount& ct, int N,
