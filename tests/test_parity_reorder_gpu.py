@@ -74,3 +74,10 @@ def test_errors():
         api.reorder(ip, ic, 1, 2, 64, device=True)   # M > 32
     with pytest.raises(Exception):
         api.reorder(ip, ic, 0, 2, 4, device=True)    # V < 1
+
+
+def test_larger_banded_many_panels():
+    # 512 panels of 64 rows, 22 Stage-1 sorts over 0.5M stored entries
+    ip, ic = graphs.banded_graph(32768, 16, 23)
+    st = _check(ip, ic, 64, 2, 8, max_outer=1)
+    assert st["stage1_iters"] > 0 and st["mb_final"] < st["mb_init"]
