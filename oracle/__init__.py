@@ -87,6 +87,9 @@ def _lib():
         L.or_spmm_rows_f64.restype = ctypes.c_int
         L.or_spmm_rows_f64.argtypes = [ctypes.c_int64, P64, P64, P32, PF64, PF64,
                                        ctypes.c_int64, ctypes.c_int, PF64, PF64]
+        L.or_stage2_trace.restype = ctypes.c_int64
+        L.or_stage2_trace.argtypes = [ctypes.c_int64, P64, P32, P32, ctypes.c_int, ctypes.c_int,
+                                      ctypes.c_int, P64]
         L.or_stage1_once.restype = ctypes.c_int
         L.or_stage1_once.argtypes = [ctypes.c_int64, P64, P32, P32, ctypes.c_int, ctypes.c_int,
                                      P32]
@@ -184,6 +187,20 @@ def stage1_once(indptr, indices, perm, N: int, M: int):
     out = np.zeros(max(n, 1), np.int32)
     _lib().or_stage1_once(n, _p(rp, P64), _p(ci, P32), _p(pm, P32), N, M, _p(out, P32))
     return out[:n]
+
+
+def stage2_trace(indptr, indices, perm, N: int, M: int, gain_rule: int = 0):
+    """ONE Stage-2 pass (Alg. 3 lines 1-23) from perm: the recorded pairs in recording order
+    as a list of (primary segment, target segment, u, v) -- u, v positions of the pass-start
+    order -- or None when the pass stops before recording anything."""
+    rp, ci, n = _csr(indptr, indices)
+    pm = np.ascontiguousarray(perm, dtype=np.int32)
+    out = np.zeros(4 * max(n, 1), np.int64)
+    k = int(_lib().or_stage2_trace(n, _p(rp, P64), _p(ci, P32), _p(pm, P32), N, M, gain_rule,
+                                   _p(out, P64)))
+    if k < 0:
+        return None
+    return [tuple(int(x) for x in out[4 * i:4 * i + 4]) for i in range(k)]
 
 
 def pack(indptr, indices, val16, one_bits: int, perm, Vp: int, Mp: int, tau: int = 0):

@@ -331,96 +331,146 @@ static int all_positions_used(const uint8_t* used, int64_t seg, int M, int64_t n
   return 1;
 }
 
+/* Scratch of one Stage-2 pass, sized for n vertices / S segments. */
+typedef struct {
+  int32_t* pscore; int64_t* est; uint8_t* inI; uint8_t* used; or_item* I; int64_t* snap;
+} s2_scratch;
+
+/* One Stage-2 pass (Alg. 3 lines 1-23) over the pass-start matrix B: records the swap
+ * pairs (u, v) -- and the (primary, target) segments they were chosen for -- in the order
+ * Alg. 3 records them.  Returns the number of recorded pairs, or -1 when the pass stops
+ * before recording ("I" empty, or a single segment in the whole matrix). */
+static int64_t stage2_pass(const or_csr* B, int N, int M, int gain_rule, s2_scratch* w,
+                           int64_t* su, int64_t* sv, int64_t* sp, int64_t* st,
+                           int64_t* max_pairs_per_primary) {
+  int64_t n = B->n, S = (n + M - 1) / M;
+  int64_t wv, mbv;
+  counts_B(B, 1, N, M, &wv, &mbv, w->pscore);              /* GetPScoreList (line 1/29) */
+  int64_t nI = 0;
+  for (int64_t s = 0; s < S; ++s)
+    if (w->pscore[s] > 0) { w->I[nI].seg = s; w->I[nI].score = w->pscore[s]; ++nI; } /* line 2/30 */
+  if (nI == 0) return -1;
+  qsort(w->I, (size_t)nI, sizeof(or_item), cmp_item);
+  for (int64_t s = 0; s < S; ++s) { w->est[s] = w->pscore[s]; w->inI[s] = 0; }
+  for (int64_t k = 0; k < nI; ++k) w->inI[w->I[k].seg] = 1;
+  memset(w->used, 0, (size_t)n);
+  int64_t nS = 0;
+  if (nI == 1) {
+    /* line 6: beneficial swaps with the sparsest segment (L402 (ii), reading #16) */
+    int64_t p = w->I[0].seg;
+    if (S == 1) return -1;
+    int64_t t = -1, tn = 0;
+    for (int64_t s = 0; s < S; ++s) {
+      if (s == p) continue;
+      int64_t z = 0;
+      for (int64_t q = s * M; q < s * M + M && q < n; ++q) z += B->rp[q + 1] - B->rp[q];
+      if (t < 0 || z < tn) { t = s; tn = z; }
+    }
+    int64_t npairs = 0;
+    for (;;) {
+      or_pair pr = freshtop(B, N, M, p, t, w->used, 1);
+      if (!pr.found) break;
+      su[nS] = pr.u; sv[nS] = pr.v; sp[nS] = p; st[nS] = t; ++nS; ++npairs;
+      w->used[pr.u] = w->used[pr.v] = 1;
+      w->est[p] -= pr.gp;
+      if (w->est[p] <= 0 || all_positions_used(w->used, p, M, n)) break;
+    }
+    if (npairs > *max_pairs_per_primary) *max_pairs_per_primary = npairs;
+  } else {
+    int64_t head = 0;
+    while (1) {
+      /* |I| > 1 ?  count live entries from head */
+      int64_t live = 0;
+      for (int64_t k = head; k < nI; ++k) live += w->inI[w->I[k].seg];
+      if (live <= 1) break;
+      while (!w->inI[w->I[head].seg]) ++head;
+      int64_t p = w->I[head].seg; /* line 9: I.pop() */
+      w->inI[p] = 0;
+      ++head;
+      int64_t ns = 0;
+      for (int64_t k = head; k < nI; ++k) if (w->inI[w->I[k].seg]) w->snap[ns++] = w->I[k].seg;
+      int64_t npairs = 0;
+      for (int64_t k = 0; k < ns; ++k) { /* line 10: targets in priority order */
+        int64_t t = w->snap[k];
+        if (!w->inI[t]) continue;
+        or_pair pr = freshtop(B, N, M, p, t, w->used, gain_rule == 1);
+        if (!pr.found) continue;
+        su[nS] = pr.u; sv[nS] = pr.v; sp[nS] = p; st[nS] = t; ++nS; ++npairs; /* line 15 */
+        w->used[pr.u] = w->used[pr.v] = 1;
+        w->est[p] -= pr.gp;                             /* line 16 */
+        w->est[t] -= pr.gt;                             /* line 17 */
+        if (w->est[t] <= 0) w->inI[t] = 0;              /* lines 18-19 */
+        if (w->est[p] <= 0 || all_positions_used(w->used, p, M, n)) break; /* lines 20-22 */
+      }
+      if (npairs > *max_pairs_per_primary) *max_pairs_per_primary = npairs;
+    }
+  }
+  return nS;
+}
+
+static int s2_alloc(int64_t n, int M, s2_scratch* w, int64_t** bufs, int nbufs) {
+  int64_t S = (n + M - 1) / M;
+  size_t Sz = (size_t)(S > 0 ? S : 1), nz = (size_t)(n > 0 ? n : 1);
+  w->pscore = (int32_t*)malloc(sizeof(int32_t) * Sz);
+  w->est = (int64_t*)malloc(sizeof(int64_t) * Sz);
+  w->inI = (uint8_t*)malloc(Sz);
+  w->used = (uint8_t*)malloc(nz);
+  w->I = (or_item*)malloc(sizeof(or_item) * Sz);
+  w->snap = (int64_t*)malloc(sizeof(int64_t) * Sz);
+  for (int k = 0; k < nbufs; ++k) bufs[k] = (int64_t*)malloc(sizeof(int64_t) * nz);
+  return 0;
+}
+
+static void s2_free(s2_scratch* w, int64_t** bufs, int nbufs) {
+  free(w->pscore); free(w->est); free(w->inI); free(w->used); free(w->I); free(w->snap);
+  for (int k = 0; k < nbufs; ++k) free(bufs[k]);
+}
+
 /* One Stage-2 run (up to MAXITER2+1 passes).  Returns #passes that applied swaps;
  * *max_pairs_per_primary receives the largest number of pairs one primary recorded. */
 static int stage2(int64_t n, const int64_t* rp, const int32_t* ci, int N, int M, int maxiter,
                   int gain_rule, int32_t* perm, int64_t* max_pairs_per_primary) {
-  int64_t S = (n + M - 1) / M;
+  s2_scratch w;
+  int64_t* b[4];
+  s2_alloc(n, M, &w, b, 4);
   int passes = 0;
-  int32_t* pscore = (int32_t*)malloc(sizeof(int32_t) * (size_t)(S > 0 ? S : 1));
-  int64_t* est = (int64_t*)malloc(sizeof(int64_t) * (size_t)(S > 0 ? S : 1));
-  uint8_t* inI = (uint8_t*)malloc((size_t)(S > 0 ? S : 1));
-  uint8_t* used = (uint8_t*)malloc((size_t)(n > 0 ? n : 1));
-  int64_t* su = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
-  int64_t* sv = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
-  or_item* I = (or_item*)malloc(sizeof(or_item) * (size_t)(S > 0 ? S : 1));
   for (int it = 0; it <= maxiter; ++it) {
     or_csr B;
     build_B(n, rp, ci, perm, &B);
-    int64_t w, mbv;
-    counts_B(&B, 1, N, M, &w, &mbv, pscore);              /* GetPScoreList (line 1/29) */
-    int64_t nI = 0;
-    for (int64_t s = 0; s < S; ++s)
-      if (pscore[s] > 0) { I[nI].seg = s; I[nI].score = pscore[s]; ++nI; } /* line 2/30 */
-    if (nI == 0) { csr_free(&B); break; }
-    qsort(I, (size_t)nI, sizeof(or_item), cmp_item);
-    for (int64_t s = 0; s < S; ++s) { est[s] = pscore[s]; inI[s] = 0; }
-    for (int64_t k = 0; k < nI; ++k) inI[I[k].seg] = 1;
-    memset(used, 0, (size_t)n);
-    int64_t nS = 0;
-    if (nI == 1) {
-      /* line 6: beneficial swaps with the sparsest segment (L402 (ii), reading #16) */
-      int64_t p = I[0].seg;
-      if (S == 1) { csr_free(&B); break; }
-      int64_t t = -1, tn = 0;
-      for (int64_t s = 0; s < S; ++s) {
-        if (s == p) continue;
-        int64_t z = 0;
-        for (int64_t q = s * M; q < s * M + M && q < n; ++q) z += B.rp[q + 1] - B.rp[q];
-        if (t < 0 || z < tn) { t = s; tn = z; }
-      }
-      int64_t npairs = 0;
-      for (;;) {
-        or_pair pr = freshtop(&B, N, M, p, t, used, 1);
-        if (!pr.found) break;
-        su[nS] = pr.u; sv[nS] = pr.v; ++nS; ++npairs;
-        used[pr.u] = used[pr.v] = 1;
-        est[p] -= pr.gp;
-        if (est[p] <= 0 || all_positions_used(used, p, M, n)) break;
-      }
-      if (npairs > *max_pairs_per_primary) *max_pairs_per_primary = npairs;
-    } else {
-      int64_t head = 0;
-      int64_t* snap = (int64_t*)malloc(sizeof(int64_t) * (size_t)nI);
-      while (1) {
-        /* |I| > 1 ?  count live entries from head */
-        int64_t live = 0;
-        for (int64_t k = head; k < nI; ++k) live += inI[I[k].seg];
-        if (live <= 1) break;
-        while (!inI[I[head].seg]) ++head;
-        int64_t p = I[head].seg; /* line 9: I.pop() */
-        inI[p] = 0;
-        ++head;
-        int64_t ns = 0;
-        for (int64_t k = head; k < nI; ++k) if (inI[I[k].seg]) snap[ns++] = I[k].seg;
-        int64_t npairs = 0;
-        for (int64_t k = 0; k < ns; ++k) { /* line 10: targets in priority order */
-          int64_t t = snap[k];
-          if (!inI[t]) continue;
-          or_pair pr = freshtop(&B, N, M, p, t, used, gain_rule == 1);
-          if (!pr.found) continue;
-          su[nS] = pr.u; sv[nS] = pr.v; ++nS; ++npairs; /* line 15 */
-          used[pr.u] = used[pr.v] = 1;
-          est[p] -= pr.gp;                             /* line 16 */
-          est[t] -= pr.gt;                             /* line 17 */
-          if (est[t] <= 0) inI[t] = 0;                 /* lines 18-19 */
-          if (est[p] <= 0 || all_positions_used(used, p, M, n)) break; /* lines 20-22 */
-        }
-        if (npairs > *max_pairs_per_primary) *max_pairs_per_primary = npairs;
-      }
-      free(snap);
-    }
+    int64_t nS = stage2_pass(&B, N, M, gain_rule, &w, b[0], b[1], b[2], b[3], max_pairs_per_primary);
     csr_free(&B);
-    if (nS == 0) break;
-    for (int64_t k = 0; k < nS; ++k) { /* lines 24-27: apply the recorded swaps together */
-      int32_t tmp = perm[su[k]];
-      perm[su[k]] = perm[sv[k]];
-      perm[sv[k]] = tmp;
+    if (nS <= 0) break;                 /* nothing recorded: the state is unchanged */
+    for (int64_t k = 0; k < nS; ++k) {  /* lines 24-27: apply the recorded swaps together */
+      int32_t tmp = perm[b[0][k]];
+      perm[b[0][k]] = perm[b[1][k]];
+      perm[b[1][k]] = tmp;
     }
     ++passes;
   }
-  free(pscore); free(est); free(inI); free(used); free(su); free(sv); free(I);
+  s2_free(&w, b, 4);
   return passes;
+}
+
+/* Trace of ONE Stage-2 pass from perm (for the hand-derived pins, tests/golden/s2_*.txt):
+ * pairs_out[4k..4k+3] = (primary segment, target segment, u, v) of the k-th recorded pair
+ * (u, v = positions of the pass-start order), in recording order.  pairs_out holds room for
+ * n pairs.  Returns the number of pairs, -1 when the pass stops before recording. */
+int64_t or_stage2_trace(int64_t n, const int64_t* rp, const int32_t* ci, const int32_t* perm, int N,
+                        int M, int gain_rule, int64_t* pairs_out) {
+  s2_scratch w;
+  int64_t* b[4];
+  s2_alloc(n, M, &w, b, 4);
+  or_csr B;
+  build_B(n, rp, ci, perm, &B);
+  int64_t mp = 0;
+  int64_t nS = stage2_pass(&B, N, M, gain_rule, &w, b[0], b[1], b[2], b[3], &mp);
+  for (int64_t k = 0; k < nS; ++k) {
+    pairs_out[4 * k] = b[2][k]; pairs_out[4 * k + 1] = b[3][k];
+    pairs_out[4 * k + 2] = b[0][k]; pairs_out[4 * k + 3] = b[1][k];
+  }
+  csr_free(&B);
+  s2_free(&w, b, 4);
+  return nS;
 }
 
 /* ------------------------------------------------------------------------------------- */
