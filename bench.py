@@ -34,6 +34,17 @@ sys.path.insert(0, ROOT)
 WORKLOADS = {
     # configs[0]: ER n = 2048, m = 16384, F = 32, 2:4, fp16 (oracle-sized correctness case)
     "c1-er-n2048-f32-1:2:4": dict(kind="er", n=2048, m=16384, F=32, V=1, M=4, dtype="f16", tau=0),
+    # configs[2]: Reddit-shaped (n 232,965, ~114.8M directed edges + I), GCN aggregation of
+    # the 602 -> 128 layer at F = 128, bf16, Ahat sym-normalised (the N = 1 headline)
+    "c3-reddit-f128-1:2:4": dict(kind="gnn", graph="reddit", F=128, V=1, M=4, dtype="bf16", tau=None),
+    "c3-reddit-f128-128:2:16": dict(kind="gnn", graph="reddit", F=128, V=128, M=16, dtype="bf16", tau=None),
+    # configs[3]: ogbn-proteins-shaped (132,534 / 79.12M directed + I), F = 256, 128:2:16
+    "c4-proteins-f256-128:2:16": dict(kind="gnn", graph="proteins", F=256, V=128, M=16, dtype="bf16",
+                                      tau=None),
+    # configs[4]: ogbn-products-shaped (2,449,029 / 123.72M directed + I), aggregation at
+    # F = 100 (aggregate-first 100 -> 256), 128:2:8
+    "c5-products-f100-128:2:8": dict(kind="gnn", graph="products", F=100, V=128, M=8, dtype="bf16",
+                                     tau=None),
 }
 # configs[1] (SuiteSparse-shaped sweep): any point named
 #   c2-{banded|powerlaw}-n{65k|262k|1m}-d{8|16|32|64}-f{F}-{V}:2:{M}[-tau{T}]
@@ -60,6 +71,13 @@ def parse_workload(name):
 METRIC = "V:N:M SpMM GFLOP/s & % sparse-MMA/HBM roofline vs cuSPARSE, 1/2/4/8 B200"
 
 
+def default_reorder_opts(w):
+    """The reorder options bench.py uses for workload w (nm_reorder defaults: MAXITER = 10 for
+    Alg. 1-3; the GNN-shaped graphs take the workload's own caps)."""
+    return dict(max_outer=w.get("max_outer", 10), max_stage1=w.get("max_stage1", 10),
+                max_stage2=w.get("max_stage2", 10), gain_rule=0)
+
+
 def make_graph(w):
     from paper_conf_ppopp_chensz0s25_b200 import graphs
     if w["kind"] == "band":
@@ -71,6 +89,11 @@ def make_graph(w):
     elif w["kind"] == "er":
         seed = 1
         ip, ic = graphs.er_graph(w["n"], w["m"], seed)
+    elif w["kind"] == "gnn":
+        ip, ic = graphs.gnn_graph(w["graph"])
+        w["n"] = len(ip) - 1
+        # Ahat values (GCN normalisation) and an N(0,1) operand of the aggregation's width
+        return ip, ic, graphs.gcn_norm_values(ip, ic), graphs.features(w["n"], w["F"], 7, "normal")
     else:
         raise ValueError(w["kind"])
     vals = graphs.symmetric_values(ip, ic, seed + 1)
@@ -220,9 +243,23 @@ def main():
     ap.add_argument("--no-cusparse", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--order", default="original", choices=["original", "permuted"])
+    ap.add_argument("--tau", type=int, default=None, help="hybrid threshold (default: the workload's / nm_hybrid_tau)")
+    ap.add_argument("--max-outer", type=int, default=None, help="Alg. 1 cap (default: the workload's, else 10, L496)")
+    ap.add_argument("--max-stage1", type=int, default=None)
+    ap.add_argument("--max-stage2", type=int, default=None)
+    ap.add_argument("--gain-rule", type=int, default=0, help="0 = paper (footnote L440), 1 = positive only")
+    ap.add_argument("--sptc-format", type=int, default=0, help="tensor-core kernel: 0 = the pack's choice, 1 = full "
+                    "records, 2 = compressed records (nm_spmm_sptc_format)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     w = parse_workload(args.workload)
+    if args.tau is not None:
+        w["tau"] = args.tau
+    ropts = default_reorder_opts(w)
+    for k in ("max_outer", "max_stage1", "max_stage2"):
+        if getattr(args, k) is not None:
+            ropts[k] = getattr(args, k)
+    ropts["gain_rule"] = args.gain_rule
     if args.impl == "reference":
         return run_reference(args, w)
 
@@ -241,10 +278,12 @@ def main():
     dev = torch.device("cuda", local_dev)
     cdev = dev if backend == "nccl" else torch.device("cpu")  # where collective buffers live
     if world > 1:
+        import datetime
+        tmo = datetime.timedelta(hours=2)  # graph generation + reorder run before the first collective
         if backend == "nccl":
-            dist.init_process_group("nccl", device_id=dev)
+            dist.init_process_group("nccl", device_id=dev, timeout=tmo)
         else:
-            dist.init_process_group("gloo")
+            dist.init_process_group("gloo", timeout=tmo)
 
     # ---------------- inputs (seeded, synthetic) and offline preprocessing ----------------
     t0 = time.perf_counter()
@@ -252,20 +291,9 @@ def main():
     gen_s = time.perf_counter() - t0
     n, F, V, M, dt = w["n"], w["F"], w["V"], w["M"], w["dtype"]
     nnz = int(ip[-1])
-    if world == 1:
-        perm, rst = api.reorder(ip, ic, V, 2, M, device=True)  # nm_reorder_gpu (untimed)
-    else:
-        # one rank reorders (nm_reorder_gpu), the permutation is broadcast over NCCL
-        keys = ("omega_init", "omega_final", "mb_init", "mb_final", "seconds")
-        buf = torch.zeros(n + len(keys), dtype=torch.float64, device=cdev)
-        if rank == 0:
-            perm, rst = api.reorder(ip, ic, V, 2, M, device=True)
-            buf[:n] = torch.from_numpy(perm.astype(np.float64)).to(cdev)
-            buf[n:] = torch.tensor([float(rst[k]) for k in keys], dtype=torch.float64, device=cdev)
-        dist.broadcast(buf, 0)
-        hb = buf.cpu().numpy()
-        perm = hb[:n].astype(np.int32)
-        rst = {k: (float(v) if k == "seconds" else int(v)) for k, v in zip(keys, hb[n:])}
+    # nm_reorder_gpu (untimed preprocessing).  Deterministic: every rank computes the same
+    # permutation itself, so no rank waits in a collective while another reorders
+    perm, rst = api.reorder(ip, ic, V, 2, M, device=True, **ropts)
     # contiguous panel-aligned row blocks balanced by stored entries + Y rows
     from paper_conf_ppopp_chensz0s25_b200.dist import balanced_bounds, panel_costs
     rb, re = balanced_bounds(panel_costs(ip, perm), n, world)[rank]
@@ -277,10 +305,13 @@ def main():
     info = P.info()
     xbits, _ = graphs.round16(X32, dt)
     tdt = torch.float16 if dt == "f16" else torch.bfloat16
-    X = torch.from_numpy(xbits.view(np.int16)).to(dev).view(tdt)
-    Y = torch.empty((n, F), dtype=torch.float32, device=dev)
+    Fp = (F + 7) // 8 * 8  # rows padded to 16 B (ldx % 8 == 0; C5's F = 100 -> 104 in memory)
+    Xpad = torch.zeros((n, Fp), dtype=torch.int16, device=dev)
+    Xpad[:, :F] = torch.from_numpy(xbits.view(np.int16)).to(dev)
+    X = Xpad.view(tdt)[:, :F]
+    Y = torch.empty((n, Fp), dtype=torch.float32, device=dev)[:, :F]
     perm_d = torch.from_numpy(perm).to(dev)
-    PX = torch.empty_like(X) if args.order == "permuted" else None
+    PX = padded_like(X) if args.order == "permuted" else None
     Yp = torch.empty((re - rb, F), dtype=torch.float32, device=dev) if args.order == "permuted" else None
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
     stream = torch.cuda.current_stream()
@@ -289,7 +320,7 @@ def main():
     def step(ev=None):
         if args.order == "original":
             if ev: ev[0].record(stream)
-            api.spmm(P, X, Y, part="sptc")
+            api.spmm(P, X, Y, part="sptc", format=args.sptc_format)
             if ev: ev[1].record(stream)
             if has_res:
                 api.spmm(P, X, Y, part="residual")
@@ -297,7 +328,7 @@ def main():
         else:
             if ev: ev[0].record(stream)
             api.permute_rows(X, PX, perm_d, dt)
-            api.spmm(P, PX, Yp, part="sptc")
+            api.spmm(P, PX, Yp, part="sptc", format=args.sptc_format)
             if ev: ev[1].record(stream)
             if has_res:
                 api.spmm(P, PX, Yp, part="residual")
@@ -427,7 +458,7 @@ def main():
                 "gpu_launches": launches_per_step * args.steps,
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "cusparse": cus,
-                "preprocess": {"gen_s": gen_s, "reorder": "nm_reorder_gpu", "reorder_s": rst["seconds"], "pack_s": pack_s,
+                "preprocess": {"gen_s": gen_s, "reorder": "nm_reorder_gpu", "reorder_opts": ropts, "reorder_s": rst["seconds"], "pack_s": pack_s,
                                "omega_init": rst["omega_init"], "omega_final": rst["omega_final"],
                                "mb_init": rst["mb_init"], "mb_final": rst["mb_final"],
                                "violation_removal": (None if rst["omega_init"] == 0 else
@@ -452,6 +483,13 @@ def main():
         dist.destroy_process_group()
 
 
+def padded_like(t):
+    """Uninitialised tensor of t's shape and dtype whose rows keep t's (16-byte padded) stride."""
+    import torch
+    base = torch.empty((t.shape[0], t.stride(0)), dtype=t.dtype, device=t.device)
+    return base[:, :t.shape[1]]
+
+
 def e2e_pipelined(P, X, Y, F, steps, useful_flop):
     """End to end through the public API with host buffers: every step copies its X from
     pinned host memory, runs nm_spmm and reads Y back to pinned host memory.  Serving-style
@@ -463,8 +501,8 @@ def e2e_pipelined(P, X, Y, F, steps, useful_flop):
     Xh = torch.empty(X.shape, dtype=X.dtype).pin_memory()
     Xh.copy_(X.cpu())
     Yh = [torch.empty((Y.shape[0], F), dtype=torch.float32).pin_memory() for _ in range(2)]
-    Xd = [X, torch.empty_like(X)]
-    Yd = [Y, torch.empty_like(Y)]
+    Xd = [X, padded_like(X)]
+    Yd = [Y, padded_like(Y)]
     s_h2d, s_cmp, s_d2h = torch.cuda.Stream(), torch.cuda.Stream(), torch.cuda.Stream()
     ev = lambda: torch.cuda.Event(enable_timing=True)
 
@@ -515,9 +553,9 @@ def permuted_csr(ip, ic, vals, perm):
     lens = ip[pv + 1] - ip[pv]
     Bp = np.concatenate([[0], np.cumsum(lens)]).astype(np.int64)
     idx = np.repeat(ip[pv] - Bp[:-1], lens) + np.arange(Bp[-1])
-    rows = np.repeat(np.arange(n), lens)
+    rows = np.repeat(np.arange(n, dtype=np.int64), lens)
     cols = iperm[ic[idx]]
-    o = np.lexsort((cols, rows))
+    o = np.argsort(rows * n + cols)
     return Bp, cols[o].astype(np.int32), vals[idx][o]
 
 

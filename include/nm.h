@@ -244,6 +244,16 @@ NM_API nm_status nm_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, f
 NM_API nm_status nm_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                            int64_t ldy, int F, void* stream);
 
+/* nm_spmm_sptc_format -- nm_spmm_sptc with an explicit choice of the tensor-core kernel, for
+ * profiling and A/B measurement:
+ *   format 0 = the pack's choice (what nm_spmm runs), 1 = full-record kernel (one bulk copy of
+ *   the MMA operands per K = 32 chunk, no expansion), 2 = compressed-record kernel (HBM holds
+ *   only the non-empty (row, meta-block) slots; loader warps expand them in shared memory).
+ * Both compute the same Yp (bitwise: identical operands and MMA order).  Errors as nm_spmm,
+ * plus INVALID_ARG for another format. */
+NM_API nm_status nm_spmm_sptc_format(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
+                                     int64_t ldy, int F, int format, void* stream);
+
 /* ---------------------------------------------------------------------------------------
  * nm_gcn_layer -- one GCN layer (Eq. 1): Hout = act(Ahat (H W) + bias).
  *   Ahat : packed normalised adjacency in permuted order (P Ahat P^T, pack flags 0), rows

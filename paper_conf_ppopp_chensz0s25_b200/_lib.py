@@ -88,6 +88,8 @@ SIGNATURES = {
                                          ctypes.c_int, VP]),
     "nm_spmm": (ctypes.c_int, [VP, VP, ctypes.c_int64, VP, ctypes.c_int64, ctypes.c_int, VP]),
     "nm_spmm_sptc": (ctypes.c_int, [VP, VP, ctypes.c_int64, VP, ctypes.c_int64, ctypes.c_int, VP]),
+    "nm_spmm_sptc_format": (ctypes.c_int, [VP, VP, ctypes.c_int64, VP, ctypes.c_int64, ctypes.c_int, ctypes.c_int,
+                                           VP]),
     "nm_spmm_residual": (ctypes.c_int, [VP, VP, ctypes.c_int64, VP, ctypes.c_int64, ctypes.c_int,
                                         VP]),
     "nm_gcn_workspace_bytes": (ctypes.c_size_t, [ctypes.c_int64, ctypes.c_int, ctypes.c_int]),

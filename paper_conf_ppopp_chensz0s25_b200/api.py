@@ -200,9 +200,16 @@ def hybrid_tau(F: int) -> int:
     return int(L.load().nm_hybrid_tau(int(F)))
 
 
-def spmm(P: Packed, PX, Yp, F=None, stream=None, part="all"):
-    """Yp (fp32 CUDA tensor, rows x F) = packed B * PX (16-bit CUDA tensor, n x F)."""
+def spmm(P: Packed, PX, Yp, F=None, stream=None, part="all", format=None):
+    """Yp (fp32 CUDA tensor, rows x F) = packed B * PX (16-bit CUDA tensor, n x F).
+    part: 'all' | 'sptc' | 'residual'; format (part='sptc' only): None / 0 = the pack's choice,
+    1 = full-record kernel, 2 = compressed-record kernel (nm_spmm_sptc_format)."""
     F = PX.shape[1] if F is None else F
+    if format is not None:
+        assert part == "sptc"
+        L.check(L.load().nm_spmm_sptc_format(P.handle, _ptr(PX), PX.stride(0), _ptr(Yp), Yp.stride(0), F,
+                                             int(format), _stream_ptr(stream)), "nm_spmm_sptc_format")
+        return
     fn = {"all": "nm_spmm", "sptc": "nm_spmm_sptc", "residual": "nm_spmm_residual"}[part]
     L.check(getattr(L.load(), fn)(P.handle, _ptr(PX), PX.stride(0), _ptr(Yp), Yp.stride(0), F,
                                   _stream_ptr(stream)), fn)

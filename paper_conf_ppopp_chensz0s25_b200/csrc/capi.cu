@@ -29,6 +29,41 @@ nm_status cuda_fail(cudaError_t e, const char* what) {
 
 uint16_t one_bits(nm_dtype dt) { return dt == NM_BF16 ? (uint16_t)0x3F80 : (uint16_t)0x3C00; }
 
+namespace {
+thread_local cudaMemPool_t t_scratch_pool = nullptr;
+}
+
+nm_status scratch_alloc(void** p, size_t bytes, cudaStream_t s) {
+  if (bytes == 0) bytes = 16;
+  if (t_scratch_pool) {
+    NM_CUDA(cudaMallocFromPoolAsync(p, bytes, t_scratch_pool, s));
+  } else {
+    NM_CUDA(cudaMallocAsync(p, bytes, s));
+  }
+  return NM_OK;
+}
+
+nm_status ScopedPool::init(int device) {
+  cudaMemPoolProps props = {};
+  props.allocType = cudaMemAllocationTypePinned;
+  props.handleTypes = cudaMemHandleTypeNone;
+  props.location.type = cudaMemLocationTypeDevice;
+  props.location.id = device;
+  NM_CUDA(cudaMemPoolCreate(&pool, &props));
+  uint64_t keep = UINT64_MAX;
+  NM_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep));
+  prev = t_scratch_pool;
+  t_scratch_pool = pool;
+  return NM_OK;
+}
+
+ScopedPool::~ScopedPool() {
+  if (!pool) return;
+  t_scratch_pool = prev;
+  cudaDeviceSynchronize();  // every stream-ordered free into the pool has executed
+  cudaMemPoolDestroy(pool);
+}
+
 nm_status validate_csr_host(int64_t n, const int64_t* rp, const int32_t* ci, bool check_sym) {
   if (n < 0) return fail(NM_ERR_INVALID_ARG, "n < 0");
   if (rp[0] != 0) return fail(NM_ERR_BAD_CSR, "rowptr[0] != 0");
@@ -186,7 +221,7 @@ void nm_packed_free(nm_packed* P) {
   cudaSetDevice(P->device);
   void* ptrs[] = {P->panel_mb_ptr, P->panel_chunk_ptr, P->unit_info, P->mb_seg, P->mb_sel,
                   P->image, P->res_rowptr, P->res_col, P->res_val, P->row_map,
-                  P->res_gather, P->res_segs, P->res_ws, P->res_cnt, P->rec_len16};
+                  P->res_gather, P->res_segs, P->rec_len16, P->image_full, P->cta_ptr};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   cudaSetDevice(cur);

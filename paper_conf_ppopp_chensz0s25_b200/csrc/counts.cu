@@ -69,8 +69,7 @@ struct Buf {
   ~Buf() { if (p) cudaFreeAsync(p, st); }
   nm_status alloc(size_t n, cudaStream_t s) {
     st = s;
-    NM_CUDA(cudaMallocAsync(&p, sizeof(T) * (n > 0 ? n : 1), s));
-    return NM_OK;
+    return scratch_alloc((void**)&p, sizeof(T) * (n > 0 ? n : 1), s);
   }
 };
 
@@ -150,8 +149,8 @@ nm_status count_violations_dev(const DevCsr& A, const int32_t* perm_dev, int V, 
 
 }  // namespace nm
 
-extern "C" nm_status nm_count_violations(const nm_csr* A, const int32_t* perm, int V, int N, int M,
-                                         int64_t* omega, int64_t* mbscore, int32_t* pscore) {
+static nm_status count_violations_impl(const nm_csr* A, const int32_t* perm, int V, int N, int M,
+                                       int64_t* omega, int64_t* mbscore, int32_t* pscore) {
   using namespace nm;
   if (!A || !omega || !mbscore) return fail(NM_ERR_INVALID_ARG, "nm_count_violations: NULL argument");
   if (V < 1 || N < 1 || M <= N || M > 32) return fail(NM_ERR_UNSUPPORTED, "nm_count_violations: bad V/N/M");
@@ -160,22 +159,35 @@ extern "C" nm_status nm_count_violations(const nm_csr* A, const int32_t* perm, i
     nm_status st = validate_csr_host(A->n, A->rowptr, A->col, false);
     if (st != NM_OK) return st;
   }
+  if (perm) {  // a bad permutation would index out of bounds on the device (k_inv)
+    std::vector<uint8_t> seen((size_t)A->n, 0);
+    for (int64_t p = 0; p < A->n; ++p) {
+      const int32_t v = perm[p];
+      if (v < 0 || v >= A->n || seen[(size_t)v]) return fail(NM_ERR_INVALID_ARG, "nm_count_violations: perm is not a permutation");
+      seen[(size_t)v] = 1;
+    }
+  }
   cudaStream_t s = 0;
   DevCsr d;
   nm_csr pattern = *A;
   pattern.val = nullptr;  // counts need the pattern only
   nm_status st = upload_csr(&pattern, NM_F16, &d, s);
   if (st != NM_OK) return st;
-  int32_t* dperm = nullptr;
+  Buf<int32_t> dperm;
   if (perm) {
-    NM_CUDA(cudaMalloc(&dperm, sizeof(int32_t) * A->n));
-    NM_CUDA(cudaMemcpy(dperm, perm, sizeof(int32_t) * A->n, cudaMemcpyHostToDevice));
+    if ((st = dperm.alloc((size_t)A->n, s))) return st;
+    NM_CUDA(cudaMemcpyAsync(dperm.p, perm, sizeof(int32_t) * A->n, cudaMemcpyHostToDevice, s));
   }
   int64_t w = 0, m = 0;
-  st = count_violations_dev(d, dperm, V, N, M, &w, &m, pscore, s);
-  if (dperm) cudaFree(dperm);
+  st = count_violations_dev(d, dperm.p, V, N, M, &w, &m, pscore, s);
   if (st != NM_OK) return st;
   *omega = w;
   *mbscore = m;
   return NM_OK;
+}
+
+extern "C" nm_status nm_count_violations(const nm_csr* A, const int32_t* perm, int V, int N, int M,
+                                         int64_t* omega, int64_t* mbscore, int32_t* pscore) {
+  return nm::guarded("nm_count_violations",
+                     [&] { return count_violations_impl(A, perm, V, N, M, omega, mbscore, pscore); });
 }

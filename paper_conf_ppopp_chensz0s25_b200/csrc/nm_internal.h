@@ -4,6 +4,9 @@
 
 #include <cuda_runtime.h>
 #include <stdint.h>
+
+#include <exception>
+#include <new>
 #include <string>
 
 #include "../../include/nm.h"
@@ -52,18 +55,21 @@ constexpr int kRecHdrBytes = 288;
 constexpr int kRecMaxBytes = kRecHdrBytes + 4 * (kPanelRows + kPanelRows * kChunkMB);  // 4896
 
 // Residual work items (DESIGN.md §6 k_residual): each row's residual nonzeros are cut into
-// segments of at most kResSeg entries, one warp each, so hub rows of power-law graphs spread
-// over many warps.  A row cut into several segments combines its segments' partial sums
-// deterministically: each writes its partial to its workspace slot, and the last segment to
-// finish (per-row arrival counter) adds all partials in segment order into Y.
+// items of at most kResSeg entries, one warp subgroup each, so hub rows of power-law graphs
+// spread over many subgroups.  A row cut into several items ("split row") combines their
+// partial sums deterministically: each item writes its partial to its workspace slot and the
+// last one to finish (per-row arrival counter) adds all partials in item order into Y.  The
+// workspace and the counters are allocated per nm_spmm call, stream-ordered (launch time),
+// never stored in the handle -- the packed matrix stays immutable, so concurrent calls on one
+// handle are safe.
 constexpr int kResSeg = 256;   // max residual nonzeros per work item
 constexpr int kResSlab = 256;  // features per residual launch (partial-sum slot width)
 struct ResSeg {
   int64_t kb;        // first residual entry
   int32_t row, len;  // packed row (local), #entries
-  int32_t slot;      // first workspace slot of the row's partials, -1 = single-segment row
+  int32_t slot;      // first workspace slot of the row's partials, -1 = single-item row
   int32_t split_id;  // arrival counter of the row (split rows only)
-  int32_t nseg, idx; // segments of the row, index of this one
+  int32_t nseg, idx; // items of the row, index of this one
   int32_t yrow;      // output row of Y (row_map applied in NM_PACK_ORIGINAL_ORDER)
   int32_t pad;
 };
@@ -89,6 +95,10 @@ struct nm_packed {
   int32_t* mb_seg = nullptr;           // [n_mb]
   uint32_t* mb_sel = nullptr;          // [n_mb] byte j = sel[j]
   uint8_t* image = nullptr;            // compressed chunk records (kRec* layout), image_bytes
+  uint8_t* image_full = nullptr;       // full chunk records (kChunkBytes each, chunk order)
+  int32_t* cta_ptr = nullptr;          // [n_ctas+1] contiguous panel range of each SpMM CTA
+  int n_ctas = 0;                      // persistent grid of the full-record kernel (#SMs)
+  int sptc_format = 1;                 // tensor-core kernel nm_spmm uses: 1 full, 2 compressed
   int64_t* res_rowptr = nullptr;       // [rows+1]
   int32_t* res_col = nullptr;          // [res_nnz] canonical (permuted) column
   uint16_t* res_val = nullptr;         // [res_nnz]
@@ -96,12 +106,11 @@ struct nm_packed {
   int flags = 0;
   int32_t* row_map = nullptr;          // [rows] output row of Y = perm[row_begin + l]
   int32_t* res_gather = nullptr;       // [res_nnz] X row to gather = perm[res_col]
-  // residual work list (kResSeg-entry segments) and the split rows' partial-sum workspace;
-  // the workspace makes concurrent nm_spmm calls on one handle unsafe (stream-order them)
+  // residual work list (kResSeg-entry items, longest first); the split rows' partial-sum
+  // workspace (n_res_slots x kResSlab floats) and arrival counters (n_res_split) are allocated
+  // by each nm_spmm call on its stream
   nm::ResSeg* res_segs = nullptr;      // [n_res_segs]
   int64_t n_res_segs = 0, n_res_slots = 0, n_res_split = 0;
-  float* res_ws = nullptr;             // [n_res_slots * kResSlab]
-  int32_t* res_cnt = nullptr;          // [n_res_split] arrival counters (0 between launches)
   size_t device_bytes = 0;
 };
 
@@ -117,6 +126,33 @@ nm_status cuda_fail(cudaError_t e, const char* what);
     cudaError_t e_ = (call);                              \
     if (e_ != cudaSuccess) return nm::cuda_fail(e_, #call); \
   } while (0)
+
+// exception guard for the extern "C" entry points: no C++ exception crosses the ABI
+// (std::vector / std::bad_alloc in the host stages, CUB temporaries); nm.h promises status codes
+template <typename Fn>
+nm_status guarded(const char* what, Fn&& f) {
+  try {
+    return f();
+  } catch (const std::bad_alloc&) {
+    return fail(NM_ERR_OOM, std::string(what) + ": host allocation failed");
+  } catch (const std::exception& e) {
+    return fail(NM_ERR_CUDA, std::string(what) + ": " + e.what());
+  } catch (...) {
+    return fail(NM_ERR_CUDA, std::string(what) + ": unknown exception");
+  }
+}
+
+// stream-ordered scratch of the offline stages (reorder Stage-1, counts).  While a ScopedPool
+// is alive on this thread the allocations come from its private pool (kept reserved between
+// the reorder's iterations and destroyed with it -- the device's default pool, which other
+// users such as PyTorch's cudaMallocAsync backend share, is never reconfigured); otherwise
+// from the current device's default pool.
+nm_status scratch_alloc(void** p, size_t bytes, cudaStream_t s);
+struct ScopedPool {
+  cudaMemPool_t pool = nullptr, prev = nullptr;
+  nm_status init(int device);
+  ~ScopedPool();
+};
 
 // host-side CSR validation (sorted, in range, no duplicates; optional symmetry check)
 nm_status validate_csr_host(int64_t n, const int64_t* rp, const int32_t* ci, bool check_sym);
@@ -140,6 +176,12 @@ uint16_t one_bits(nm_dtype dt);
 // kernels launched from other translation units
 nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                            int64_t ldy, int F, cudaStream_t s);
+nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy,
+                           int F, cudaStream_t s, int format);
+nm_status launch_spmm_sptc_full(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
+                                int64_t ldy, int F, cudaStream_t s);
+nm_status launch_spmm_sptc_compressed(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
+                                      int64_t ldy, int F, cudaStream_t s);
 nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                                int64_t ldy, int F, cudaStream_t s);
 nm_status count_violations_dev(const DevCsr& A, const int32_t* perm_dev, int V, int N, int M,

@@ -37,8 +37,23 @@ __device__ __forceinline__ float fma16(unsigned short a, unsigned short b, float
 // time) is read next to the first (col, val) batch.  A row with one item adds its sum into Y;
 // the items of a split row (hub rows) write partials to their workspace slots and the last
 // one to arrive (per-row counter) adds the partials in item order -- deterministic, no float
-// atomics.  F tail: the 16-byte vector at column f < F is inside the row (ldx % 8 == 0), only
+// atomics.  The workspace and counters are the calling nm_spmm's own (stream-ordered
+// allocation, counters zeroed per call), so the packed handle is only read.  F tail: the 16-byte vector at column f < F is inside the row (ldx % 8 == 0), only
 // the accumulate/store is masked.
+#ifndef NM_RES_CPASYNC
+#define NM_RES_CPASYNC 1  // X rows via cp.async into a per-subgroup shared-memory ring (0: registers)
+#endif
+constexpr int kResBatch = 8;  // entries per cp.async batch (two batches in flight per subgroup)
+
+template <int LPR>
+constexpr int res_smem_bytes() {
+  return NM_RES_CPASYNC ? 8 * (32 / LPR) * 2 * (LPR < kResBatch ? LPR : kResBatch) * LPR * 16 : 0;
+}
+
+__device__ __forceinline__ void cp_async16_z(uint32_t dst, const void* src, uint32_t nbytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(nbytes) : "memory");
+}
+
 template <int BF, int LPR>
 __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ segs, int64_t n_segs,
                                                   const int32_t* __restrict__ rc, const uint16_t* __restrict__ rv,
@@ -47,12 +62,20 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
                                                   float* __restrict__ ws, int32_t* __restrict__ cnt) {
   constexpr int SUB = 32 / LPR;
   constexpr int kUnroll = NM_RES_UNROLL;
+  constexpr int KB = LPR < kResBatch ? LPR : kResBatch;
+  extern __shared__ __align__(16) uint8_t res_smem[];
   const int lane = threadIdx.x & 31;
   const int sub = lane / LPR, li = lane % LPR;
   const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (sub * LPR));
   const int f = f_base + li * 8;  // first feature of this lane
   const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5) * SUB;  // subgroups in the grid
   const bool vec_y = ((ldy & 3) == 0) && ((((uintptr_t)Y) & 15) == 0) && f + 8 <= F;
+  // this lane's slots of its subgroup's ring: slot (batch parity b, entry j) at
+  // ring + ((b * KB + j) * LPR) * 16 (a lane reads back only the pieces it copied itself, so
+  // cp.async.wait_group is all the synchronisation the ring needs)
+  const uint32_t ring = (uint32_t)__cvta_generic_to_shared(res_smem) +
+                        (uint32_t)((((threadIdx.x >> 5) * SUB + sub) * 2 * KB * LPR + li) * 16);
+  const uint32_t xbytes = f < F ? 16u : 0u;
   int64_t w = ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5) * SUB + sub;
   ResSeg gn;
   if (w < n_segs) gn = segs[w];
@@ -70,6 +93,61 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
     float acc[8];
 #pragma unroll
     for (int q = 0; q < 8; ++q) acc[q] = 0.f;
+#if NM_RES_CPASYNC
+    // two batches of KB entries in flight: batch k+1's X rows are copied (cp.async, no
+    // registers held) while batch k is accumulated from shared memory
+    const int nb = (g.len + KB - 1) / KB;
+    int32_t cn = 0;
+    uint32_t vn = 0u, vc = 0u;
+    if (li < KB && li < g.len) {
+      cn = __ldg(rc + g.kb + li);
+      vn = __ldg(rv + g.kb + li);
+    }
+    {  // issue batch 0
+      const int cnt0 = min(KB, g.len);
+      for (int j = 0; j < cnt0; ++j) {
+        const int32_t cc = __shfl_sync(gmask, cn, j, LPR);
+        cp_async16_z(ring + j * LPR * 16, X + (int64_t)cc * ldx + (xbytes ? f : 0), xbytes);
+      }
+      asm volatile("cp.async.commit_group;" ::: "memory");
+    }
+    for (int k = 0; k < nb; ++k) {
+      vc = vn;
+      const int cntk = min(KB, g.len - k * KB);
+      if (k + 1 < nb) {
+        const int e1 = (k + 1) * KB;
+        const int cnt1 = min(KB, g.len - e1);
+        cn = 0;
+        vn = 0u;
+        if (li < cnt1) {
+          cn = __ldg(rc + g.kb + e1 + li);
+          vn = __ldg(rv + g.kb + e1 + li);
+        }
+        const uint32_t rb = ring + ((k + 1) & 1) * KB * LPR * 16;
+        for (int j = 0; j < cnt1; ++j) {
+          const int32_t cc = __shfl_sync(gmask, cn, j, LPR);
+          cp_async16_z(rb + j * LPR * 16, X + (int64_t)cc * ldx + (xbytes ? f : 0), xbytes);
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+      } else {
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
+      }
+      const uint32_t rb = ring + (k & 1) * KB * LPR * 16;
+      for (int j = 0; j < cntk; ++j) {
+        const unsigned short a = (unsigned short)__shfl_sync(gmask, vc, j, LPR);
+        uint32_t wv[4];
+        asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                     : "=r"(wv[0]), "=r"(wv[1]), "=r"(wv[2]), "=r"(wv[3])
+                     : "r"(rb + j * LPR * 16));
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          acc[2 * q] = fma16<BF>(a, (unsigned short)(wv[q] & 0xFFFFu), acc[2 * q]);
+          acc[2 * q + 1] = fma16<BF>(a, (unsigned short)(wv[q] >> 16), acc[2 * q + 1]);
+        }
+      }
+    }
+#else
     for (int base = 0; base < g.len; base += LPR) {
       const int cnt_ = min(LPR, g.len - base);
       int32_t c = 0;
@@ -105,6 +183,7 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
         }
       }
     }
+#endif
     if (early_y) {
       y0.x += acc[0]; y0.y += acc[1]; y0.z += acc[2]; y0.w += acc[3];
       y1.x += acc[4]; y1.y += acc[5]; y1.z += acc[6]; y1.w += acc[7];
@@ -145,7 +224,6 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
           acc[4] += pb[u].x; acc[5] += pb[u].y; acc[6] += pb[u].z; acc[7] += pb[u].w;
         }
       }
-      if (li == 0) cnt[g.split_id] = 0;  // ready for the next launch
     }
     if (f < F) {
       if (vec_y) {
@@ -222,6 +300,16 @@ nm_status check_spmm_args(const nm_packed* P, const void* PX, int64_t ldx, float
 
 }  // namespace
 
+// Tensor-core part: the full-record kernel (spmm_full_sm100.cu) or the compressed-record one
+// (spmm_sm100.cu).  format 0 = the pack's choice (nm_packed::sptc_format), 1 = full,
+// 2 = compressed.
+nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
+                           cudaStream_t s, int format) {
+  if (format == 0) format = P->sptc_format;
+  if (format == 2) return launch_spmm_sptc_compressed(P, PX, ldx, Yp, ldy, F, s);
+  return launch_spmm_sptc_full(P, PX, ldx, Yp, ldy, F, s);
+}
+
 nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
                                cudaStream_t s) {
   const int64_t rows = P->row_end - P->row_begin;
@@ -233,10 +321,37 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
   const int sub_per_warp = 32 / lpr;
   int64_t g = (P->n_res_segs + 8 * sub_per_warp - 1) / (8 * sub_per_warp);
   if (g > 148 * 16) g = 148 * 16;
-#define NM_RES_LAUNCH(BF, LPR)                                                                            \
-  k_residual<BF, LPR><<<(unsigned)g, 256, 0, s>>>(P->res_segs, P->n_res_segs, rcol, P->res_val, \
-                                                  (const uint16_t*)PX, ldx, Yp, ldy, F, f_base, P->res_ws,      \
-                                                  P->res_cnt)
+  // this call's split-row workspace: partial-sum slots + arrival counters (one set per slab
+  // launch, so the counters need no reset between the launches of one call)
+  const int nslab = (F + lpr * 8 - 1) / (lpr * 8);
+  float* ws = nullptr;
+  int32_t* cnt = nullptr;
+  if (P->n_res_split > 0) {
+    NM_CUDA(cudaMallocAsync((void**)&ws, sizeof(float) * kResSlab * P->n_res_slots, s));
+    cudaError_t e = cudaMallocAsync((void**)&cnt, sizeof(int32_t) * P->n_res_split * nslab, s);
+    if (e != cudaSuccess) {
+      cudaFreeAsync(ws, s);
+      return cuda_fail(e, "cudaMallocAsync(residual counters)");
+    }
+    e = cudaMemsetAsync(cnt, 0, sizeof(int32_t) * P->n_res_split * nslab, s);
+    if (e != cudaSuccess) {
+      cudaFreeAsync(ws, s);
+      cudaFreeAsync(cnt, s);
+      return cuda_fail(e, "cudaMemsetAsync(residual counters)");
+    }
+  }
+#define NM_RES_LAUNCH(BF, LPR)                                                                              \
+  do {                                                                                                      \
+    static bool attr_set = false;                                                                           \
+    if (!attr_set && res_smem_bytes<LPR>() > 48 * 1024) {                                                   \
+      cudaFuncSetAttribute(k_residual<BF, LPR>, cudaFuncAttributeMaxDynamicSharedMemorySize,                \
+                           res_smem_bytes<LPR>());                                                          \
+      attr_set = true;                                                                                      \
+    }                                                                                                       \
+    k_residual<BF, LPR><<<(unsigned)g, 256, res_smem_bytes<LPR>(), s>>>(                                    \
+        P->res_segs, P->n_res_segs, rcol, P->res_val, (const uint16_t*)PX, ldx, Yp, ldy, F, f_base, ws,     \
+        cnt ? cnt + P->n_res_split * (f_base / (lpr * 8)) : nullptr);                                       \
+  } while (0)
   for (int f_base = 0; f_base < F; f_base += lpr * 8) {
     switch (lpr * 2 + bf) {
       case 8: NM_RES_LAUNCH(0, 4); break;
@@ -250,7 +365,10 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
     }
   }
 #undef NM_RES_LAUNCH
-  NM_CUDA(cudaGetLastError());
+  const cudaError_t le = cudaGetLastError();
+  if (ws) cudaFreeAsync(ws, s);
+  if (cnt) cudaFreeAsync(cnt, s);
+  if (le != cudaSuccess) return cuda_fail(le, "k_residual launch");
   return NM_OK;
 }
 
@@ -274,7 +392,15 @@ nm_status nm_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Y
                        void* stream) {
   nm_status st = check_spmm_args(P, PX, ldx, Yp, ldy, F);
   if (st != NM_OK) return st;
-  return launch_spmm_sptc(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream);
+  return launch_spmm_sptc(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream, 0);
+}
+
+nm_status nm_spmm_sptc_format(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
+                              int format, void* stream) {
+  nm_status st = check_spmm_args(P, PX, ldx, Yp, ldy, F);
+  if (st != NM_OK) return st;
+  if (format < 0 || format > 2) return fail(NM_ERR_INVALID_ARG, "nm_spmm_sptc_format: format must be 0, 1 or 2");
+  return launch_spmm_sptc(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream, format);
 }
 
 nm_status nm_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
@@ -288,7 +414,7 @@ nm_status nm_spmm(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, in
                   void* stream) {
   nm_status st = check_spmm_args(P, PX, ldx, Yp, ldy, F);
   if (st != NM_OK) return st;
-  st = launch_spmm_sptc(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream);
+  st = launch_spmm_sptc(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream, 0);
   if (st != NM_OK) return st;
   return launch_spmm_residual(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream);
 }

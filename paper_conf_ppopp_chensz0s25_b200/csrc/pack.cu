@@ -541,6 +541,41 @@ __global__ void k_map(const int32_t* __restrict__ perm, int32_t* __restrict__ a,
   }
 }
 
+// Contiguous split of P panels into G ranges minimising the largest range cost, cost of panel r
+// = its chunks + per_panel (linear partition: bisection on the bound, greedy feasibility).
+// Returns G+1 boundaries (trailing ranges may be empty).
+std::vector<int32_t> balanced_ranges(const std::vector<int64_t>& chp, int64_t P, int G, int64_t per_panel) {
+  auto cost = [&](int64_t r) { return chp[r + 1] - chp[r] + per_panel; };
+  auto cuts_for = [&](int64_t T, std::vector<int32_t>* out) {
+    int used = 1;
+    int64_t acc = 0;
+    if (out) out->assign(1, 0);
+    for (int64_t r = 0; r < P; ++r) {
+      const int64_t c = cost(r);
+      if (acc + c > T && acc > 0) {
+        ++used;
+        acc = 0;
+        if (out) out->push_back((int32_t)r);
+      }
+      acc += c;
+    }
+    return used;
+  };
+  int64_t lo = 0, hi = 0;
+  for (int64_t r = 0; r < P; ++r) {
+    lo = std::max(lo, cost(r));
+    hi += cost(r);
+  }
+  while (lo < hi) {
+    const int64_t mid = lo + (hi - lo) / 2;
+    if (cuts_for(mid, nullptr) <= G) hi = mid; else lo = mid + 1;
+  }
+  std::vector<int32_t> cuts;
+  cuts_for(lo, &cuts);
+  while ((int)cuts.size() < G + 1) cuts.push_back((int32_t)P);
+  return cuts;
+}
+
 nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int M, int Vp,
                     nm_dtype dtype, int64_t rb, int64_t re, int flags, int tau, cudaStream_t s,
                     nm_packed** out) {
@@ -555,8 +590,8 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   const int64_t n = A->n;
   if (n <= 0 || A->nnz < 0) return fail(NM_ERR_INVALID_ARG, "nm_pack: empty graph");
   if (n >= (int64_t)1 << 31) return fail(NM_ERR_UNSUPPORTED, "nm_pack: n >= 2^31");
-  if (rb < 0 || re > n || rb > re || rb % Vp != 0)
-    return fail(NM_ERR_INVALID_ARG, "nm_pack_rows: bad row range (row_begin must be a multiple of Vp)");
+  if (rb < 0 || re > n || rb > re || (rb % Vp != 0 && rb != re))
+    return fail(NM_ERR_INVALID_ARG, "nm_pack_rows: bad row range (row_begin must be a multiple of Vp unless the range is empty)");
   const int Mp = (V == 1) ? 4 : M;
   const int64_t rows = re - rb;
   const int64_t P = (rows + Vp - 1) / Vp;
@@ -726,10 +761,10 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
 
   NM_TRY(palloc((void**)&Pk->mb_seg, sizeof(int32_t) * n_mb));
   NM_TRY(palloc((void**)&Pk->mb_sel, sizeof(uint32_t) * n_mb));
-  // the full MMA-layout records are assembled in a scratch buffer, then compressed (step 5)
-  DevBuf d_full;
-  NM_TRY(dalloc(d_full, (size_t)kChunkBytes * n_chunks, s));
-  uint8_t* full = d_full.as<uint8_t>();
+  // the full MMA-layout records (the image of the full-record SpMM kernel); step 5 also
+  // compresses them into the HBM form of the compressed-record kernel
+  NM_TRY(palloc((void**)&Pk->image_full, (size_t)kChunkBytes * n_chunks));
+  uint8_t* full = Pk->image_full;
   if (n_chunks) {
     NM_CUDA(cudaMemsetAsync(full, 0, (size_t)kChunkBytes * n_chunks, s));
     k_meta_init<<<grid_for(n_chunks * 128, 256), 256, 0, s>>>(full, n_chunks);
@@ -773,7 +808,7 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
                                                        Pk->res_rowptr, Pk->res_col, Pk->res_val);
   NM_CUDA(cudaGetLastError());
   if (res_nnz) {
-    // residual work list (kResSeg-entry segments) + the split rows' workspace
+    // residual work list: one item per row, hub rows cut into kResSeg-entry items
     DevBuf d_nseg, d_nslot, d_nsplit, d_segp, d_slotp, d_splitp;
     for (DevBuf* b : {&d_nseg, &d_nslot, &d_nsplit, &d_segp, &d_slotp, &d_splitp})
       NM_TRY(dalloc(*b, sizeof(int64_t) * (rows + 1), s));
@@ -794,9 +829,6 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     Pk->n_res_slots = tot[1];
     Pk->n_res_split = tot[2];
     NM_TRY(palloc((void**)&Pk->res_segs, sizeof(ResSeg) * tot[0]));
-    NM_TRY(palloc((void**)&Pk->res_ws, sizeof(float) * kResSlab * tot[1]));
-    NM_TRY(palloc((void**)&Pk->res_cnt, sizeof(int32_t) * tot[2]));
-    NM_CUDA(cudaMemsetAsync(Pk->res_cnt, 0, sizeof(int32_t) * (tot[2] > 0 ? tot[2] : 1), s));
     DevBuf d_segs, d_k1, d_k2, d_i1, d_i2;
     NM_TRY(dalloc(d_segs, sizeof(ResSeg) * tot[0], s));
     k_seg_fill<<<grid_for(rows, 256), 256, 0, s>>>(Pk->res_rowptr, rows, d_segp.as<int64_t>(), d_slotp.as<int64_t>(),
@@ -887,6 +919,18 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     NM_CUDA(cudaStreamSynchronize(s));
   }
 
+  // persistent-grid work split of the full-record kernel: one contiguous panel range per SM,
+  // balanced by chunk count (+ a per-panel term for its epilogue)
+  {
+    int sms = 148;
+    NM_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, Pk->device));
+    const int G = (int)std::max<int64_t>(1, std::min<int64_t>(sms, P));
+    std::vector<int32_t> cp = balanced_ranges(chp, P, G, /*per_panel=*/4);
+    Pk->n_ctas = G;
+    NM_TRY(palloc((void**)&Pk->cta_ptr, sizeof(int32_t) * cp.size()));
+    NM_CUDA(cudaMemcpyAsync(Pk->cta_ptr, cp.data(), sizeof(int32_t) * cp.size(), cudaMemcpyHostToDevice, s));
+  }
+
   NM_CUDA(cudaStreamSynchronize(s));
   guard.ok = true;
   *out = Pk;
@@ -899,25 +943,25 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
 extern "C" nm_status nm_pack(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
                              nm_dtype dtype, void* stream, nm_packed** out) {
   if (!A) return nm::fail(NM_ERR_INVALID_ARG, "nm_pack: NULL graph");
-  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, 0, A->n, 0, 0, (cudaStream_t)stream, out);
+  return nm::guarded("nm_pack", [&] { return nm::pack_impl(A, perm, V, N, M, Vp, dtype, 0, A->n, 0, 0, (cudaStream_t)stream, out); });
 }
 
 extern "C" nm_status nm_pack_rows(const nm_csr* A, const int32_t* perm, int V, int N, int M,
                                   int Vp, nm_dtype dtype, int64_t row_begin, int64_t row_end,
                                   void* stream, nm_packed** out) {
-  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, 0, 0, (cudaStream_t)stream, out);
+  return nm::guarded("nm_pack", [&] { return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, 0, 0, (cudaStream_t)stream, out); });
 }
 
 extern "C" nm_status nm_pack_ex(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
                                 nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags, void* stream,
                                 nm_packed** out) {
   if (flags & ~NM_PACK_ORIGINAL_ORDER) return nm::fail(NM_ERR_INVALID_ARG, "nm_pack_ex: unknown flags");
-  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, flags, 0, (cudaStream_t)stream, out);
+  return nm::guarded("nm_pack", [&] { return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, flags, 0, (cudaStream_t)stream, out); });
 }
 
 extern "C" nm_status nm_pack_hybrid(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
                                     nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags, int tau,
                                     void* stream, nm_packed** out) {
   if (flags & ~NM_PACK_ORIGINAL_ORDER) return nm::fail(NM_ERR_INVALID_ARG, "nm_pack_hybrid: unknown flags");
-  return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, flags, tau, (cudaStream_t)stream, out);
+  return nm::guarded("nm_pack", [&] { return nm::pack_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, flags, tau, (cudaStream_t)stream, out); });
 }

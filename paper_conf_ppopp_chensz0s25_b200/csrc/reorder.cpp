@@ -565,8 +565,8 @@ nm_status check_graph_arg(const nm_csr* A) {
 }  // namespace
 }  // namespace nm
 
-extern "C" nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
-                                int32_t* perm_out, nm_reorder_stats* st) {
+static nm_status reorder_host_impl(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
+                                   int32_t* perm_out, nm_reorder_stats* st) {
   if (!A || !perm_out) return fail(NM_ERR_INVALID_ARG, "nm_reorder: NULL argument");
   if (V < 1 || N < 1 || M <= N) return fail(NM_ERR_INVALID_ARG, "nm_reorder: need V >= 1, 1 <= N < M");
   if (M > 32) return fail(NM_ERR_UNSUPPORTED, "nm_reorder: M > 32");
@@ -581,8 +581,8 @@ extern "C" nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_r
   return reorder_core(hg.g, be, V, N, M, o, perm_out, st);
 }
 
-extern "C" nm_status nm_reorder_gpu(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
-                                    int32_t* perm_out, nm_reorder_stats* st, void* stream) {
+static nm_status reorder_gpu_impl(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
+                                  int32_t* perm_out, nm_reorder_stats* st, void* stream) {
   if (!A || !perm_out) return fail(NM_ERR_INVALID_ARG, "nm_reorder_gpu: NULL argument");
   if (V < 1 || N < 1 || M <= N) return fail(NM_ERR_INVALID_ARG, "nm_reorder_gpu: need V >= 1, 1 <= N < M");
   if (M > 32) return fail(NM_ERR_UNSUPPORTED, "nm_reorder_gpu: M > 32");
@@ -599,27 +599,22 @@ extern "C" nm_status nm_reorder_gpu(const nm_csr* A, int V, int N, int M, const 
   pattern.val = nullptr;  // the reorder needs the pattern only
   s = upload_csr(&pattern, NM_F16, &d, cs);
   if (s != NM_OK) return s;
-  // the per-iteration scratch of Stage-1 and the counts comes from the device's default
-  // stream-ordered pool: keep it reserved between iterations, give it back at the end
+  // the per-iteration scratch of Stage-1 and the counts comes from a private stream-ordered
+  // pool, kept reserved between iterations and destroyed at the end of the call
   int dev = 0;
-  cudaMemPool_t pool;
   NM_CUDA(cudaGetDevice(&dev));
-  NM_CUDA(cudaDeviceGetDefaultMemPool(&pool, dev));
-  uint64_t keep = UINT64_MAX, thr0 = 0;
-  NM_CUDA(cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr0));
-  NM_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep));
+  ScopedPool pool;
+  NM_TRY(pool.init(dev));
   {
     DeviceBackend be(d, cs);
     s = reorder_core(hg.g, be, V, N, M, o, perm_out, st);
   }
   cudaStreamSynchronize(cs);
-  cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr0);
-  cudaMemPoolTrimTo(pool, 0);
   return s;
 }
 
-extern "C" nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, const nm_reorder_opts* opts,
-                                       int32_t* perm_out, int* V_out, int* M_out, nm_reorder_stats* st) {
+static nm_status select_pattern_impl(const nm_csr* A, int max_M, int max_V, const nm_reorder_opts* opts,
+                                     int32_t* perm_out, int* V_out, int* M_out, nm_reorder_stats* st) {
   if (!A || !perm_out || !V_out || !M_out) return fail(NM_ERR_INVALID_ARG, "nm_select_pattern: NULL argument");
   if (max_M < 4 || max_M > 32 || max_V < 1) return fail(NM_ERR_INVALID_ARG, "nm_select_pattern: need 4 <= max_M <= 32, max_V >= 1");
   nm_status s = check_graph_arg(A);
@@ -658,4 +653,20 @@ extern "C" nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, co
   *V_out = bestV;
   *M_out = bestM;
   return NM_OK;
+}
+
+extern "C" nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
+                                int32_t* perm_out, nm_reorder_stats* st) {
+  return guarded("nm_reorder", [&] { return reorder_host_impl(A, V, N, M, opts, perm_out, st); });
+}
+
+extern "C" nm_status nm_reorder_gpu(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
+                                    int32_t* perm_out, nm_reorder_stats* st, void* stream) {
+  return guarded("nm_reorder_gpu", [&] { return reorder_gpu_impl(A, V, N, M, opts, perm_out, st, stream); });
+}
+
+extern "C" nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, const nm_reorder_opts* opts,
+                                       int32_t* perm_out, int* V_out, int* M_out, nm_reorder_stats* st) {
+  return guarded("nm_select_pattern",
+                 [&] { return select_pattern_impl(A, max_M, max_V, opts, perm_out, V_out, M_out, st); });
 }

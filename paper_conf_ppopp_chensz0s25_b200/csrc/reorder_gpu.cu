@@ -10,11 +10,9 @@
 //      contiguous run of at most M entries, ascending in segment inside each row;
 //   2. one thread per group start folds the run into its mask and count, and emits (x, c);
 //   3. per-row group offsets (count + scan);
-//   4. merge sort (thrust::stable_sort) of the row indices with a comparator that walks two
+//   4. merge sort (cub::DeviceMergeSort::StableSortKeys) of the row indices with a comparator that walks two
 //      rows' pair sequences — stability gives the "ties keep the current position" rule.
 #include <cub/cub.cuh>
-#include <thrust/execution_policy.h>
-#include <thrust/sort.h>
 
 #include "nm_internal.h"
 
@@ -112,6 +110,11 @@ struct RowKeyLess {
   }
 };
 
+__global__ void k_s1_iota(int32_t* __restrict__ a, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    a[i] = (int32_t)i;
+}
+
 template <typename T>
 struct DBuf {
   // stream-ordered pool allocations: the reorder calls these once per Stage-1 iteration
@@ -120,8 +123,7 @@ struct DBuf {
   ~DBuf() { if (p) cudaFreeAsync(p, st); }
   nm_status alloc(size_t n, cudaStream_t s) {
     st = s;
-    NM_CUDA(cudaMallocAsync(&p, sizeof(T) * (n > 0 ? n : 1), s));
-    return NM_OK;
+    return scratch_alloc((void**)&p, sizeof(T) * (n > 0 ? n : 1), s);
   }
 };
 
@@ -189,8 +191,11 @@ nm_status stage1_sort_dev(const DevCsr& A, int32_t* perm_dev, int N, int M, cuda
   if ((st = with_temp([&](void* t, size_t& b) { return cub::DeviceScan::ExclusiveSum(t, b, np_, go, n + 1, s); }, s)))
     return st;
   NM_CUDA(cudaGetLastError());
-  thrust::sequence(thrust::cuda::par.on(s), order.p, order.p + n, 0);
-  thrust::stable_sort(thrust::cuda::par.on(s), order.p, order.p + n, RowKeyLess{goff.p, gx.p, gc.p});
+  k_s1_iota<<<grid_for(n, B), B, 0, s>>>(order.p, n);
+  int32_t* op = order.p;
+  const RowKeyLess less{goff.p, gx.p, gc.p};
+  if ((st = with_temp([&](void* t, size_t& b) { return cub::DeviceMergeSort::StableSortKeys(t, b, op, n, less, s); }, s)))
+    return st;
   k_s1_apply<<<grid_for(n, B), B, 0, s>>>(perm_dev, order.p, n, nperm.p);
   NM_CUDA(cudaMemcpyAsync(perm_dev, nperm.p, sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
   NM_CUDA(cudaGetLastError());

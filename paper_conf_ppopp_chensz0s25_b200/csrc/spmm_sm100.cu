@@ -93,6 +93,14 @@ struct SpmmParams {
   unsigned long long* trace;  // NM_SPMM_TRACE: per-chunk clock64 timeline of CTA 0
 };
 
+// profiling switches (NM_SPMM_DEBUG, results invalid): compiled in only with
+// -DNM_SPMM_DEBUG_BUILD (NM_NVCC_FLAGS); the product kernel reads no switch and skips nothing
+#ifdef NM_SPMM_DEBUG_BUILD
+#define NM_DBG(p) ((p).debug)
+#else
+#define NM_DBG(p) 0
+#endif
+
 // clock64 timeline of CTA 0 (tools/trace_spmm.py): compiled in only with -DNM_SPMM_TRACE_BUILD
 // (NM_NVCC_FLAGS), so the product kernel carries no trace instructions
 #ifdef NM_SPMM_TRACE_BUILD
@@ -326,7 +334,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
     int nsb = 0;                       // sub-batch counter (trace only)
     auto prefetch_unit = [&](int4 b) {  // the records of a panel are contiguous: one L2 prefetch
       const int64_t len = lo_hi(b.z, b.w);
-      if (lane == 0 && len > 0 && !(p.debug & 512))
+      if (lane == 0 && len > 0 && !(NM_DBG(p) & 512))
         asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p.image + lo_hi(b.x, b.y)),
                      "r"((uint32_t)len)
                      : "memory");
@@ -356,7 +364,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
       const int nch = cur.y;
       int64_t boff = lo_hi(curb.x, curb.y);
       uint32_t blen = 0;  // sizes of the next batch of 32 records of this unit, one batch ahead
-      for (int b0 = 0; b0 < ((p.debug & 1024) ? 0 : nch); b0 += 32) {
+      for (int b0 = 0; b0 < ((NM_DBG(p) & 1024) ? 0 : nch); b0 += 32) {
         const int cnt = min(32, nch - b0);
         if (b0 > 0) len = blen;
         if (b0 + 32 < nch) blen = lane < nch - b0 - 32 ? 16u * __ldg(p.rec_len16 + c0 + b0 + 32 + lane) : 0u;
@@ -485,12 +493,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
         const uint32_t rph = (uint32_t)(li >> kSlotsShift) & 1u;
         mbar_wait(bEmpty + 8 * s, ph ^ 1);       // the MMA has finished with stage s
         if (t == 0) NM_TRACE(7);
-        if (!(p.debug & 1024)) mbar_wait(bRecFull + 8 * rs, rph);  // the compressed record has landed
+        if (!(NM_DBG(p) & 1024)) mbar_wait(bRecFull + 8 * rs, rph);  // the compressed record has landed
         if (t == 0) NM_TRACE(1);
-        const uint32_t rec = sRec + pw * C::kRingStride + ((p.debug & 1024) ? 0u : rec_off[rs]);
+        const uint32_t rec = sRec + pw * C::kRingStride + ((NM_DBG(p) & 1024) ? 0u : rec_off[rs]);
         // 8-row groups of consecutive X rows come in by TMA tile loads (one 8 x 64 box per
         // 64-column slab, written into the SW128 atom); the other rows by cp.async gathers
-        const uint32_t cmask = (p.debug & 32) ? 0u : lds8(rec + kRecContOff);
+        const uint32_t cmask = (NM_DBG(p) & 32) ? 0u : lds8(rec + kRecContOff);
         if (t < 32 && cmask) {  // first warp of the group: one TMA tile load per lane
           constexpr int kSlabs = BN / 64;
           if (t == 0)
@@ -515,7 +523,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
           // BN = 64 / 128 / 256: the thread's column piece is the same for every q, so the
           // source column, byte count and swizzle term are per-unit constants
           const uint32_t sbase = sB + s * C::kBBytes + dcol16;
-          if (p.debug & 128) {
+          if (NM_DBG(p) & 128) {
             // profiling: no gathers
           } else if (colbytes == 16u) {  // unit-uniform: full pieces, a zero row is an ignore-src zero fill
 #pragma unroll
@@ -560,7 +568,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
         if (t == 0) NM_TRACE(4);
         // expand row r of the record (its non-empty (row, group) value pairs and nibble word)
         // into the A tile and the stage's TMEM metadata column
-        const uint32_t mask = (p.debug & 64) ? 0u : lds8(rec + kRecMaskOff + r);
+        const uint32_t mask = (NM_DBG(p) & 64) ? 0u : lds8(rec + kRecMaskOff + r);
         const int ne = __popc(mask), nr = mask != 0u;
         // inclusive prefix sums over the quarter's 32 rows from ballots (no shuffle chain):
         // ne = sum of its bits 2^k, each bit's prefix is a popc of the ballot below this lane
@@ -636,7 +644,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
         // the A tile (st.shared) and the gathers (cp.async) were written through the generic
         // proxy: make them visible to the tensor core's async-proxy operand reads (without
         // this fence stale stage contents were observed on B200 -- test_parity_fullsize.py)
-        if (!(p.debug & 16)) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        if (!(NM_DBG(p) & 16)) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         // metadata column: even column address + sparse_id2 selects the odd one
         asm volatile(
@@ -737,7 +745,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm_sptc(const SpmmParams p, c
 #pragma unroll
             for (int j = 0; j < 32; ++j) v[j] = 0u;
           }
-          if (p.debug & 2) continue;
+          if (NM_DBG(p) & 2) continue;
           if (full_tile) {  // unit-uniform fast path: every column in range, 8-byte stores
             float* ylo = p.Y + olo * p.ldy + ft * BN + cc + cpair;
             float* yhi = p.Y + ohi * p.ldy + ft * BN + cc + cpair;
@@ -828,10 +836,16 @@ nm_status launch_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, 
   if (prm.n_units + 4 * (int64_t)sms >= ((int64_t)1 << 31))
     return fail(NM_ERR_UNSUPPORTED, "nm_spmm: too many work units for one launch (row-shard the matrix)");
   prm.idesc = make_idesc(P->dtype, BN);
+  prm.debug = 0;
+  prm.trace = nullptr;
+  const char* tr = nullptr;
+#ifdef NM_SPMM_DEBUG_BUILD
   const char* dbg = getenv("NM_SPMM_DEBUG");
   prm.debug = dbg ? atoi(dbg) : 0;
-  prm.trace = nullptr;
-  const char* tr = getenv("NM_SPMM_TRACE");
+#endif
+#ifdef NM_SPMM_TRACE_BUILD
+  tr = getenv("NM_SPMM_TRACE");
+#endif
   if (tr) {
     NM_CUDA(cudaMalloc(&prm.trace, 16384 * 8));
     NM_CUDA(cudaMemset(prm.trace, 0, 16384 * 8));
@@ -873,8 +887,8 @@ nm_status launch_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, 
 
 }  // namespace
 
-nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
-                           cudaStream_t s) {
+nm_status launch_spmm_sptc_compressed(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy,
+                                      int F, cudaStream_t s) {
   if (F <= 64) return launch_bn<64>(P, PX, ldx, Yp, ldy, F, s);
   if (F <= 128) return launch_bn<128>(P, PX, ldx, Yp, ldy, F, s);
   if (F <= 192) return launch_bn<192>(P, PX, ldx, Yp, ldy, F, s);

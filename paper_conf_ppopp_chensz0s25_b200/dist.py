@@ -10,8 +10,10 @@
 * ``gcn_forward``: a K-layer GCN forward (Eq. 1) in the permuted vertex order with
   X replicated: per layer each rank computes its row block of Ahat (H W) with libnm
   (nm_gcn_layer) and the next layer's full operand is assembled with one NCCL
-  ``all_gather_into_tensor`` over NVLink.  Shards are padded to equal row counts so the
-  collective needs no reshuffle; padding rows are dropped after the gather.
+  ``all_gather_into_tensor`` over NVLink (in place: each rank's block of the receive buffer
+  is its send buffer).  Shards are padded to equal row counts so the collective needs no
+  reshuffle; with equal shards the padding sits at the end and the gathered buffer is used
+  as is, otherwise the padding rows are dropped after the gather.
 * ``local_layer`` is injectable so the host-side logic (sharding, padding, collective order)
   is testable with the ``gloo`` backend on CPU (tests/test_dist.py).
 """
@@ -106,13 +108,14 @@ def gcn_forward(H, layers, local_layer, group=None, bounds=None):
             cur = out_loc
             continue
         f = out_loc.shape[1]
-        send = torch.zeros((rows_pad, f), dtype=out_loc.dtype, device=out_loc.device)
-        send[: re - rb] = out_loc
         full = torch.empty((rows_pad * world, f), dtype=out_loc.dtype, device=out_loc.device)
-        dist.all_gather_into_tensor(full, send, group=group)
-        # drop each rank's padding rows
-        parts = []
-        for r, (a, b) in enumerate(bounds):
-            parts.append(full[r * rows_pad: r * rows_pad + (b - a)])
-        cur = torch.cat(parts, dim=0)
+        mine = full[rank * rows_pad: (rank + 1) * rows_pad]  # in-place all-gather: send = own block
+        mine[: re - rb] = out_loc
+        if re - rb < rows_pad:
+            mine[re - rb:].zero_()
+        dist.all_gather_into_tensor(full, mine, group=group)
+        if all(b - a == rows_pad for a, b in bounds[:-1]):
+            cur = full[:n]  # equal shards: the padding is all at the end, no copy
+        else:  # drop each rank's padding rows
+            cur = torch.cat([full[r * rows_pad: r * rows_pad + (b - a)] for r, (a, b) in enumerate(bounds)], dim=0)
     return cur

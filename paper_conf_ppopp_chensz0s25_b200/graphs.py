@@ -42,11 +42,35 @@ def _symmetric_csr(n: int, a: np.ndarray, b: np.ndarray, self_loops: bool = Fals
     return _csr_from_pairs(n, u, v)
 
 
+def _sorted_unique(x: np.ndarray) -> np.ndarray:
+    """np.unique(x) for 1-D int64 (sorted distinct values) via sort + mask: numpy 2.x's
+    np.unique/union1d take minutes at the C3-C5 sizes (~10^8 keys), np.sort seconds."""
+    s = np.sort(x)
+    if s.size == 0:
+        return s
+    keep = np.empty(s.size, bool)
+    keep[0] = True
+    np.not_equal(s[1:], s[:-1], out=keep[1:])
+    return s[keep]
+
+
+def _union(a: np.ndarray, b: np.ndarray) -> np.ndarray:
+    return _sorted_unique(np.concatenate([a, b]))
+
+
+def _searchsorted_right(cum: np.ndarray, q: np.ndarray) -> np.ndarray:
+    """np.searchsorted(cum, q, side='right') (exact float64 comparisons, identical result);
+    torch's CPU kernel is ~10x faster on 10^8 unsorted queries."""
+    import torch
+    return torch.searchsorted(torch.from_numpy(np.ascontiguousarray(cum)),
+                              torch.from_numpy(np.ascontiguousarray(q)), right=True).numpy()
+
+
 def _unique_pairs(a: np.ndarray, b: np.ndarray, n: int):
     lo = np.minimum(a, b).astype(np.int64)
     hi = np.maximum(a, b).astype(np.int64)
     keep = lo != hi
-    key = np.unique(lo[keep] * n + hi[keep])
+    key = _sorted_unique(lo[keep] * n + hi[keep])
     return key
 
 
@@ -58,7 +82,7 @@ def er_graph(n: int, m: int, seed: int, self_loops: bool = False):
         k = int((m - key.size) * 1.2) + 16
         a = rng.integers(0, n, k)
         b = rng.integers(0, n, k)
-        key = np.union1d(key, _unique_pairs(a, b, n))
+        key = _union(key, _unique_pairs(a, b, n))
     key = key[np.sort(rng.permutation(key.size)[:m])]
     return _symmetric_csr(n, key // n, key % n, self_loops)
 
@@ -91,7 +115,7 @@ def lmcl_graph(n: int, m: int, gamma: float, C: int, rho: float, seed: int,
     key = np.empty(0, np.int64)
     while key.size < m:
         k = int((m - key.size) * 1.3) + 1024
-        u = np.searchsorted(cum, rng.random(k) * total, side="right") - 1
+        u = _searchsorted_right(cum, rng.random(k) * total) - 1
         u = np.clip(u, 0, n - 1)
         local = rng.random(k) < rho
         cu = comm_of[u]
@@ -99,8 +123,8 @@ def lmcl_graph(n: int, m: int, gamma: float, C: int, rho: float, seed: int,
         hi = cum[bounds[cu + 1]]
         r = rng.random(k)
         tgt = np.where(local, lo + r * (hi - lo), r * total)
-        v = np.clip(np.searchsorted(cum, tgt, side="right") - 1, 0, n - 1)
-        key = np.union1d(key, _unique_pairs(u, v, n))
+        v = np.clip(_searchsorted_right(cum, tgt) - 1, 0, n - 1)
+        key = _union(key, _unique_pairs(u, v, n))
     key = key[np.sort(rng.permutation(key.size)[:m])]
     a, b = key // n, key % n
     if scramble:
@@ -122,7 +146,7 @@ def banded_graph(n: int, d: int, seed: int, self_loops: bool = False):
         i = rng.integers(0, n, k)
         j = i + rng.integers(1, 4 * d + 1, k)
         ok = j < n
-        key = np.union1d(key, _unique_pairs(i[ok], j[ok], n))
+        key = _union(key, _unique_pairs(i[ok], j[ok], n))
     key = key[np.sort(rng.permutation(key.size)[:m])]
     return _symmetric_csr(n, key // n, key % n, self_loops)
 
@@ -201,3 +225,35 @@ def features(n: int, F: int, seed: int, dist: str = "uniform"):
     if dist == "uniform":
         return (rng.random((n, F), dtype=np.float32) * 2.0 - 1.0)
     return rng.standard_normal((n, F), dtype=np.float32)
+
+
+# ---------------------------------------------------------------- GNN-shaped graphs (C3-C5)
+# Shapes from the paper's Table 2: n and directed edge counts are the
+# datasets'; gamma, community count and rho are assumptions, natural order
+# (contiguous communities), self-loops added as GCN's A + I (Eq. 1; reading #22).
+
+GNN_SHAPES = {
+    # name: (n, undirected edges m, gamma, communities, rho)
+    "reddit": (232_965, 57_400_000, 2.3, 41, 0.6),        # C3: ~114.8M directed (L520)
+    "proteins": (132_534, 39_561_252, 3.0, 8, 0.8),       # C4: 79.12M directed (L521)
+    "products": (2_449_029, 61_859_140, 2.5, 47, 0.7),    # C5: 123.72M directed (L522)
+}
+
+
+def gnn_graph(name: str, scale: int = 1):
+    """Reddit / ogbn-proteins / ogbn-products-shaped graph (C3 / C4 / C5) as a symmetric CSR
+    with self-loops.  scale > 1 divides n and m by that factor (test-sized replicas with the
+    same average degree, degree-distribution family and community structure)."""
+    n, m, gamma, C, rho = GNN_SHAPES[name]
+    n, m = n // scale, m // scale
+    return lmcl_graph(n, m, gamma, C, rho, seed_of(name, n, m), self_loops=True)
+
+
+def gcn_norm_values(indptr, indices):
+    """Values of Ahat = D^-1/2 (A + I) D^-1/2 (GCN, Eq. 1) for a CSR that
+    already holds the self-loops: v_ij = 1/sqrt(d_i d_j), d = row lengths.  float32."""
+    n = len(indptr) - 1
+    deg = np.diff(indptr).astype(np.float64)
+    dinv = np.where(deg > 0, 1.0 / np.sqrt(np.maximum(deg, 1.0)), 0.0)
+    rows = np.repeat(np.arange(n), np.diff(indptr))
+    return (dinv[rows] * dinv[indices]).astype(np.float32)

@@ -1,0 +1,134 @@
+"""The row-partitioned multi-GPU path with the REAL per-rank compute (libnm), two ranks
+sharing cuda:0 over the gloo backend (this environment has one GPU; the product collective
+is NCCL, one rank per GPU):
+
+* dist.gcn_forward with nm_pack_rows + nm_gcn_layer per rank: the world-2 output equals the
+  world-1 output BITWISE (row shards change no arithmetic), for equal and
+  cost-balanced shards, and matches the oracle's fp64 GCN within the GCN bound;
+* bench.py under torch.distributed.run with NM_DIST_BACKEND=gloo, 2 ranks: one JSON line with
+  n_gpus = 2 and a positive value.
+"""
+import json
+import os
+import socket
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _problem():
+    from paper_conf_ppopp_chensz0s25_b200 import graphs
+    n = 3000  # 24 panels, ragged tail (3000 % 128 = 56)
+    ip, ic = graphs.lmcl_graph(n, 40000, 2.3, 4, 0.6, 17, self_loops=True)
+    vals = graphs.gcn_norm_values(ip, ic)
+    rng = np.random.default_rng(1)
+    H = rng.standard_normal((n, 64)).astype(np.float32)
+    Ws = [(rng.standard_normal((64, 64)) / 8).astype(np.float32), (rng.standard_normal((64, 32)) / 8).astype(np.float32)]
+    bs = [(rng.standard_normal(64) * 0.1).astype(np.float32), (rng.standard_normal(32) * 0.1).astype(np.float32)]
+    return ip, ic, vals, H, Ws, bs
+
+
+def _run(world, rank, balanced):
+    """GCN forward (2 layers, bf16, 1:2:4) for this rank; returns the full output (bf16 bits)."""
+    from paper_conf_ppopp_chensz0s25_b200 import api, graphs
+    from paper_conf_ppopp_chensz0s25_b200 import dist as nmdist
+    dev = torch.device("cuda:0")
+    ip, ic, vals, H, Ws, bs = _problem()
+    n = len(ip) - 1
+    perm = np.random.default_rng(3).permutation(n).astype(np.int32)
+    bounds = (nmdist.balanced_bounds(nmdist.panel_costs(ip, perm), n, world) if balanced
+              else [nmdist.shard_rows(n, world, r) for r in range(world)])
+    rb, re = bounds[rank]
+    P = api.pack(ip, ic, perm, 1, 2, 4, dtype="bf16", val=vals, row_begin=rb, row_end=re)
+
+    def bf(a):
+        b, _ = graphs.round16(np.asarray(a, np.float32), "bf16")
+        return torch.from_numpy(b.view(np.int16)).to(dev).view(torch.bfloat16)
+
+    layers = [(bf(W), torch.from_numpy(b).to(dev), relu) for W, b, relu in ((Ws[0], bs[0], True), (Ws[1], bs[1], False))]
+
+    def local_layer(li, Hf, W, b, relu, a, z):
+        Hd = Hf.to(dev).view(torch.bfloat16)
+        out = torch.empty((z - a, W.shape[1]), dtype=torch.bfloat16, device=dev)
+        ws = torch.empty(api.gcn_workspace_bytes(n, W.shape[0], W.shape[1]), dtype=torch.uint8, device=dev)
+        api.gcn_layer(P, Hd, W, b, out, ws, relu=relu, order="linear")
+        torch.cuda.synchronize()
+        return out.view(torch.int16).cpu()  # gloo collectives run on host tensors
+
+    Hp = bf(H[perm]).view(torch.int16).cpu()
+    out = nmdist.gcn_forward(Hp, layers, local_layer, bounds=bounds)
+    return out.numpy().copy(), perm
+
+
+def _worker(rank, world, port, balanced, q):
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    out, _ = _run(world, rank, balanced)
+    q.put((rank, out))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("balanced", [False, True])
+def test_gcn_forward_world2_bitwise_equals_world1(balanced):
+    import torch.multiprocessing as mp
+
+    import oracle
+    from paper_conf_ppopp_chensz0s25_b200 import graphs
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    ref, perm = _run(1, 0, balanced)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, balanced, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    got = dict(q.get(timeout=600) for _ in range(2))
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    for r in range(2):
+        assert np.array_equal(got[r], ref), "rank %d differs from the 1-rank result" % r
+    # and the 1-rank result is a correct GCN (fp64 oracle on the same bf16-rounded inputs;
+    # loose Frobenius bound: two bf16 layers)
+    ip, ic, vals, H, Ws, bs = _problem()
+    _, v64 = graphs.round16(vals, "bf16")
+    h = graphs.round16(H, "bf16")[1]
+    for W, b, relu in ((Ws[0], bs[0], True), (Ws[1], bs[1], False)):
+        h, _ = oracle.gcn_layer(ip, ic, v64, h, graphs.round16(W, "bf16")[1], b, relu)
+    y = np.empty_like(h)
+    y[perm] = graphs.bf16_bits_to_f64(ref.view(np.uint16))
+    assert np.linalg.norm(y - h) <= 2e-2 * np.linalg.norm(h)
+
+
+def test_bench_two_ranks_gloo_on_one_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    env = dict(os.environ, NM_DIST_BACKEND="gloo")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), os.path.join(ROOT, "bench.py"),
+           "--gpus", "2", "--steps", "5", "--warmup", "3", "--workload", "c1-er-n2048-f32-1:2:4"]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, env=env, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["steps"] == 5

@@ -328,3 +328,70 @@ def test_residual_split_hub_rows(F, dtype):
     err = np.abs(outs[0].astype(np.float64) - Y_ref)
     assert (err <= TOL * E).all(), err.max()
     assert all(np.array_equal(outs[0], o) for o in outs[1:])
+
+
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+def test_concurrent_spmm_on_one_handle(dtype):
+    """nm.h "Handles": the packed matrix is immutable after nm_pack, so two nm_spmm calls on
+    the SAME handle on two streams (hub rows split over several residual work items, plus the
+    tensor-core part) must both be right -- repeated many times with the launches interleaved."""
+    dev = _cuda()
+    ip, ic = _star_plus_er(n=6000, hubs=(0, 17, 999), m=18000, seed=52)
+    n = len(ip) - 1
+    F = 128
+    perm = np.random.default_rng(5).permutation(n).astype(np.int32)
+    v32, bits, v64 = _values(ip, ic, dtype, 6)
+    P = api.pack(ip, ic, perm, 1, 2, 4, dtype=dtype, val=v32, order="original", tau=2)
+    st = P.stats()
+    assert st["residual_split_rows"] > 0 and st["n_mb"] > 0
+    tdt = torch.float16 if dtype == "f16" else torch.bfloat16
+    Xs, refs = [], []
+    for seed in (7, 8):
+        xbits, x64 = graphs.round16(graphs.features(n, F, seed), dtype)
+        Xs.append(torch.from_numpy(xbits.view(np.int16)).to(dev).view(tdt))
+        refs.append(oracle.spmm(ip, ic, v64, x64)[:2])
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    Ys = [torch.empty((n, F), device=dev) for _ in range(2)]
+    for it in range(20):
+        for k in (0, 1) if it % 2 == 0 else (1, 0):
+            Ys[k].fill_(float("nan"))
+        torch.cuda.synchronize()
+        for k in (0, 1):
+            api.spmm(P, Xs[k], Ys[k], stream=streams[k])
+        torch.cuda.synchronize()
+        for k in (0, 1):
+            Y_ref, E = refs[k]
+            err = np.abs(Ys[k].cpu().numpy().astype(np.float64) - Y_ref)
+            assert (err <= TOL * E).all(), (it, k, err.max())
+
+
+@pytest.mark.parametrize("kind,seed,V,M", CASES)
+@pytest.mark.parametrize("F", [32, 128, 300])
+def test_sptc_formats_agree_bitwise(kind, seed, V, M, F):
+    """The full-record kernel (format 1, nm_spmm's default) and the compressed-record kernel
+    (format 2) feed the tensor core identical operands in the same order: Yp must agree
+    bitwise, and both must meet the oracle bound."""
+    dev = _cuda()
+    ip, ic = _graph(kind, seed)
+    n = len(ip) - 1
+    perm = np.random.default_rng(seed + 100).permutation(n).astype(np.int32)
+    dtype = "bf16" if seed % 2 else "f16"
+    v32, bits, v64 = _values(ip, ic, dtype, seed)
+    xbits, x64 = graphs.round16(graphs.features(n, F, seed + 1), dtype)
+    tdt = torch.float16 if dtype == "f16" else torch.bfloat16
+    ldx = (F + 7) // 8 * 8
+    Xb = torch.zeros((n, ldx), dtype=torch.int16, device=dev)
+    Xb[:, :F] = torch.from_numpy(xbits.view(np.int16)).to(dev)
+    X = Xb.view(tdt)[:, :F]
+    P = api.pack(ip, ic, perm, V, 2, M, dtype=dtype, val=v32, order="original")
+    outs = []
+    for fmt in (1, 2):
+        Y = torch.full((n, F), float("nan"), device=dev)
+        api.spmm(P, X, Y, part="sptc", format=fmt)
+        api.spmm(P, X, Y, part="residual")
+        torch.cuda.synchronize()
+        outs.append(Y.cpu().numpy())
+    assert np.array_equal(outs[0], outs[1])
+    Y_ref, E, _ = oracle.spmm(ip, ic, v64, x64)
+    err = np.abs(outs[0].astype(np.float64) - Y_ref)
+    assert (err <= TOL * E).all(), err.max()
