@@ -31,20 +31,24 @@ import numpy as np
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+_GNN_RO = dict(max_outer=0, max_stage1=10, max_stage2=0)
 WORKLOADS = {
     # configs[0]: ER n = 2048, m = 16384, F = 32, 2:4, fp16 (oracle-sized correctness case)
     "c1-er-n2048-f32-1:2:4": dict(kind="er", n=2048, m=16384, F=32, V=1, M=4, dtype="f16", tau=0),
     # configs[2]: Reddit-shaped (n 232,965, ~114.8M directed edges + I), GCN aggregation of
     # the 602 -> 128 layer at F = 128, bf16, Ahat sym-normalised (the N = 1 headline)
-    "c3-reddit-f128-1:2:4": dict(kind="gnn", graph="reddit", F=128, V=1, M=4, dtype="bf16", tau=None),
-    "c3-reddit-f128-128:2:16": dict(kind="gnn", graph="reddit", F=128, V=128, M=16, dtype="bf16", tau=None),
+    # (reorder: one Alg. 1 iteration -- Stage-1 sorts + one Stage-2 pass; the full MAXITER = 10
+    # schedule takes tens of minutes at 115M entries with the host Stage-2)
+    "c3-reddit-f128-1:2:4": dict(kind="gnn", graph="reddit", F=128, V=1, M=4, dtype="bf16", tau=None, **_GNN_RO),
+    "c3-reddit-f128-128:2:16": dict(kind="gnn", graph="reddit", F=128, V=128, M=16, dtype="bf16", tau=None,
+                                    **_GNN_RO),
     # configs[3]: ogbn-proteins-shaped (132,534 / 79.12M directed + I), F = 256, 128:2:16
     "c4-proteins-f256-128:2:16": dict(kind="gnn", graph="proteins", F=256, V=128, M=16, dtype="bf16",
-                                      tau=None),
+                                      tau=None, **_GNN_RO),
     # configs[4]: ogbn-products-shaped (2,449,029 / 123.72M directed + I), aggregation at
     # F = 100 (aggregate-first 100 -> 256), 128:2:8
     "c5-products-f100-128:2:8": dict(kind="gnn", graph="products", F=100, V=128, M=8, dtype="bf16",
-                                     tau=None),
+                                     tau=None, **_GNN_RO),
 }
 # configs[1] (SuiteSparse-shaped sweep): any point named
 #   c2-{banded|powerlaw}-n{65k|262k|1m}-d{8|16|32|64}-f{F}-{V}:2:{M}[-tau{T}]
@@ -99,6 +103,34 @@ def make_graph(w):
     vals = graphs.symmetric_values(ip, ic, seed + 1)
     X32 = graphs.features(w["n"], w["F"], seed + 2)
     return ip, ic, vals, X32
+
+
+def l2_gather_peak():
+    """Random 256-byte X-row gathers served by L2, GB/s: tools/probes/probe_gather_rate.cu's best
+    figure on B200 (cp.async.cg 16 B + commit/wait_group, 148 CTAs, L2-resident X), read from its
+    committed output; the fallback is the same measurement's value."""
+    p = os.path.join(ROOT, "tools", "probes", "probe_gather_rate.b200.txt")
+    best = 0.0
+    if os.path.exists(p):
+        import re
+        for ln in open(p):
+            m = re.search(r"X=(\d+)MB\s*:.*?([\d.]+) GB/s", ln)
+            if m and int(m.group(1)) <= 128:  # L2-resident sizes only
+                best = max(best, float(m.group(2)))
+    return (best, "measured (tools/probes/probe_gather_rate.b200.txt)") if best else (18944.0, "fallback")
+
+
+def sparse_peak(bf16_tf):
+    """Sparse (2:4) tensor peak, logical TFLOP/s: tools/probes/probe_sparse_peak.b200.txt if it
+    holds a measurement, else 2x the measured dense bf16 rate (NVIDIA's 2:4 ratio), labelled so."""
+    p = os.path.join(ROOT, "tools", "probes", "probe_sparse_peak.b200.txt")
+    if os.path.exists(p):
+        import re
+        for ln in open(p):
+            m = re.match(r"BEST sparse ([\d.]+) TFLOP/s", ln)
+            if m and float(m.group(1)) > 0:
+                return float(m.group(1)), "measured (tools/probes/probe_sparse_peak.b200.txt)"
+    return 2.0 * bf16_tf, "assumed 2x measured dense bf16"
 
 
 def peaks():
@@ -243,6 +275,9 @@ def main():
     ap.add_argument("--no-cusparse", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--order", default="original", choices=["original", "permuted"])
+    ap.add_argument("--layout", default="auto", choices=["auto", "reordered", "natural"],
+                    help="timed layout: the reorder's, the natural order, or the faster of the two (auto)")
+    ap.add_argument("--no-reorder", action="store_true", help="profiling: skip nm_reorder (natural order)")
     ap.add_argument("--tau", type=int, default=None, help="hybrid threshold (default: the workload's / nm_hybrid_tau)")
     ap.add_argument("--max-outer", type=int, default=None, help="Alg. 1 cap (default: the workload's, else 10, L496)")
     ap.add_argument("--max-stage1", type=int, default=None)
@@ -293,7 +328,12 @@ def main():
     nnz = int(ip[-1])
     # nm_reorder_gpu (untimed preprocessing).  Deterministic: every rank computes the same
     # permutation itself, so no rank waits in a collective while another reorders
-    perm, rst = api.reorder(ip, ic, V, 2, M, device=True, **ropts)
+    if args.no_reorder:  # profiling runs: natural order, no reorder kernels in the launch list
+        perm = np.arange(n, dtype=np.int32)
+        rst = {"omega_init": 0, "omega_final": 0, "mb_init": 0, "mb_final": 0, "seconds": 0.0}
+        args.layout = "reordered"
+    else:
+        perm, rst = api.reorder(ip, ic, V, 2, M, device=True, **ropts)
     # contiguous panel-aligned row blocks balanced by stored entries + Y rows
     from paper_conf_ppopp_chensz0s25_b200.dist import balanced_bounds, panel_costs
     rb, re = balanced_bounds(panel_costs(ip, perm), n, world)[rank]
@@ -302,7 +342,6 @@ def main():
     P = api.pack(ip, ic, perm, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order=args.order, tau=tau)
     torch.cuda.synchronize()
     pack_s = time.perf_counter() - t0
-    info = P.info()
     xbits, _ = graphs.round16(X32, dt)
     tdt = torch.float16 if dt == "f16" else torch.bfloat16
     Fp = (F + 7) // 8 * 8  # rows padded to 16 B (ldx % 8 == 0; C5's F = 100 -> 104 in memory)
@@ -310,10 +349,41 @@ def main():
     Xpad[:, :F] = torch.from_numpy(xbits.view(np.int16)).to(dev)
     X = Xpad.view(tdt)[:, :F]
     Y = torch.empty((n, Fp), dtype=torch.float32, device=dev)[:, :F]
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+    # layout choice (offline, like picking a cuSPARSE algorithm): the reorder's layout vs the
+    # natural order, each packed and timed for a few L2-flushed steps; the faster one is timed
+    layout_trial = None
+    if args.layout == "auto" and args.order == "original":
+        P_nat = api.pack(ip, ic, None, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order="original", tau=tau)
+        trial = {}
+        for name, Pk in (("reordered", P), ("natural", P_nat)):
+            for _ in range(3):
+                api.spmm(Pk, X, Y)
+            ts = []
+            for _ in range(8):
+                flush.zero_()
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record()
+                api.spmm(Pk, X, Y)
+                b.record()
+                ts.append((a, b))
+            torch.cuda.synchronize()
+            t = torch.tensor([statistics.median(x.elapsed_time(y) for x, y in ts)], dtype=torch.float64, device=cdev)
+            if world > 1:
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            trial[name] = float(t.item())
+        layout_trial = dict(trial_ms=trial, chosen=min(trial, key=trial.get))
+        if layout_trial["chosen"] == "natural":
+            P, perm = P_nat, np.arange(n, dtype=np.int32)
+        else:
+            del P_nat
+    elif args.layout == "natural":
+        P = api.pack(ip, ic, None, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order=args.order, tau=tau)
+        perm = np.arange(n, dtype=np.int32)
+    info = P.info()
     perm_d = torch.from_numpy(perm).to(dev)
     PX = padded_like(X) if args.order == "permuted" else None
     Yp = torch.empty((re - rb, F), dtype=torch.float32, device=dev) if args.order == "permuted" else None
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
     stream = torch.cuda.current_stream()
     has_res = info["residual_nnz"] > 0
 
@@ -383,31 +453,52 @@ def main():
     x_rows_res = int(np.count_nonzero(col_res))
     res_rows = int(np.count_nonzero(np.diff(res["res_rowptr"])))
     x_rows = int(np.count_nonzero(col_all))
-    # algorithmic bytes per launch
-    #   k_spmm_sptc: the compressed chunk records it streams (image_bytes: gather rows, row
-    #                masks, non-empty value pairs and nibble words) + X read once + Y written
-    #                once (rows * F * 4 B)
-    #   k_residual : (col, value) 6 B per residual nonzero + row pointers + X read once + the
-    #                read-modify-write of the Y rows it touches (8 F B each)
+    # Roofline terms per kernel, algorithmic bytes / flops per launch:
+    #   k_spmm_sptc: HBM = the chunk records it streams (full records: 4736 B per K = 32 chunk =
+    #                SURVEY §8(d)'s #mb * (Vp * 4.5 + 4) slot formula; compressed: image_bytes)
+    #                + X read once + Y written once (rows * F * 4 B);  L2 = the gathered X rows
+    #                (gather_rows * F * 2 B, served from L2 when X fits) + the records per F tile;
+    #                tensor = one sparse M128 x BN x K32 MMA per chunk and F tile at the sparse peak
+    #   k_residual : HBM = (col, value) 6 B per residual nonzero + row pointers + the Y rows it
+    #                read-modify-writes (8 F B each);  L2 = one gathered X row per nonzero (F * 2 B)
+    # bound = the largest of the terms' times; frac = that time / the measured kernel time.
     pst = P.stats()
-    kern = {"k_spmm_sptc": {"alg_bytes": pst["image_bytes"] + x_rows_sptc * F * 2 + rows_b * F * 4,
-                            "ms": statistics.mean(sptc_ms)}}
+    fmt = args.sptc_format or 1
+    BN = 64 if F <= 64 else (128 if F <= 128 else 256)
+    nft = (F + BN - 1) // BN
+    rec_bytes = pst["full_image_bytes"] if fmt != 2 else pst["image_bytes"]
+    l2_gbs, l2_src = l2_gather_peak()
+    sp_tf, sp_src = sparse_peak(bf16_tf)
+    kern = {"k_spmm_sptc": {"hbm_bytes": rec_bytes + x_rows_sptc * F * 2 + rows_b * F * 4,
+                            "l2_bytes": pst["gather_rows"] * F * 2 + rec_bytes * nft,
+                            "mma_flop": 2.0 * chunks * nft * 128 * BN * 32,
+                            "ms": statistics.mean(sptc_ms), "format": "full" if fmt != 2 else "compressed"}}
     if has_res:
-        kern["k_residual"] = {"alg_bytes": res["res_nnz"] * 6 + (rows_b + 1) * 8 + x_rows_res * F * 2 +
-                                           res_rows * F * 8,
+        kern["k_residual"] = {"hbm_bytes": res["res_nnz"] * 6 + (rows_b + 1) * 8 + res_rows * F * 8,
+                              "l2_bytes": res["res_nnz"] * F * 2, "mma_flop": 0.0,
                               "ms": statistics.mean(b - a for a, b in zip(sptc_ms, step_ms))}
     for k in kern.values():
-        k["achieved_gbs"] = k["alg_bytes"] / (k["ms"] * 1e-3) / 1e9
-        k["frac"] = k["achieved_gbs"] / hbm_gbs
+        t = {"hbm": k["hbm_bytes"] / (hbm_gbs * 1e9) * 1e3, "l2": k["l2_bytes"] / (l2_gbs * 1e9) * 1e3,
+             "tensor": k["mma_flop"] / (sp_tf * 1e12) * 1e3}
+        k["t_roof_ms"] = t
+        k["bound"] = max(t, key=t.get)
+        k["frac"] = t[k["bound"]] / k["ms"]
+        k["hbm_frac"] = t["hbm"] / k["ms"]
     dom = max(kern, key=lambda k: kern[k]["ms"])
-    alg_bytes, k_ms = kern[dom]["alg_bytes"], kern[dom]["ms"]
-    achieved = alg_bytes / (k_ms * 1e-3) / 1e9
-    t_mma_ms = 2.0 * chunks * 128 * max(F, 64) * 32 / (2 * bf16_tf * 1e12) * 1e3  # sparse = 2x dense rate
-    roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_gbs, "unit": "GB/s",
-                "frac": achieved / hbm_gbs, "traffic": None, "peak_source": peak_src,
-                "kernel": dom, "kernel_ms": k_ms, "alg_bytes_per_launch": alg_bytes,
-                "t_hbm_ms": alg_bytes / (hbm_gbs * 1e9) * 1e3, "t_mma_ms_sptc": t_mma_ms,
-                "kernels": kern}
+    kd = kern[dom]
+    k_ms = kd["ms"]
+    if kd["bound"] == "tensor":
+        achieved, peak, unit = kd["mma_flop"] / (k_ms * 1e-3) / 1e12, sp_tf, "TFLOP/s"
+    elif kd["bound"] == "l2":
+        achieved, peak, unit = kd["l2_bytes"] / (k_ms * 1e-3) / 1e9, l2_gbs, "GB/s"
+    else:
+        achieved, peak, unit = kd["hbm_bytes"] / (k_ms * 1e-3) / 1e9, hbm_gbs, "GB/s"
+    roofline = {"bound": kd["bound"], "achieved": achieved, "peak": peak, "unit": unit, "frac": achieved / peak,
+                "traffic": None, "kernel": dom, "kernel_ms": k_ms,
+                "peaks": {"hbm_gbs": hbm_gbs, "hbm_source": peak_src, "l2_gather_gbs": l2_gbs, "l2_source": l2_src,
+                          "sparse_tflops": sp_tf, "sparse_source": sp_src},
+                "kernels": kern,
+                "step_frac": sum(max(k["t_roof_ms"].values()) for k in kern.values()) / ms_per_step}
     prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(prof) and world == 1:  # the committed capture is of the 1-GPU launch
         try:
@@ -451,14 +542,15 @@ def main():
         line = {"metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": dt, "data": "synthetic",
-                "config": {"workload": args.workload, "graph": w["kind"], "n": n, "nnz": nnz, "F": F,
+                "config": {"workload": args.workload, "graph": w.get("graph", w["kind"]), "n": n, "nnz": nnz, "F": F,
+                           "layout": (layout_trial or {}).get("chosen", args.layout),
                            "pattern": "%d:2:%d" % (V, M), "order": args.order, "tau": tau,
                            "parallelism": "row-shard x%d" % world,
                            "l2": "flushed between steps (256 MiB write outside the event-timed intervals)"},
                 "gpu_launches": launches_per_step * args.steps,
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "cusparse": cus,
-                "preprocess": {"gen_s": gen_s, "reorder": "nm_reorder_gpu", "reorder_opts": ropts, "reorder_s": rst["seconds"], "pack_s": pack_s,
+                "preprocess": {"gen_s": gen_s, "reorder": "nm_reorder_gpu", "reorder_opts": ropts, "layout": layout_trial, "reorder_s": rst["seconds"], "pack_s": pack_s,
                                "omega_init": rst["omega_init"], "omega_final": rst["omega_final"],
                                "mb_init": rst["mb_init"], "mb_final": rst["mb_final"],
                                "violation_removal": (None if rst["omega_init"] == 0 else

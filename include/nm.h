@@ -192,12 +192,15 @@ NM_API nm_status nm_packed_info(const nm_packed* P, int64_t* n_mb, int64_t* pack
                          int64_t* residual_nnz, int64_t* device_bytes, int64_t* n_chunks);
 
 /* All sizes of a packed matrix (superset of nm_packed_info).  image_bytes = the compressed
- * chunk records nm_spmm streams from HBM; residual_items = warp work items of
- * the residual SpMM (<= 256 nonzeros each), residual_split_rows = rows cut into several. */
+ * chunk records of the compressed-record kernel, full_image_bytes = the full
+ * records of the default kernel (4736 B per K = 32 chunk); residual_items = work items of the
+ * residual SpMM (<= 256 nonzeros each), residual_split_rows = rows cut into several. */
 typedef struct {
   int64_t n, row_begin, row_end, n_panels, n_mb, n_chunks, packed_nnz, residual_nnz;
   int64_t image_bytes, device_bytes, residual_items, residual_split_rows;
   int32_t V, M, Mp, Vp, tau, flags;
+  int64_t full_image_bytes;  /* full MMA-operand records (what the default kernel streams) */
+  int64_t gather_rows;       /* X rows the tensor-core part gathers (non-empty selected columns) */
 } nm_packed_stat;
 NM_API nm_status nm_packed_stats(const nm_packed* P, nm_packed_stat* st);
 

@@ -49,7 +49,8 @@ class nm_packed_stat(ctypes.Structure):
     _fields_ = [(k, ctypes.c_int64) for k in ("n", "row_begin", "row_end", "n_panels", "n_mb", "n_chunks",
                                               "packed_nnz", "residual_nnz", "image_bytes", "device_bytes",
                                               "residual_items", "residual_split_rows")] + \
-               [(k, ctypes.c_int32) for k in ("V", "M", "Mp", "Vp", "tau", "flags")]
+               [(k, ctypes.c_int32) for k in ("V", "M", "Mp", "Vp", "tau", "flags")] + \
+               [(k, ctypes.c_int64) for k in ("full_image_bytes", "gather_rows")]
 
 
 # name -> (restype, argtypes); mirrors include/nm.h exactly

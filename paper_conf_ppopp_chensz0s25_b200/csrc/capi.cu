@@ -259,6 +259,8 @@ nm_status nm_packed_stats(const nm_packed* P, nm_packed_stat* st) {
   st->Vp = P->Vp;
   st->tau = P->tau;
   st->flags = P->flags;
+  st->full_image_bytes = (int64_t)kChunkBytes * P->n_chunks;
+  st->gather_rows = P->gather_rows;
   return NM_OK;
 }
 

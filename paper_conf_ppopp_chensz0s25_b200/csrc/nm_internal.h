@@ -99,6 +99,7 @@ struct nm_packed {
   int32_t* cta_ptr = nullptr;          // [n_ctas+1] contiguous panel range of each SpMM CTA
   int n_ctas = 0;                      // persistent grid of the full-record kernel (#SMs)
   int sptc_format = 1;                 // tensor-core kernel nm_spmm uses: 1 full, 2 compressed
+  int64_t gather_rows = 0;             // non-negative gather rows over all chunks
   int64_t* res_rowptr = nullptr;       // [rows+1]
   int32_t* res_col = nullptr;          // [res_nnz] canonical (permuted) column
   uint16_t* res_val = nullptr;         // [res_nnz]

@@ -131,6 +131,15 @@ __global__ void k_meta_init(uint8_t* __restrict__ image, int64_t n_chunks) {
 }
 
 // perm == nullptr: initialise every record's xrow to -1; else map xrow entries through perm
+__global__ void k_count_gather(const uint8_t* __restrict__ image, int64_t n_chunks,
+                               unsigned long long* __restrict__ total) {
+  unsigned long long c = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_chunks * 32; i += (int64_t)gridDim.x * blockDim.x)
+    c += ((const int32_t*)(image + (i >> 5) * kChunkBytes + kChunkXrowOff))[i & 31] >= 0;
+  for (int o = 16; o > 0; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
+  if ((threadIdx.x & 31) == 0 && c) atomicAdd(total, c);
+}
+
 __global__ void k_xrow_map(const int32_t* __restrict__ perm, uint8_t* __restrict__ image, int64_t n_chunks) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_chunks * 32;
        i += (int64_t)gridDim.x * blockDim.x) {
@@ -919,6 +928,16 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     NM_CUDA(cudaStreamSynchronize(s));
   }
 
+  if (n_chunks) {  // X rows the tensor-core part gathers (roofline accounting)
+    DevBuf d_g;
+    NM_TRY(dalloc(d_g, sizeof(unsigned long long), s));
+    NM_CUDA(cudaMemsetAsync(d_g.p, 0, sizeof(unsigned long long), s));
+    k_count_gather<<<grid_for(n_chunks * 32, 256), 256, 0, s>>>(Pk->image_full, n_chunks, d_g.as<unsigned long long>());
+    unsigned long long gr = 0;
+    NM_CUDA(cudaMemcpyAsync(&gr, d_g.p, sizeof(gr), cudaMemcpyDeviceToHost, s));
+    NM_CUDA(cudaStreamSynchronize(s));
+    Pk->gather_rows = (int64_t)gr;
+  }
   // persistent-grid work split of the full-record kernel: one contiguous panel range per SM,
   // balanced by chunk count (+ a per-panel term for its epilogue)
   {

@@ -38,6 +38,11 @@ namespace {
 #define NM_FULL_MAX_STAGES 16
 #endif
 constexpr int kFGroups = NM_FULL_GROUPS;            // gather groups (4 warps each)
+#ifdef NM_FULL_MMA_ONLY
+#define NM_FULL_MMA_ONLY_ON 1
+#else
+#define NM_FULL_MMA_ONLY_ON 0
+#endif
 constexpr int kWProd = 0, kWG0 = 1, kWMma = kWG0 + 4 * kFGroups, kWEpi0 = kWMma + 1;
 constexpr int kFThreads = (kWEpi0 + 4) * 32;        // 14 warps
 constexpr int kGThreads = 128;                      // threads per gather group
@@ -111,32 +116,39 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t
 
 template <int BN>
 struct FCfg {
-  static constexpr int kBBytes = 32 * BN * 2;       // 32 gathered rows x BN 16-bit values
+  // chunks per pipeline stage: two K = 32 chunks share one barrier round trip (one record
+  // copy of 2 x 4736 B -- consecutive chunks are adjacent in the image -- two gather sets, one
+  // tcgen05.st.x2 of the two metadata columns, two MMAs and one commit)
+  static constexpr int kCPS = BN <= 128 ? 2 : 1;
+  static constexpr int kBBytes = 32 * BN * 2;       // one chunk's 32 gathered rows x BN
   static constexpr int kRecBytes = kChunkBytes;     // A (4096) + metadata (512) + gather rows (128)
-  static constexpr int kStageBytes = kBBytes + kRecBytes;
+  static constexpr int kStageBytes = kCPS * (kBBytes + kRecBytes);
   static constexpr int kStagesRaw = (222 * 1024 - 2048) / kStageBytes;
-  static constexpr int kStages =
-      ((kStagesRaw > NM_FULL_MAX_STAGES ? NM_FULL_MAX_STAGES : kStagesRaw) / kFGroups) * kFGroups;
-  static constexpr int kNAcc = (3 * BN + kStages <= 512) ? 3 : (2 * BN + kStages <= 512) ? 2 : 1;
-  static constexpr int kMeta0 = kNAcc * BN;         // metadata column of stage s: kMeta0 + s
+  static constexpr int kMaxStages = NM_FULL_MAX_STAGES / kCPS;
+  static constexpr int kStages = ((kStagesRaw > kMaxStages ? kMaxStages : kStagesRaw) / kFGroups) * kFGroups;
+  static constexpr int kMetaCols = kCPS * kStages;
+  static constexpr int kNAcc = (3 * BN + kMetaCols <= 512) ? 3 : (2 * BN + kMetaCols <= 512) ? 2 : 1;
+  static constexpr int kMeta0 = kNAcc * BN;         // metadata column of (stage s, chunk j): kMeta0 + kCPS*s + j
   static constexpr int kSmem = 1024 + kStages * kStageBytes + 1024;
-  static_assert(kMeta0 + kStages <= 512, "TMEM budget");
+  static_assert(kMeta0 + kMetaCols <= 512, "TMEM budget");
   static_assert(kRecBytes % 16 == 0, "bulk copy granularity");
   static_assert(kSmem <= 227 * 1024, "smem");
+  static_assert(kStages >= 2, "stages");
   static_assert((32 * (BN / 8)) % kGThreads == 0 && kGThreads % (BN / 8) == 0, "gather piece mapping");
 };
 
 template <int BN>
 __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) {
   using C = FCfg<BN>;
+  constexpr int CPS = C::kCPS;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  const uint32_t sB = smem_u32(smem);                    // kStages B tiles (1024-aligned, SW128)
-  const uint32_t sRec = sB + C::kStages * C::kBBytes;    // kStages records
+  const uint32_t sB = smem_u32(smem);                          // stage s: CPS B tiles (SW128)
+  const uint32_t sRec = sB + C::kStages * CPS * C::kBBytes;    // stage s: CPS adjacent records
   uint64_t* bars = (uint64_t*)(smem + C::kStages * C::kStageBytes);
-  uint64_t* full_rec = bars;                 // record landed (tx)
+  uint64_t* full_rec = bars;                 // records landed (tx)
   uint64_t* full_b = full_rec + C::kStages;  // gathers landed + metadata written
-  uint64_t* empty = full_b + C::kStages;     // MMA done with the stage (tcgen05.commit)
+  uint64_t* empty = full_b + C::kStages;     // MMAs done with the stage (tcgen05.commit)
   uint64_t* tfull = empty + C::kStages;      // accumulator ready
   uint64_t* tempty = tfull + 4;              // accumulator drained
   uint32_t* tmem_slot = (uint32_t*)(tempty + 4);
@@ -188,20 +200,27 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
                        : "memory");
       }
       for (int ft = 0; ft < nft; ++ft) {
-        for (int c = 0; c < nch; ++c) {
-          mbar_wait(bEmpty + 8 * s, ph ^ 1);  // the MMA has finished with stage s
+        for (int c = 0; c < nch; c += CPS) {
+          const int sub = min(CPS, nch - c);
+          mbar_wait(bEmpty + 8 * s, ph ^ 1);  // the MMAs have finished with stage s
+#ifdef NM_FULL_MMA_ONLY  // timing experiment (results invalid): no record copies
+          if (lane == 0) mbar_arrive(bRec + 8 * s);
+          __syncwarp();
+          if (++s == C::kStages) { s = 0; ph ^= 1; }
+          continue;
+#endif
           if (lane == 0) {
             if (c + kPfChunks < nch && ft == 0)
               asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p.image + (c0 + c + kPfChunks) * kChunkBytes),
-                           "r"((uint32_t)kChunkBytes)
+                           "r"((uint32_t)(min(CPS, nch - c - kPfChunks) * kChunkBytes))
                            : "memory");
-            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bRec + 8 * s),
-                         "r"((uint32_t)kChunkBytes)
+            const uint32_t bytes = (uint32_t)(sub * kChunkBytes);
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bRec + 8 * s), "r"(bytes)
                          : "memory");
             asm volatile(
                 "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                    sRec + s * C::kRecBytes),
-                "l"(p.image + (c0 + c) * kChunkBytes), "r"((uint32_t)kChunkBytes), "r"(bRec + 8 * s)
+                    sRec + s * CPS * C::kRecBytes),
+                "l"(p.image + (c0 + c) * kChunkBytes), "r"(bytes), "r"(bRec + 8 * s)
                 : "memory");
           }
           __syncwarp();
@@ -216,13 +235,13 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
     const int quarter = warp & 3;          // TMEM lane quarter this warp may access
     const int t = threadIdx.x - (kWG0 + 4 * group) * 32;  // 0..127 within the group
     constexpr int kRowPieces = BN / 8;     // 16-byte pieces per gathered row
-    constexpr int kPer = 32 * kRowPieces / kGThreads;  // pieces per thread
+    constexpr int kPer = 32 * kRowPieces / kGThreads;  // pieces per thread and chunk
     constexpr int kRowsPerPass = kGThreads / kRowPieces;
     const int c16 = t % kRowPieces, kk0 = t / kRowPieces;
     const uint32_t dcol = (uint32_t)(c16 >> 3) * 4096u;  // 64-column slab of the SW128 tile
     const int32_t ldx32 = (int32_t)p.ldx;
     const uint32_t mword = 4u * (uint32_t)(quarter * 32 + lane);  // this lane's metadata word
-    int64_t i = 0;  // CTA chunk counter
+    int64_t i = 0;  // CTA stage counter
     int s = 0;
     uint32_t ph = 0;
     int64_t c0 = pa < pz ? __ldg(p.panel_chunk_ptr + pa) : 0;
@@ -234,40 +253,59 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
         const int col0 = ft * BN + c16 * 8;
         const uint32_t colbytes = col0 >= p.F ? 0u : (p.F - col0 >= 8 ? 16u : (uint32_t)(p.F - col0) * 2u);
         const uint16_t* xcol = p.X + (colbytes ? col0 : 0);
-        for (int c = 0; c < nch; ++c, ++i) {
+        for (int c = 0; c < nch; c += CPS, ++i) {
           if ((int)(i % kFGroups) == group) {  // kFGroups divides kStages: group g owns s = g (mod kFGroups)
-            mbar_wait(bRec + 8 * s, ph);  // record landed (gather rows, metadata, A)
-            const uint32_t rec = sRec + s * C::kRecBytes;
-            const uint32_t sbase = sB + s * C::kBBytes + dcol;
-            if (colbytes == 16u) {
+            const int sub = min(CPS, nch - c);
+            mbar_wait(bRec + 8 * s, ph);  // records landed (gather rows, metadata, A)
+            const uint32_t rec0 = sRec + s * CPS * C::kRecBytes;
+            uint32_t mw[CPS];
 #pragma unroll
-              for (int q = 0; q < kPer; ++q) {
-                const int kk = q * kRowsPerPass + kk0;
-                const int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * kk);
-                asm volatile(
-                    "{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %2, 0;\n\t"
-                    "cp.async.cg.shared.global [%0], [%1], 16, q;\n\t}" ::"r"(
-                        sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
-                    "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(xr)
-                    : "memory");
-              }
-            } else {  // the F tail: partial or empty pieces
+            for (int j = 0; j < CPS; ++j) {
+              if (j < sub) {
+                const uint32_t rec = rec0 + j * C::kRecBytes;
+                const uint32_t sbase = sB + (s * CPS + j) * C::kBBytes + dcol;
+#ifdef NM_FULL_MMA_ONLY  // timing experiment (results invalid): no gathers
+                if (false) {
+#else
+                if (colbytes == 16u) {
+#endif
 #pragma unroll
-              for (int q = 0; q < kPer; ++q) {
-                const int kk = q * kRowsPerPass + kk0;
-                const int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * kk);
-                const uint32_t nb = xr >= 0 ? colbytes : 0u;
-                asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(
-                                 sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
-                             "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(nb)
-                             : "memory");
+                  for (int q = 0; q < kPer; ++q) {
+                    const int kk = q * kRowsPerPass + kk0;
+                    const int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * kk);
+                    asm volatile(
+                        "{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %2, 0;\n\t"
+                        "cp.async.cg.shared.global [%0], [%1], 16, q;\n\t}" ::"r"(
+                            sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
+                        "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(xr)
+                        : "memory");
+                  }
+                } else if (!NM_FULL_MMA_ONLY_ON) {  // the F tail: partial or empty pieces
+#pragma unroll
+                  for (int q = 0; q < kPer; ++q) {
+                    const int kk = q * kRowsPerPass + kk0;
+                    const int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * kk);
+                    const uint32_t nb = xr >= 0 ? colbytes : 0u;
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(
+                                     sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
+                                 "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(nb)
+                                 : "memory");
+                  }
+                }
+                mw[j] = lds32(rec + kChunkValBytes + mword);
+              } else {
+                mw[j] = 0x44444444u;  // unused column (legal no-value nibbles)
               }
             }
             asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bFull + 8 * s) : "memory");
-            // metadata: this lane's word of the record into the stage's TMEM column
-            const uint32_t w = lds32(rec + kChunkValBytes + mword);
-            const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + s;
-            asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(w) : "memory");
+            // metadata: this lane's words of the stage's records into its TMEM columns
+            const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + CPS * s;
+            if constexpr (CPS == 2)
+              asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1, %2};" ::"r"(taddr), "r"(mw[0]),
+                           "r"(mw[CPS - 1])
+                           : "memory");
+            else
+              asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(mw[0]) : "memory");
             asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
             asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
             __syncwarp();
@@ -285,8 +323,6 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
     uint32_t aphase = 0;
     const uint64_t adesc0 = sdesc(sRec, 128, 256, 0);   // A: K-major, no swizzle (LBO 128, SBO 256)
     const uint64_t bdesc0 = sdesc(sB, 4096, 1024, 2);   // B: MN-major, SWIZZLE_128B
-    uint64_t ad = adesc0, bd = bdesc0;
-    uint32_t mcol = C::kMeta0;
     int64_t c0 = pa < pz ? __ldg(p.panel_chunk_ptr + pa) : 0;
     for (int pn = pa; pn < pz; ++pn) {
       const int64_t c1 = __ldg(p.panel_chunk_ptr + pn + 1);
@@ -296,31 +332,35 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
         mbar_wait(bTempty + 8 * acc, aphase ^ 1);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t dcol = tbase + acc * BN;
-        for (int c = 0; c < nch; ++c) {
+        for (int c = 0; c < nch; c += CPS) {
+          const int sub = min(CPS, nch - c);
           mbar_wait(bFull + 8 * s, ph);
           // the gathers (cp.async) were written through the generic proxy: make them visible
           // to the tensor core's async-proxy operand reads
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          asm volatile(
-              "{\n\t.reg .pred e, q;\n\t"
-              "elect.sync _|e, 0xffffffff;\n\t"
-              "setp.ne.b32 q, %5, 0;\n\t"
-              "@e tcgen05.mma.sp.cta_group::1.kind::f16 [%0], %1, %2, [%3], %4, q;\n\t"
-              "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%6];\n\t}" ::"r"(dcol),
-              "l"(ad), "l"(bd), "r"(tbase + (mcol & ~1u)), "r"(p.idesc | (mcol & 1u)), "r"(c), "r"(bEmpty + 8 * s)
-              : "memory");
-          if (++s == C::kStages) {
-            s = 0;
-            ph ^= 1;
-            ad = adesc0;
-            bd = bdesc0;
-            mcol = C::kMeta0;
-          } else {
-            ad += (uint64_t)(C::kRecBytes >> 4);
-            bd += (uint64_t)(C::kBBytes >> 4);
-            ++mcol;
+#pragma unroll
+          for (int j = 0; j < CPS; ++j) {
+            if (j < sub) {
+              const uint64_t ad = adesc0 + (uint64_t)(((s * CPS + j) * C::kRecBytes) >> 4);
+              const uint64_t bd = bdesc0 + (uint64_t)(((s * CPS + j) * C::kBBytes) >> 4);
+              const uint32_t mcol = C::kMeta0 + CPS * s + j;
+              // metadata column: even column address + sparse_id2 selects the odd one
+              asm volatile(
+                  "{\n\t.reg .pred e, q;\n\t"
+                  "elect.sync _|e, 0xffffffff;\n\t"
+                  "setp.ne.b32 q, %5, 0;\n\t"
+                  "@e tcgen05.mma.sp.cta_group::1.kind::f16 [%0], %1, %2, [%3], %4, q;\n\t}" ::"r"(dcol),
+                  "l"(ad), "l"(bd), "r"(tbase + (mcol & ~1u)), "r"(p.idesc | (mcol & 1u)), "r"(c + j)
+                  : "memory");
+            }
           }
+          asm volatile(
+              "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+              "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(bEmpty +
+                                                                                                            8 * s)
+              : "memory");
+          if (++s == C::kStages) { s = 0; ph ^= 1; }
         }
         if (nch > 0)
           asm volatile(
