@@ -15,7 +15,7 @@
  *  - Every function returns nm_status; no exception or longjmp crosses the ABI.  On error
  *    the out-parameters are left untouched and nm_last_error() (thread-local) says why.
  *  - perm[p] = old vertex id placed at new position p (the paper's phi' as a list, Alg. 1
- *    output L358).  B[p][q] = A[perm[p]][perm[q]];  (P X)[p] = X[perm[p]]  (Fig. 1 caption
+ *    output L255).  B[p][q] = A[perm[p]][perm[q]];  (P X)[p] = X[perm[p]]  (Fig. 1 caption
  *    L38: "the corresponding rows in the dense matrix ... must be swapped too").
  *  - Graphs are CSR: rowptr int64[n+1], col int32[nnz], columns sorted ascending, no
  *    duplicates, symmetric pattern (undirected graph, L188), self-loops allowed.
@@ -70,8 +70,8 @@ typedef struct {
 /* Reordering options (Alg. 1-3).  Zero-initialise and set what you need, or pass NULL for
  * the defaults {10, 10, 10, 0, 1}. */
 typedef struct {
-  int max_outer;   /* Alg. 1 loop cap ("max. iteration", L359; MAXITER = 10, L496)        */
-  int max_stage1;  /* Alg. 2 MAXITER (L421)                                                */
+  int max_outer;   /* Alg. 1 loop cap ("max. iteration", L256; MAXITER = 10, L496)        */
+  int max_stage1;  /* Alg. 2 MAXITER (L336)                                                */
   int max_stage2;  /* Alg. 3 MAXITER (L451)                                                */
   int gain_rule;   /* 0 = paper: freshtop() takes the best fresh pair whatever its gain
                       (footnote L440); 1 = only pairs with positive gain                   */
@@ -88,7 +88,7 @@ typedef struct {
 } nm_reorder_stats;
 
 /* ---------------------------------------------------------------------------------------
- * nm_reorder -- the SGRP heuristic (Alg. 1, L354-362: repeat Stage-1 (Alg. 2, vertical
+ * nm_reorder -- the SGRP heuristic (Alg. 1, L248-260: repeat Stage-1 (Alg. 2, vertical
  * constraint, Hamming position codes + sort, L366-384) and Stage-2 (Alg. 3, horizontal
  * constraint, greedy pair swaps, L386-422) while violations remain).  Deterministic; the
  * permutation is bit-identical to the CPU oracle's (DESIGN.md §3 readings).
@@ -132,8 +132,8 @@ NM_API nm_status nm_count_violations(const nm_csr* A, const int32_t* perm, int V
  * Packed V:N:M matrix (the SPTC form of L492).  Rows of B are grouped in
  * panels of Vp = 128 rows; columns in segments of Mp columns, Mp = 4 when V == 1 (2:4 at
  * V = 1) and Mp = M otherwise; per non-empty (panel, segment) meta-block the k = 4 columns
- * with the most nonzeros are selected (vertical constraint, L338-339) and each row keeps
- * its first <= 2 nonzeros among them (N = 2, horizontal constraint L340-341) as two 16-bit
+ * with the most nonzeros are selected (vertical constraint, L226-227) and each row keeps
+ * its first <= 2 nonzeros among them (N = 2, horizontal constraint L229-230) as two 16-bit
  * values plus a 4-bit index pair.  Everything else goes to a residual CSR.  Device memory
  * holds the MMA-native image consumed by nm_spmm (tcgen05.mma.sp operands).
  * Supported: N = 2; M in {4, 8, 16}; any V >= 1 (V = 1 -> Mp = 4); Vp = 128 (pass 0 or

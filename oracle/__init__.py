@@ -3,16 +3,19 @@
 Plain, slow, obviously correct CPU reference of what the hot path of Chen et al.,
 "Accelerating GNNs on GPU Sparse Tensor Cores through N:M Sparsity-Oriented Graph
 Reordering" (PPoPP'25) computes.  The arithmetic lives in ``oracle/oracle.c`` (plain C,
-fp64 for floating point); this module only marshals numpy arrays through ctypes.
+fp64 for floating point); this module marshals numpy arrays through ctypes, except for the
+dense parts of the GCN layer reference (``gcn_layer`` / ``gcn_layer_backward``: fp64 numpy
+matmul and elementwise steps around the C SpMM, plus ``csr_transpose``) and the canonical
+``unpack`` used by the pack invariants.
 
 Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
 ``--impl reference`` legs may import this package.  It shares no code with the CUDA path
 (``paper_conf_ppopp_chensz0s25_b200``) and neither imports the other.
 
-Pins (see tests/test_oracle_*.py): worked values of PAPER.md:L383-411 (§4.2), brute-force
+Pins (see tests/test_oracle_*.py): worked values of PAPER.md:L286-319 (§4.2), brute-force
 minimal cumulative-Hamming orders, brute-force violation counts, the Figure-1 fixture F1,
-brute-force optimum bounds on tiny graphs, pack/unpack invariants, dense A@X.
-The reorder permutation itself is "parity unpinned" beyond those pins.
+four hand-derived Stage-2 passes (tests/golden/s2_fixture_*.txt), brute-force optimum
+bounds on tiny graphs, pack/unpack invariants, dense A@X.
 """
 from __future__ import annotations
 
@@ -108,12 +111,12 @@ def _csr(indptr, indices):
 
 
 def hamming_code(b: int) -> int:
-    """Rank of bit string b in the Hamming-distance order (PAPER.md:L399-404)."""
+    """Rank of bit string b in the Hamming-distance order (PAPER.md:L306-311)."""
     return int(_lib().or_hamming_code(int(b)))
 
 
 def position_code(b: int, N: int) -> int:
-    """Hamming position code, negated for an N:M-violating string (L405-411)."""
+    """Hamming position code, negated for an N:M-violating string (L313-319)."""
     return int(_lib().or_position_code(int(b), int(N)))
 
 
@@ -138,7 +141,7 @@ def counts(indptr, indices, perm, V: int, N: int, M: int):
 
 def reorder(indptr, indices, V: int, N: int, M: int, max_outer: int = 10, max_stage1: int = 10,
             max_stage2: int = 10, gain_rule: int = 0, keep_best: int = 1):
-    """Alg. 1 (PAPER.md:L354-362) with Stage-1 (Alg. 2) and Stage-2 (Alg. 3).
+    """Alg. 1 (PAPER.md:L248-260) with Stage-1 (Alg. 2) and Stage-2 (Alg. 3).
     Returns (perm, stats) with perm[new position] = old vertex."""
     rp, ci, n = _csr(indptr, indices)
     perm = np.zeros(max(n, 1), dtype=np.int32)

@@ -13,13 +13,14 @@
  * (paper_conf_ppopp_chensz0s25_b200/csrc) and includes nothing from it.
  *
  * Pins (tests/test_oracle_*.py, -m "not gpu"):
- *   or_hamming_code / or_position_code -- worked values PAPER.md:L383-411, brute-force minimal
+ *   or_hamming_code / or_position_code -- worked values PAPER.md:L286-319, brute-force minimal
  *       cumulative-Hamming orders, reflected-Gray construction.
  *   or_counts (omega, PScore, MBscore) -- brute force on dense matrices in Python.
- *   or_reorder -- Figure-1 fixture F1 (unique answer), brute-force optimum bound on tiny
- *       graphs, invariants (bijection, keep-best, <= M pairs per primary).  The exact
- *       permutation of the greedy heuristic has no closed form: "parity unpinned" beyond
- *       those pins.
+ *   or_reorder / or_stage2_trace -- Figure-1 fixture F1 (unique answer), four hand-derived
+ *       Stage-2 passes (tests/golden/s2_fixture_{a,b,c,d}.txt: priority order, gain tables,
+ *       recorded pairs of both branches of Alg. 3; 13 oracle mutants killed,
+ *       tools/oracle_mutants.py), brute-force optimum bound on tiny graphs, invariants
+ *       (bijection, keep-best, <= M pairs per primary).
  *   or_pack_* -- unpack(pack)+residual == B bitwise, conforming => empty residual, F1 nibbles.
  *   or_spmm_f64 -- dense numpy A@X on small cases; closed forms (identity, all-ones).
  */
@@ -34,11 +35,11 @@
 #define OR_K 4 /* k of the vertical constraint: "4 by default" (Fig. 2 table) */
 
 /* ------------------------------------------------------------------------------------- */
-/* Hamming position code (PAPER.md:L394-411, §4.2)                                        */
+/* Hamming position code (PAPER.md:L300-319, §4.2)                                        */
 /* ------------------------------------------------------------------------------------- */
 
 /* Rank of the bit string b in the Hamming-distance order of all strings of its length.
- * The Hamming-distance order the paper uses ({00,01,11,10} for 2 digits, L389-391) is the
+ * The Hamming-distance order the paper uses ({00,01,11,10} for 2 digits, L294-296) is the
  * binary reflected Gray code, whose i-th element is i ^ (i>>1); the rank of b is therefore
  * the inverse Gray code b ^ b>>1 ^ b>>2 ^ ... (reading #1). */
 int64_t or_hamming_code(uint64_t b) {
@@ -49,7 +50,7 @@ int64_t or_hamming_code(uint64_t b) {
 
 static int popc64(uint64_t x) { int c = 0; while (x) { c += (int)(x & 1u); x >>= 1; } return c; }
 
-/* Position code with the horizontal-violation negation (L405-411, Alg. 2 lines 8-10). */
+/* Position code with the horizontal-violation negation (L313-319, Alg. 2 lines 8-10 at L344-346). */
 int64_t or_position_code(uint64_t b, int N) {
   int64_t h = or_hamming_code(b);
   return popc64(b) > N ? -h : h;
@@ -210,7 +211,7 @@ int or_counts(int64_t n, const int64_t* rp, const int32_t* ci, const int32_t* pe
 }
 
 /* ------------------------------------------------------------------------------------- */
-/* Stage-1 (Alg. 2, L414-435; steps (i)-(v) L374-382)                                     */
+/* Stage-1 (Alg. 2, L326-362; steps (i)-(v) L374-382)                                     */
 /* ------------------------------------------------------------------------------------- */
 
 typedef struct { int64_t* key; int64_t len; int64_t row; } s1_key; /* key = pairs flattened */
@@ -474,7 +475,7 @@ int64_t or_stage2_trace(int64_t n, const int64_t* rp, const int32_t* ci, const i
 }
 
 /* ------------------------------------------------------------------------------------- */
-/* Alg. 1 (L354-362): repeat Stage-1, Stage-2 while violations remain                    */
+/* Alg. 1 (L248-260): repeat Stage-1, Stage-2 while violations remain                    */
 /* ------------------------------------------------------------------------------------- */
 
 typedef struct {

@@ -50,8 +50,11 @@ constexpr int res_smem_bytes() {
   return NM_RES_CPASYNC ? 8 * (32 / LPR) * 2 * (LPR < kResBatch ? LPR : kResBatch) * LPR * 16 : 0;
 }
 
-__device__ __forceinline__ void cp_async16_z(uint32_t dst, const void* src, uint32_t nbytes) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(nbytes) : "memory");
+// X rows of the residual: L2 evict-last (they are re-read by other rows' nonzeros)
+__device__ __forceinline__ void cp_async16_z(uint32_t dst, const void* src, uint32_t nbytes, uint64_t pol) {
+  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(dst), "l"(src), "r"(nbytes),
+               "l"(pol)
+               : "memory");
 }
 
 template <int BF, int LPR>
@@ -76,6 +79,8 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
   const uint32_t ring = (uint32_t)__cvta_generic_to_shared(res_smem) +
                         (uint32_t)((((threadIdx.x >> 5) * SUB + sub) * 2 * KB * LPR + li) * 16);
   const uint32_t xbytes = f < F ? 16u : 0u;
+  uint64_t pol_x;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_x));
   int64_t w = ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5) * SUB + sub;
   ResSeg gn;
   if (w < n_segs) gn = segs[w];
@@ -100,14 +105,14 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
     int32_t cn = 0;
     uint32_t vn = 0u, vc = 0u;
     if (li < KB && li < g.len) {
-      cn = __ldg(rc + g.kb + li);
-      vn = __ldg(rv + g.kb + li);
+      cn = __ldcs(rc + g.kb + li);  // streamed once: evict-first
+      vn = __ldcs(rv + g.kb + li);
     }
     {  // issue batch 0
       const int cnt0 = min(KB, g.len);
       for (int j = 0; j < cnt0; ++j) {
         const int32_t cc = __shfl_sync(gmask, cn, j, LPR);
-        cp_async16_z(ring + j * LPR * 16, X + (int64_t)cc * ldx + (xbytes ? f : 0), xbytes);
+        cp_async16_z(ring + j * LPR * 16, X + (int64_t)cc * ldx + (xbytes ? f : 0), xbytes, pol_x);
       }
       asm volatile("cp.async.commit_group;" ::: "memory");
     }
@@ -120,13 +125,13 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
         cn = 0;
         vn = 0u;
         if (li < cnt1) {
-          cn = __ldg(rc + g.kb + e1 + li);
-          vn = __ldg(rv + g.kb + e1 + li);
+          cn = __ldcs(rc + g.kb + e1 + li);
+          vn = __ldcs(rv + g.kb + e1 + li);
         }
         const uint32_t rb = ring + ((k + 1) & 1) * KB * LPR * 16;
         for (int j = 0; j < cnt1; ++j) {
           const int32_t cc = __shfl_sync(gmask, cn, j, LPR);
-          cp_async16_z(rb + j * LPR * 16, X + (int64_t)cc * ldx + (xbytes ? f : 0), xbytes);
+          cp_async16_z(rb + j * LPR * 16, X + (int64_t)cc * ldx + (xbytes ? f : 0), xbytes, pol_x);
         }
         asm volatile("cp.async.commit_group;" ::: "memory");
         asm volatile("cp.async.wait_group 1;" ::: "memory");

@@ -4,7 +4,7 @@
 //  2. Meta-blocks = distinct (panel, segment) pairs with any nonzero, ascending (radix sort +
 //     run-length encode of panel*S + col/Mp keys).
 //  3. Column counts per meta-block -> the k = 4 selected columns (vertical constraint,
-//     L338-339): largest counts, ties to the smaller offset, ascending.
+//     L226-227): largest counts, ties to the smaller offset, ascending.
 //  4. Per (row, meta-block): the first <= 2 nonzeros among the selected columns (horizontal
 //     constraint, N = 2) go to the two MMA slots with a 4-bit index pair; the rest to the
 //     residual CSR.  Values and metadata are written straight into the MMA-native image.
@@ -168,7 +168,7 @@ __global__ void k_colcount(const int64_t* __restrict__ Brp, const int32_t* __res
 }
 
 // selected columns of every candidate meta-block: the 4 largest counts, ties -> smaller
-// offset, stored ascending (vertical constraint, L338-339; reading #19)
+// offset, stored ascending (vertical constraint, L226-227; reading #19)
 __global__ void k_select(const int32_t* __restrict__ cnt, int Mp, int64_t n_mb, uint32_t* __restrict__ selc) {
   for (int64_t m = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; m < n_mb;
        m += (int64_t)gridDim.x * blockDim.x) {

@@ -145,7 +145,7 @@ void stage1_sort(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t
       k.reserve(2 * rs.seg.size() + 2);
       for (size_t j = 0; j < rs.seg.size(); ++j) {
         const int64_t h = hamming_rank(rs.bits[j]);
-        const int64_t c = (rs.cnt[j] > N) ? -h : h;  // negated when violating N:M (L405-411)
+        const int64_t c = (rs.cnt[j] > N) ? -h : h;  // negated when violating N:M (L313-319)
         if (c == 0) continue;
         k.push_back((c > 0 ? 1 : -1) * (S - rs.seg[j]));
         k.push_back(c);

@@ -183,6 +183,10 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
 
   if (warp == kWProd) {
     // ------------------------------------------------------------ record producer
+    // records are streamed once: L2 evict-first, so they do not push the gathered X rows
+    // (evict-last) out of L2 (ncu, C3: DRAM reads 4.08 GB for 2.57 GB of records without it)
+    uint64_t pol_stream;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_stream));
     int s = 0;
     uint32_t ph = 0;
     int64_t c0 = pa < pz ? __ldg(p.panel_chunk_ptr + pa) : 0;
@@ -195,8 +199,8 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
         const int64_t n2 = __ldg(p.panel_chunk_ptr + pn + 2) - c1;
         const int64_t k = n2 < kPfChunks ? n2 : kPfChunks;
         if (k > 0)
-          asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p.image + c1 * kChunkBytes),
-                       "r"((uint32_t)(k * kChunkBytes))
+          asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;" ::"l"(p.image + c1 * kChunkBytes),
+                       "r"((uint32_t)(k * kChunkBytes)), "l"(pol_stream)
                        : "memory");
       }
       for (int ft = 0; ft < nft; ++ft) {
@@ -211,16 +215,17 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
 #endif
           if (lane == 0) {
             if (c + kPfChunks < nch && ft == 0)
-              asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p.image + (c0 + c + kPfChunks) * kChunkBytes),
-                           "r"((uint32_t)(min(CPS, nch - c - kPfChunks) * kChunkBytes))
+              asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;" ::"l"(
+                               p.image + (c0 + c + kPfChunks) * kChunkBytes),
+                           "r"((uint32_t)(min(CPS, nch - c - kPfChunks) * kChunkBytes)), "l"(pol_stream)
                            : "memory");
             const uint32_t bytes = (uint32_t)(sub * kChunkBytes);
             asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bRec + 8 * s), "r"(bytes)
                          : "memory");
             asm volatile(
-                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                    sRec + s * CPS * C::kRecBytes),
-                "l"(p.image + (c0 + c) * kChunkBytes), "r"(bytes), "r"(bRec + 8 * s)
+                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], "
+                "%4;" ::"r"(sRec + s * CPS * C::kRecBytes),
+                "l"(p.image + (c0 + c) * kChunkBytes), "r"(bytes), "r"(bRec + 8 * s), "l"(pol_stream)
                 : "memory");
           }
           __syncwarp();
@@ -241,6 +246,8 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
     const uint32_t dcol = (uint32_t)(c16 >> 3) * 4096u;  // 64-column slab of the SW128 tile
     const int32_t ldx32 = (int32_t)p.ldx;
     const uint32_t mword = 4u * (uint32_t)(quarter * 32 + lane);  // this lane's metadata word
+    uint64_t pol_x;  // gathered X rows stay in L2 (reused by the other panels' meta-blocks)
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_x));
     int64_t i = 0;  // CTA stage counter
     int s = 0;
     uint32_t ph = 0;
@@ -275,9 +282,9 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
                     const int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * kk);
                     asm volatile(
                         "{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %2, 0;\n\t"
-                        "cp.async.cg.shared.global [%0], [%1], 16, q;\n\t}" ::"r"(
+                        "cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, q, %3;\n\t}" ::"r"(
                             sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
-                        "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(xr)
+                        "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(xr), "l"(pol_x)
                         : "memory");
                   }
                 } else if (!NM_FULL_MMA_ONLY_ON) {  // the F tail: partial or empty pieces
@@ -286,9 +293,9 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
                     const int kk = q * kRowsPerPass + kk0;
                     const int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * kk);
                     const uint32_t nb = xr >= 0 ? colbytes : 0u;
-                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(
+                    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(
                                      sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
-                                 "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(nb)
+                                 "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(nb), "l"(pol_x)
                                  : "memory");
                   }
                 }

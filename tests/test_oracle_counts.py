@@ -2,7 +2,7 @@
 matrices, written here independently of the oracle).
 
 omega, PScore (L396), MBscore (L382, Fig. 3 caption L370, reading #5),
-Stage-1 order (Alg. 2 lines 4-13, L414-435; reading #6: ascending lexicographic order of the
+Stage-1 order (Alg. 2 lines 4-13, L326-362; reading #6: ascending lexicographic order of the
 per-row code vectors, stable).
 """
 import numpy as np
