@@ -299,6 +299,38 @@ NM_API nm_status nm_gcn_layer_backward(const nm_packed* Ahat, const void* H, con
                                        int flags, void* ws, size_t ws_bytes, void* stream);
 
 /* ------------------------------------------------------------------------------------- */
+/* ---------------------------------------------------------------------------------------
+ * The other GNN aggregations the paper evaluates (Table 3 "SGC",
+ * "SAGE", "Cheb"), on the same packed SpMM.  All need a pack of ALL rows (row_begin = 0,
+ * row_end = n); SAGE and Cheb a pack in permuted order (flags 0).  16-bit operands in the pack
+ * dtype, fp32 accumulation.  F_in / F_out multiples of 8.  Stream-ordered.
+ *
+ * nm_sgc_propagate -- SGC's propagation Y = Ahat^K X (K >= 1 SpMM hops).  X: n x F (ldx,
+ *   ldx % 8 == 0), Y: fp32 n x F (ldy); Y16: optional 16-bit copy of Y (ld = ldx) or NULL.  The
+ *   operand of hop k+1 is hop k's fp32 result rounded to the pack dtype.  Chains in the pack's
+ *   order (original order for NM_PACK_ORIGINAL_ORDER packs).  ws: nm_sgc_workspace_bytes.
+ * nm_sage_layer -- GraphSAGE, mean aggregator:
+ *   Hout = act([H | Amean H] [W_self; W_neigh] + bias), Amean = the pack of D^-1 A (row-
+ *   normalised values, supplied by the caller).  H: n x F_in; W_*: F_in x F_out; bias fp32 or
+ *   NULL; Hout: n x F_out.  flags: NM_RELU or 0.  ws: nm_sage_workspace_bytes.
+ * nm_cheb_layer -- Chebyshev convolution of order K:
+ *   Hout = act(sum_{k<K} T_k W_k + bias), T_0 = H, T_1 = Lhat H, T_k = 2 Lhat T_{k-1} - T_{k-2}
+ *   (each T_k rounded to the pack dtype), Lhat = the caller's scaled Laplacian pack (e.g.
+ *   -D^-1/2 A D^-1/2 for lambda_max = 2).  W: (K F_in) x F_out, W_0 on top.  ws:
+ *   nm_cheb_workspace_bytes.
+ * Errors: INVALID_ARG (NULL, sizes, workspace), UNSUPPORTED (row-sharded / fused-order pack,
+ * F not a multiple of 8), CUDA. */
+NM_API size_t nm_sgc_workspace_bytes(int64_t n, int F);
+NM_API nm_status nm_sgc_propagate(const nm_packed* Ahat, const void* X, int64_t ldx, float* Y, int64_t ldy,
+                                  void* Y16, int F, int K, void* ws, size_t ws_bytes, void* stream);
+NM_API size_t nm_sage_workspace_bytes(int64_t n, int F_in, int F_out);
+NM_API nm_status nm_sage_layer(const nm_packed* Amean, const void* H, const void* W_self, const void* W_neigh,
+                               const float* bias, void* Hout, int F_in, int F_out, int flags, void* ws,
+                               size_t ws_bytes, void* stream);
+NM_API size_t nm_cheb_workspace_bytes(int64_t n, int F_in, int F_out, int K);
+NM_API nm_status nm_cheb_layer(const nm_packed* Lhat, const void* H, const void* W, const float* bias, void* Hout,
+                               int F_in, int F_out, int K, int flags, void* ws, size_t ws_bytes, void* stream);
+
 NM_API const char* nm_status_string(nm_status s);
 NM_API const char* nm_last_error(void);   /* thread-local detail of the last failure on this thread */
 NM_API int nm_version(void);              /* ABI version, currently 1 */

@@ -335,3 +335,31 @@ def gcn_layer_backward(indptr, indices, val, H, W, Z, dHout, relu: bool):
     dW = np.asarray(H, dtype=np.float64).T @ dT
     dH = dT @ np.asarray(W, dtype=np.float64).T
     return dH, dW, db, dT
+
+
+def sgc_propagate(indptr, indices, val, X, K: int):
+    """SGC propagation (Table 3 "SGC" L546-553): Ahat^K X in fp64 (K SpMMs)."""
+    Y = np.asarray(X, dtype=np.float64)
+    for _ in range(K):
+        Y, _, _ = spmm(indptr, indices, val, Y)
+    return Y
+
+
+def sage_layer(indptr, indices, val_mean, H, W_self, W_neigh, b, relu: bool):
+    """GraphSAGE layer with the mean aggregator (Table 3 "SAGE"), fp64:
+    act(H W_self + (Amean H) W_neigh + b) with Amean = D^-1 A given as CSR values."""
+    Hd = np.asarray(H, dtype=np.float64)
+    agg, _, _ = spmm(indptr, indices, val_mean, Hd)
+    Z = Hd @ np.asarray(W_self, np.float64) + agg @ np.asarray(W_neigh, np.float64) + np.asarray(b, np.float64)
+    return (np.maximum(Z, 0.0) if relu else Z), agg
+
+
+def cheb_layer(indptr, indices, val_L, H, Ws, b, relu: bool):
+    """Chebyshev convolution (Table 3 "Cheb"), fp64: act(sum_k T_k Ws[k] + b) with
+    T_0 = H, T_1 = L H, T_k = 2 L T_{k-1} - T_{k-2} (Defferrard et al.'s recurrence)."""
+    T = [np.asarray(H, dtype=np.float64)]
+    for k in range(1, len(Ws)):
+        LT, _, _ = spmm(indptr, indices, val_L, T[k - 1])
+        T.append(LT if k == 1 else 2.0 * LT - T[k - 2])
+    Z = sum(T[k] @ np.asarray(Ws[k], np.float64) for k in range(len(Ws))) + np.asarray(b, np.float64)
+    return (np.maximum(Z, 0.0) if relu else Z), T

@@ -254,3 +254,37 @@ def gcn_layer_backward(P: Packed, H, W, Hout, dHout, dH, dW, db, ws, relu=True, 
                                            L.NM_RELU if relu else 0, _ptr(ws), ws.numel(),
                                            _stream_ptr(stream)),
             "nm_gcn_layer_backward")
+
+
+def sgc_propagate(P: Packed, X, Y, K: int, Y16=None, ws=None, stream=None):
+    """nm_sgc_propagate: Y (fp32, n x F) = Ahat^K X (SGC propagation)."""
+    import torch
+    F = X.shape[1]
+    if ws is None:
+        ws = torch.empty(int(L.load().nm_sgc_workspace_bytes(P.n, F)), dtype=torch.uint8, device=X.device)
+    L.check(L.load().nm_sgc_propagate(P.handle, _ptr(X), X.stride(0), _ptr(Y), Y.stride(0), _ptr(Y16), F, int(K),
+                                      _ptr(ws), ws.numel(), _stream_ptr(stream)), "nm_sgc_propagate")
+
+
+def sage_layer(P: Packed, H, W_self, W_neigh, bias, Hout, relu=True, ws=None, stream=None):
+    """nm_sage_layer: Hout = act([H | Amean H] [W_self; W_neigh] + bias) (GraphSAGE mean)."""
+    import torch
+    F_in, F_out = W_self.shape
+    if ws is None:
+        ws = torch.empty(int(L.load().nm_sage_workspace_bytes(P.n, F_in, F_out)), dtype=torch.uint8, device=H.device)
+    L.check(L.load().nm_sage_layer(P.handle, _ptr(H), _ptr(W_self), _ptr(W_neigh), _ptr(bias), _ptr(Hout), F_in, F_out,
+                                   L.NM_RELU if relu else 0, _ptr(ws), ws.numel(), _stream_ptr(stream)),
+            "nm_sage_layer")
+
+
+def cheb_layer(P: Packed, H, W, bias, Hout, K: int, relu=True, ws=None, stream=None):
+    """nm_cheb_layer: Hout = act(sum_k T_k(Lhat) H W_k + bias); W is (K F_in) x F_out."""
+    import torch
+    F_in = H.shape[1]
+    F_out = W.shape[1]
+    if ws is None:
+        ws = torch.empty(int(L.load().nm_cheb_workspace_bytes(P.n, F_in, F_out, K)), dtype=torch.uint8,
+                         device=H.device)
+    L.check(L.load().nm_cheb_layer(P.handle, _ptr(H), _ptr(W), _ptr(bias), _ptr(Hout), F_in, F_out, int(K),
+                                   L.NM_RELU if relu else 0, _ptr(ws), ws.numel(), _stream_ptr(stream)),
+            "nm_cheb_layer")

@@ -195,6 +195,15 @@ inline int grid_for(int64_t total) {
 }
 
 }  // namespace
+
+// row-major C[m x nc] = A[m x k] W[k x nc] (leading dimensions in elements; cuBLASLt, fp32
+// accumulation) for the other model layers (models.cu)
+nm_status gemm_rm(const void* A, int64_t lda, const void* W, int64_t ldw, void* C, int64_t ldc, int64_t m, int k,
+                  int nc, nm_dtype dt, bool c_f32, void* ws, cudaStream_t s) {
+  return lt_gemm(false, false, nc, m, k, W, ldw, A, lda, C, ldc, dt, c_f32, ws, s);
+}
+size_t lt_workspace_bytes() { return kLtWorkspace; }
+
 }  // namespace nm
 
 using namespace nm;

@@ -112,6 +112,13 @@ struct nm_packed {
   // by each nm_spmm call on its stream
   nm::ResSeg* res_segs = nullptr;      // [n_res_segs]
   int64_t n_res_segs = 0, n_res_slots = 0, n_res_split = 0;
+  // the same items in panel order for the residual fused into the full-record kernel: per
+  // panel the split rows' items (grouped by row, in item order), then single-item rows
+  // longest first; res_rowmask bit r of panel p = row 128p + r has residual entries
+  nm::ResSeg* res_items = nullptr;     // [n_res_segs]
+  int64_t* res_pptr = nullptr;         // [n_panels + 1]
+  int64_t* res_psplit = nullptr;       // [n_panels]
+  uint32_t* res_rowmask = nullptr;     // [n_panels * 4]
   size_t device_bytes = 0;
 };
 
@@ -121,6 +128,12 @@ namespace nm {
 void set_error(const std::string& msg);
 nm_status fail(nm_status s, const std::string& msg);
 nm_status cuda_fail(cudaError_t e, const char* what);
+
+#define NM_TRY_STATUS(x)             \
+  do {                               \
+    nm_status st_try_ = (x);         \
+    if (st_try_ != NM_OK) return st_try_; \
+  } while (0)
 
 #define NM_CUDA(call)                                     \
   do {                                                    \
@@ -178,13 +191,16 @@ uint16_t one_bits(nm_dtype dt);
 nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                            int64_t ldy, int F, cudaStream_t s);
 nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy,
-                           int F, cudaStream_t s, int format);
+                           int F, cudaStream_t s, int format, bool fuse_residual = false);
 nm_status launch_spmm_sptc_full(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
-                                int64_t ldy, int F, cudaStream_t s);
+                                int64_t ldy, int F, cudaStream_t s, bool fuse_residual);
 nm_status launch_spmm_sptc_compressed(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                                       int64_t ldy, int F, cudaStream_t s);
 nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                                int64_t ldy, int F, cudaStream_t s);
+nm_status gemm_rm(const void* A, int64_t lda, const void* W, int64_t ldw, void* C, int64_t ldc, int64_t m, int k,
+                  int nc, nm_dtype dt, bool c_f32, void* ws, cudaStream_t s);
+size_t lt_workspace_bytes();
 nm_status count_violations_dev(const DevCsr& A, const int32_t* perm_dev, int V, int N, int M,
                                int64_t* omega, int64_t* mb, int32_t* pscore_host,
                                cudaStream_t s);

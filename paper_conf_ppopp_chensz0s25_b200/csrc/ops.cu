@@ -50,11 +50,8 @@ constexpr int res_smem_bytes() {
   return NM_RES_CPASYNC ? 8 * (32 / LPR) * 2 * (LPR < kResBatch ? LPR : kResBatch) * LPR * 16 : 0;
 }
 
-// X rows of the residual: L2 evict-last (they are re-read by other rows' nonzeros)
-__device__ __forceinline__ void cp_async16_z(uint32_t dst, const void* src, uint32_t nbytes, uint64_t pol) {
-  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(dst), "l"(src), "r"(nbytes),
-               "l"(pol)
-               : "memory");
+__device__ __forceinline__ void cp_async16_z(uint32_t dst, const void* src, uint32_t nbytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(nbytes) : "memory");
 }
 
 template <int BF, int LPR>
@@ -79,8 +76,6 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
   const uint32_t ring = (uint32_t)__cvta_generic_to_shared(res_smem) +
                         (uint32_t)((((threadIdx.x >> 5) * SUB + sub) * 2 * KB * LPR + li) * 16);
   const uint32_t xbytes = f < F ? 16u : 0u;
-  uint64_t pol_x;
-  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_x));
   int64_t w = ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5) * SUB + sub;
   ResSeg gn;
   if (w < n_segs) gn = segs[w];
@@ -100,38 +95,37 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
     for (int q = 0; q < 8; ++q) acc[q] = 0.f;
 #if NM_RES_CPASYNC
     // two batches of KB entries in flight: batch k+1's X rows are copied (cp.async, no
-    // registers held) while batch k is accumulated from shared memory
+    // registers held) while batch k is accumulated from shared memory.  Both loops have a fixed
+    // trip count (KB): entries past the item's end are zero-filled copies (ignore-src) with a
+    // zero value, so the batch needs no per-entry branch and no divergent shuffles.
     const int nb = (g.len + KB - 1) / KB;
     int32_t cn = 0;
     uint32_t vn = 0u, vc = 0u;
     if (li < KB && li < g.len) {
-      cn = __ldcs(rc + g.kb + li);  // streamed once: evict-first
-      vn = __ldcs(rv + g.kb + li);
+      cn = __ldg(rc + g.kb + li);  // streamed once
+      vn = __ldg(rv + g.kb + li);
     }
-    {  // issue batch 0
-      const int cnt0 = min(KB, g.len);
-      for (int j = 0; j < cnt0; ++j) {
-        const int32_t cc = __shfl_sync(gmask, cn, j, LPR);
-        cp_async16_z(ring + j * LPR * 16, X + (int64_t)cc * ldx + (xbytes ? f : 0), xbytes, pol_x);
-      }
-      asm volatile("cp.async.commit_group;" ::: "memory");
+#pragma unroll
+    for (int j = 0; j < KB; ++j) {  // issue batch 0
+      const int32_t cc = __shfl_sync(gmask, cn, j, LPR);
+      cp_async16_z(ring + j * LPR * 16, X + (int64_t)cc * ldx + (xbytes ? f : 0), j < g.len ? xbytes : 0u);
     }
+    asm volatile("cp.async.commit_group;" ::: "memory");
     for (int k = 0; k < nb; ++k) {
       vc = vn;
-      const int cntk = min(KB, g.len - k * KB);
       if (k + 1 < nb) {
         const int e1 = (k + 1) * KB;
-        const int cnt1 = min(KB, g.len - e1);
         cn = 0;
         vn = 0u;
-        if (li < cnt1) {
-          cn = __ldcs(rc + g.kb + e1 + li);
-          vn = __ldcs(rv + g.kb + e1 + li);
+        if (li < KB && e1 + li < g.len) {
+          cn = __ldg(rc + g.kb + e1 + li);
+          vn = __ldg(rv + g.kb + e1 + li);
         }
         const uint32_t rb = ring + ((k + 1) & 1) * KB * LPR * 16;
-        for (int j = 0; j < cnt1; ++j) {
+#pragma unroll
+        for (int j = 0; j < KB; ++j) {
           const int32_t cc = __shfl_sync(gmask, cn, j, LPR);
-          cp_async16_z(rb + j * LPR * 16, X + (int64_t)cc * ldx + (xbytes ? f : 0), xbytes, pol_x);
+          cp_async16_z(rb + j * LPR * 16, X + (int64_t)cc * ldx + (xbytes ? f : 0), e1 + j < g.len ? xbytes : 0u);
         }
         asm volatile("cp.async.commit_group;" ::: "memory");
         asm volatile("cp.async.wait_group 1;" ::: "memory");
@@ -139,7 +133,8 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
         asm volatile("cp.async.wait_group 0;" ::: "memory");
       }
       const uint32_t rb = ring + (k & 1) * KB * LPR * 16;
-      for (int j = 0; j < cntk; ++j) {
+#pragma unroll
+      for (int j = 0; j < KB; ++j) {
         const unsigned short a = (unsigned short)__shfl_sync(gmask, vc, j, LPR);
         uint32_t wv[4];
         asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
@@ -309,10 +304,10 @@ nm_status check_spmm_args(const nm_packed* P, const void* PX, int64_t ldx, float
 // (spmm_sm100.cu).  format 0 = the pack's choice (nm_packed::sptc_format), 1 = full,
 // 2 = compressed.
 nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
-                           cudaStream_t s, int format) {
+                           cudaStream_t s, int format, bool fuse_residual) {
   if (format == 0) format = P->sptc_format;
   if (format == 2) return launch_spmm_sptc_compressed(P, PX, ldx, Yp, ldy, F, s);
-  return launch_spmm_sptc_full(P, PX, ldx, Yp, ldy, F, s);
+  return launch_spmm_sptc_full(P, PX, ldx, Yp, ldy, F, s, fuse_residual);
 }
 
 nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
@@ -419,8 +414,11 @@ nm_status nm_spmm(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, in
                   void* stream) {
   nm_status st = check_spmm_args(P, PX, ldx, Yp, ldy, F);
   if (st != NM_OK) return st;
-  st = launch_spmm_sptc(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream, 0);
-  if (st != NM_OK) return st;
+  // full-record packs run the residual inside the tensor-core kernel (one launch); the
+  // compressed-record path keeps the separate residual kernel
+  const bool fused = P->sptc_format != 2 && P->image_full && P->res_items;
+  st = launch_spmm_sptc(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream, 0, fused);
+  if (st != NM_OK || fused) return st;
   return launch_spmm_residual(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream);
 }
 

@@ -63,16 +63,18 @@ def _run(world, rank, balanced):
     layers = [(bf(W), torch.from_numpy(b).to(dev), relu) for W, b, relu in ((Ws[0], bs[0], True), (Ws[1], bs[1], False))]
 
     def local_layer(li, Hf, W, b, relu, a, z):
-        Hd = Hf.to(dev).view(torch.bfloat16)
+        Hd = Hf.view(torch.int16).to(dev).view(torch.bfloat16)
         out = torch.empty((z - a, W.shape[1]), dtype=torch.bfloat16, device=dev)
         ws = torch.empty(api.gcn_workspace_bytes(n, W.shape[0], W.shape[1]), dtype=torch.uint8, device=dev)
         api.gcn_layer(P, Hd, W, b, out, ws, relu=relu, order="linear")
         torch.cuda.synchronize()
-        return out.view(torch.int16).cpu()  # gloo collectives run on host tensors
+        # gloo collectives run on host tensors and have no 16-bit types: ship the bf16 bits as
+        # int32 pairs (F is even), bit-exact
+        return out.view(torch.int16).cpu().view(torch.int32)
 
-    Hp = bf(H[perm]).view(torch.int16).cpu()
+    Hp = bf(H[perm]).view(torch.int16).cpu().view(torch.int32)
     out = nmdist.gcn_forward(Hp, layers, local_layer, bounds=bounds)
-    return out.numpy().copy(), perm
+    return out.view(torch.int16).numpy().copy(), perm
 
 
 def _worker(rank, world, port, balanced, q):
@@ -101,7 +103,7 @@ def test_gcn_forward_world2_bitwise_equals_world1(balanced):
     procs = [ctx.Process(target=_worker, args=(r, 2, port, balanced, q)) for r in range(2)]
     for p in procs:
         p.start()
-    got = dict(q.get(timeout=600) for _ in range(2))
+    got = dict(q.get(timeout=300) for _ in range(2))
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0

@@ -37,6 +37,7 @@ __global__ void __launch_bounds__(128, 1) peak_kernel(int sparse, int N, int nac
   uint8_t* s = (uint8_t*)(((uintptr_t)sm + 1023) & ~(uintptr_t)1023);
   __shared__ uint32_t tslot;
   __shared__ __align__(8) uint64_t bar;
+  __shared__ __align__(8) uint64_t bar_end;
   const int warp = threadIdx.x / 32;
   for (int i = threadIdx.x; i < 48 * 1024 / 4; i += 128) ((uint32_t*)s)[i] = 0x3c003c00u;  // 1.0 halves
   if (warp == 0) {
@@ -45,6 +46,7 @@ __global__ void __launch_bounds__(128, 1) peak_kernel(int sparse, int N, int nac
   }
   if (threadIdx.x == 0) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar)));
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar_end)));
     asm volatile("fence.mbarrier_init.release.cluster;");
   }
   asm volatile("fence.proxy.async.shared::cta;");
@@ -86,7 +88,7 @@ __global__ void __launch_bounds__(128, 1) peak_kernel(int sparse, int N, int nac
             "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, q;\n\t}" ::"r"(dcol),
             "l"(ad), "l"(bd), "r"(idesc), "r"(en)
             : "memory");
-      if ((i + 1) % cgroup == 0 && i + 1 < iters)
+      if ((i + 1) % cgroup == 0)
         asm volatile(
             "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
             "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(
@@ -94,22 +96,21 @@ __global__ void __launch_bounds__(128, 1) peak_kernel(int sparse, int N, int nac
             : "memory");
       if (++acc == nacc) acc = 0;
     }
-    // final commit: tracks completion of every MMA issued by this thread
+    // final commit on its own barrier (one phase): completes when every MMA issued by this
+    // thread has completed.  (Waiting for the intermediate commits by phase parity can alias
+    // phases and hang -- the first version of this probe did.)
     asm volatile(
         "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
-        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(su32(&bar))
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(su32(&bar_end))
         : "memory");
-    // wait until every commit arrived: the barrier has count 1, so each commit completes one
-    // phase; the number of phases = number of commits
-    const int ncommit = (iters - 1) / cgroup + 1;
-    for (int k = 0; k < ncommit; ++k) {
-      uint32_t done = 0;
-      while (!done)
-        asm volatile(
-            "{\n\t.reg .pred q;\n\tmbarrier.try_wait.parity.shared::cta.b64 q, [%1], %2;\n\tselp.b32 %0, 1, 0, q;\n\t}"
-            : "=r"(done)
-            : "r"(su32(&bar)), "r"((uint32_t)(k & 1)));
-    }
+    uint32_t done = 0;
+    const uint64_t deadline = gtime() + 2000000000ull;  // 2 s watchdog
+    while (!done && gtime() < deadline)
+      asm volatile(
+          "{\n\t.reg .pred q;\n\tmbarrier.try_wait.parity.shared::cta.b64 q, [%1], 0;\n\tselp.b32 %0, 1, 0, q;\n\t}"
+          : "=r"(done)
+          : "r"(su32(&bar_end)));
+    if (!done && threadIdx.x == 32) printf("CTA %d: watchdog expired\n", blockIdx.x);
     const long long c1 = clock64();
     const uint64_t t1 = gtime();
     if (threadIdx.x == 32) {
