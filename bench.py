@@ -386,38 +386,28 @@ def main():
     stream = torch.cuda.current_stream()
     has_res = info["residual_nnz"] > 0
 
-    # full-record packs run the residual inside the tensor-core kernel (nm_spmm: ONE launch,
-    # k_spmm_full with its residual warps); the compressed-record kernel keeps the separate
-    # k_residual launch
-    fused = args.sptc_format in (0, 1)
-
+    # nm_spmm = the tensor-core kernel, then the residual kernel (stream-ordered); the two are
+    # timed separately here (a residual fused into the tensor-core kernel was measured slower,
+    # DESIGN.md §6)
     def step(ev=None):
         if args.order == "original":
             if ev: ev[0].record(stream)
-            if fused:
-                api.spmm(P, X, Y)
-                if ev: ev[1].record(stream)
-            else:
-                api.spmm(P, X, Y, part="sptc", format=args.sptc_format)
-                if ev: ev[1].record(stream)
-                if has_res:
-                    api.spmm(P, X, Y, part="residual")
+            api.spmm(P, X, Y, part="sptc", format=args.sptc_format)
+            if ev: ev[1].record(stream)
+            if has_res:
+                api.spmm(P, X, Y, part="residual")
             if ev: ev[2].record(stream)
         else:
             if ev: ev[0].record(stream)
             api.permute_rows(X, PX, perm_d, dt)
-            if fused:
-                api.spmm(P, PX, Yp)
-                if ev: ev[1].record(stream)
-            else:
-                api.spmm(P, PX, Yp, part="sptc", format=args.sptc_format)
-                if ev: ev[1].record(stream)
-                if has_res:
-                    api.spmm(P, PX, Yp, part="residual")
+            api.spmm(P, PX, Yp, part="sptc", format=args.sptc_format)
+            if ev: ev[1].record(stream)
+            if has_res:
+                api.spmm(P, PX, Yp, part="residual")
             api.unpermute_rows(Yp, Y, perm_d[rb:re], "f32")
             if ev: ev[2].record(stream)
 
-    launches_per_step = (1 if fused else 1 + int(has_res)) + (2 if args.order == "permuted" else 0)
+    launches_per_step = 1 + int(has_res) + (2 if args.order == "permuted" else 0)
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
@@ -486,18 +476,10 @@ def main():
                   "mma_flop": 2.0 * chunks * nft * 128 * BN * 32}
     res_terms = {"hbm_bytes": res["res_nnz"] * 6 + (rows_b + 1) * 8 + res_rows * F * 8,
                  "l2_bytes": res["res_nnz"] * F * 2, "mma_flop": 0.0} if has_res else None
-    if fused:  # one kernel: the tensor-core part and the residual share its time
-        kd0 = dict(sptc_terms)
-        if res_terms:  # + (col, val) and row pointers, the residual rows' Y write (the epilogue
-            #            re-reads them from L2 and writes the final Y once), the X row gathers
-            kd0["hbm_bytes"] += res["res_nnz"] * 6 + (rows_b + 1) * 8 + res_rows * F * 4
-            kd0["l2_bytes"] += res_terms["l2_bytes"]
-        kern = {"k_spmm_full+residual": dict(kd0, ms=statistics.mean(sptc_ms), format="full, fused residual")}
-    else:
-        kern = {"k_spmm_sptc": dict(sptc_terms, ms=statistics.mean(sptc_ms),
-                                    format="full" if fmt != 2 else "compressed")}
-        if has_res:
-            kern["k_residual"] = dict(res_terms, ms=statistics.mean(b - a for a, b in zip(sptc_ms, step_ms)))
+    kern = {"k_spmm_sptc": dict(sptc_terms, ms=statistics.mean(sptc_ms),
+                                format="full" if fmt != 2 else "compressed")}
+    if has_res:
+        kern["k_residual"] = dict(res_terms, ms=statistics.mean(b - a for a, b in zip(sptc_ms, step_ms)))
     for k in kern.values():
         t = {"hbm": k["hbm_bytes"] / (hbm_gbs * 1e9) * 1e3, "l2": k["l2_bytes"] / (l2_gbs * 1e9) * 1e3,
              "tensor": k["mma_flop"] / (sp_tf * 1e12) * 1e3}

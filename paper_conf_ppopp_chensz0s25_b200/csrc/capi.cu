@@ -221,8 +221,7 @@ void nm_packed_free(nm_packed* P) {
   cudaSetDevice(P->device);
   void* ptrs[] = {P->panel_mb_ptr, P->panel_chunk_ptr, P->unit_info, P->mb_seg, P->mb_sel,
                   P->image, P->res_rowptr, P->res_col, P->res_val, P->row_map,
-                  P->res_gather, P->res_segs, P->rec_len16, P->image_full, P->cta_ptr,
-                  P->res_items, P->res_pptr, P->res_psplit, P->res_rowmask};
+                  P->res_gather, P->res_segs, P->rec_len16, P->image_full, P->cta_ptr};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   cudaSetDevice(cur);

@@ -112,13 +112,6 @@ struct nm_packed {
   // by each nm_spmm call on its stream
   nm::ResSeg* res_segs = nullptr;      // [n_res_segs]
   int64_t n_res_segs = 0, n_res_slots = 0, n_res_split = 0;
-  // the same items in panel order for the residual fused into the full-record kernel: per
-  // panel the split rows' items (grouped by row, in item order), then single-item rows
-  // longest first; res_rowmask bit r of panel p = row 128p + r has residual entries
-  nm::ResSeg* res_items = nullptr;     // [n_res_segs]
-  int64_t* res_pptr = nullptr;         // [n_panels + 1]
-  int64_t* res_psplit = nullptr;       // [n_panels]
-  uint32_t* res_rowmask = nullptr;     // [n_panels * 4]
   size_t device_bytes = 0;
 };
 
@@ -191,9 +184,9 @@ uint16_t one_bits(nm_dtype dt);
 nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                            int64_t ldy, int F, cudaStream_t s);
 nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy,
-                           int F, cudaStream_t s, int format, bool fuse_residual = false);
+                           int F, cudaStream_t s, int format);
 nm_status launch_spmm_sptc_full(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
-                                int64_t ldy, int F, cudaStream_t s, bool fuse_residual);
+                                int64_t ldy, int F, cudaStream_t s);
 nm_status launch_spmm_sptc_compressed(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                                       int64_t ldy, int F, cudaStream_t s);
 nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,

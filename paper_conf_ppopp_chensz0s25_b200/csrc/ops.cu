@@ -304,10 +304,10 @@ nm_status check_spmm_args(const nm_packed* P, const void* PX, int64_t ldx, float
 // (spmm_sm100.cu).  format 0 = the pack's choice (nm_packed::sptc_format), 1 = full,
 // 2 = compressed.
 nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
-                           cudaStream_t s, int format, bool fuse_residual) {
+                           cudaStream_t s, int format) {
   if (format == 0) format = P->sptc_format;
   if (format == 2) return launch_spmm_sptc_compressed(P, PX, ldx, Yp, ldy, F, s);
-  return launch_spmm_sptc_full(P, PX, ldx, Yp, ldy, F, s, fuse_residual);
+  return launch_spmm_sptc_full(P, PX, ldx, Yp, ldy, F, s);
 }
 
 nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
@@ -414,11 +414,8 @@ nm_status nm_spmm(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, in
                   void* stream) {
   nm_status st = check_spmm_args(P, PX, ldx, Yp, ldy, F);
   if (st != NM_OK) return st;
-  // full-record packs run the residual inside the tensor-core kernel (one launch); the
-  // compressed-record path keeps the separate residual kernel
-  const bool fused = P->sptc_format != 2 && P->image_full && P->res_items;
-  st = launch_spmm_sptc(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream, 0, fused);
-  if (st != NM_OK || fused) return st;
+  st = launch_spmm_sptc(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream, 0);
+  if (st != NM_OK) return st;
   return launch_spmm_residual(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream);
 }
 

@@ -497,39 +497,6 @@ __global__ void k_seg_gather(const ResSeg* __restrict__ in, const int32_t* __res
     out[i] = in[idx[i]];
 }
 
-// panel-order key of a residual item for the fused kernel: panel, then the split rows' items
-// (grouped by row, in item order), then single-item rows longest first
-__global__ void k_pitem_key(const ResSeg* __restrict__ segs, int64_t n, uint64_t* __restrict__ key,
-                            int32_t* __restrict__ idx) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const ResSeg g = segs[i];
-    const uint64_t panel = (uint64_t)(g.row / kPanelRows);
-    key[i] = (panel << 40) | (g.nseg > 1 ? ((uint64_t)(g.row % kPanelRows) << 24) | (uint64_t)g.idx
-                                         : ((uint64_t)1 << 39) | (uint64_t)(0x7FFFFFFF - g.len));
-    idx[i] = (int32_t)i;
-  }
-}
-
-__global__ void k_pitem_count(const ResSeg* __restrict__ segs, int64_t n, int64_t* __restrict__ cnt,
-                              int64_t* __restrict__ nsplit, uint32_t* __restrict__ rowmask) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const ResSeg g = segs[i];
-    const int64_t panel = g.row / kPanelRows;
-    atomicAdd((unsigned long long*)&cnt[panel], 1ull);
-    if (g.nseg > 1) atomicAdd((unsigned long long*)&nsplit[panel], 1ull);
-    if (g.idx == 0) {
-      const int r = g.row % kPanelRows;
-      atomicOr(&rowmask[panel * 4 + r / 32], 1u << (r % 32));
-    }
-  }
-}
-
-__global__ void k_psplit(const int64_t* __restrict__ pptr, const int64_t* __restrict__ nsplit, int64_t P,
-                         int64_t* __restrict__ psplit) {
-  for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < P; r += (int64_t)gridDim.x * blockDim.x)
-    psplit[r] = pptr[r] + nsplit[r];
-}
-
 struct DevBuf {
   void* p = nullptr;
   cudaStream_t s = nullptr;
@@ -910,43 +877,6 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     }
     NM_CUDA(cudaGetLastError());
   }
-  // ---- 4b. the residual items in panel order (for the residual fused into k_spmm_full) ----
-  NM_TRY(palloc((void**)&Pk->res_pptr, sizeof(int64_t) * (P + 1)));
-  NM_TRY(palloc((void**)&Pk->res_psplit, sizeof(int64_t) * (P > 0 ? P : 1)));
-  NM_TRY(palloc((void**)&Pk->res_rowmask, sizeof(uint32_t) * 4 * (P > 0 ? P : 1)));
-  NM_TRY(palloc((void**)&Pk->res_items, sizeof(ResSeg) * (Pk->n_res_segs > 0 ? Pk->n_res_segs : 1)));
-  NM_CUDA(cudaMemsetAsync(Pk->res_rowmask, 0, sizeof(uint32_t) * 4 * (P > 0 ? P : 1), s));
-  {
-    const int64_t ni = Pk->n_res_segs;
-    DevBuf d_cnt2, d_nsp;
-    NM_TRY(dalloc(d_cnt2, sizeof(int64_t) * (P + 1), s));
-    NM_TRY(dalloc(d_nsp, sizeof(int64_t) * (P + 1), s));
-    NM_CUDA(cudaMemsetAsync(d_cnt2.p, 0, sizeof(int64_t) * (P + 1), s));
-    NM_CUDA(cudaMemsetAsync(d_nsp.p, 0, sizeof(int64_t) * (P + 1), s));
-    if (ni > 0) {
-      DevBuf d_k1, d_k2, d_i1, d_i2;
-      NM_TRY(dalloc(d_k1, sizeof(uint64_t) * ni, s));
-      NM_TRY(dalloc(d_k2, sizeof(uint64_t) * ni, s));
-      NM_TRY(dalloc(d_i1, sizeof(int32_t) * ni, s));
-      NM_TRY(dalloc(d_i2, sizeof(int32_t) * ni, s));
-      k_pitem_key<<<grid_for(ni, 256), 256, 0, s>>>(Pk->res_segs, ni, d_k1.as<uint64_t>(), d_i1.as<int32_t>());
-      size_t bytes = 0;
-      NM_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, bytes, d_k1.as<uint64_t>(), d_k2.as<uint64_t>(),
-                                              d_i1.as<int32_t>(), d_i2.as<int32_t>(), ni, 0, 64, s));
-      DevBuf tmp;
-      NM_TRY(dalloc(tmp, bytes, s));
-      NM_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, bytes, d_k1.as<uint64_t>(), d_k2.as<uint64_t>(),
-                                              d_i1.as<int32_t>(), d_i2.as<int32_t>(), ni, 0, 64, s));
-      k_seg_gather<<<grid_for(ni, 256), 256, 0, s>>>(Pk->res_segs, d_i2.as<int32_t>(), ni, Pk->res_items);
-      k_pitem_count<<<grid_for(ni, 256), 256, 0, s>>>(Pk->res_segs, ni, d_cnt2.as<int64_t>(), d_nsp.as<int64_t>(),
-                                                      Pk->res_rowmask);
-    }
-    NM_TRY(scan_excl(d_cnt2.as<int64_t>(), Pk->res_pptr, P + 1, s));
-    if (P > 0) k_psplit<<<grid_for(P, 256), 256, 0, s>>>(Pk->res_pptr, d_nsp.as<int64_t>(), P, Pk->res_psplit);
-    NM_CUDA(cudaGetLastError());
-    NM_CUDA(cudaStreamSynchronize(s));
-  }
-
   // ---- 5. compression of the records (HBM form) ----
   std::vector<int64_t> coff(n_chunks + 1, 0);
   {

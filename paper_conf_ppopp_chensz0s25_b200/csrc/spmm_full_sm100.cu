@@ -25,7 +25,6 @@
 // picks per pack (launch_spmm_sptc).
 #include <cuda.h>
 #include <cudaTypedefs.h>
-#include <cuda_fp16.h>
 
 #include "nm_internal.h"
 
@@ -45,9 +44,7 @@ constexpr int kFGroups = NM_FULL_GROUPS;            // gather groups (4 warps ea
 #define NM_FULL_MMA_ONLY_ON 0
 #endif
 constexpr int kWProd = 0, kWG0 = 1, kWMma = kWG0 + 4 * kFGroups, kWEpi0 = kWMma + 1;
-constexpr int kWRes0 = kWEpi0 + 4, kRW = 8;         // residual warps (fused residual CSR SpMM)
-constexpr int kFThreads = (kWRes0 + kRW) * 32;      // 22 warps
-constexpr int kRB = 4;                              // residual entries per cp.async batch
+constexpr int kFThreads = (kWEpi0 + 4) * 32;        // 14 warps
 constexpr int kGThreads = 128;                      // threads per gather group
 constexpr int kPfChunks = 24;                       // records L2-prefetched for the next unit
 
@@ -64,15 +61,6 @@ struct FullParams {
   int64_t rows;
   int n_ftiles;
   uint32_t idesc;
-  // fused residual (nm_spmm): per-panel work items, their (col, val), the rows of each panel
-  // that carry residual entries (the epilogue adds the tensor-core result into them)
-  int fuse;
-  const ResSeg* res_items;       // panel order: per panel the split rows' items, then single rows
-  const int64_t* res_pptr;       // [n_panels + 1]
-  const int64_t* res_psplit;     // [n_panels] first single-row item of each panel
-  const uint32_t* res_rowmask;   // [n_panels * 4]
-  const int32_t* res_col;        // X row per residual entry
-  const uint16_t* res_val;
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -135,18 +123,13 @@ struct FCfg {
   static constexpr int kBBytes = 32 * BN * 2;       // one chunk's 32 gathered rows x BN
   static constexpr int kRecBytes = kChunkBytes;     // A (4096) + metadata (512) + gather rows (128)
   static constexpr int kStageBytes = kCPS * (kBBytes + kRecBytes);
-  static constexpr int kLPR = BN / 8;               // residual lanes per row (8 features each)
-  static constexpr int kRSub = 32 / kLPR;            // residual subgroups per warp
-  static constexpr int kRNSub = kRW * kRSub;          // residual subgroups per CTA
-  static constexpr int kResRing = kRW * 32 * 2 * kRB * 16;   // cp.async rings (2 batches per subgroup)
-  static constexpr int kResPart = kRNSub * kLPR * 8 * 4;      // split-row partial sums
-  static constexpr int kStagesRaw = (222 * 1024 - 2048 - kResRing - kResPart) / kStageBytes;
+  static constexpr int kStagesRaw = (222 * 1024 - 2048) / kStageBytes;
   static constexpr int kMaxStages = NM_FULL_MAX_STAGES / kCPS;
   static constexpr int kStages = ((kStagesRaw > kMaxStages ? kMaxStages : kStagesRaw) / kFGroups) * kFGroups;
   static constexpr int kMetaCols = kCPS * kStages;
   static constexpr int kNAcc = (3 * BN + kMetaCols <= 512) ? 3 : (2 * BN + kMetaCols <= 512) ? 2 : 1;
   static constexpr int kMeta0 = kNAcc * BN;         // metadata column of (stage s, chunk j): kMeta0 + kCPS*s + j
-  static constexpr int kSmem = 1024 + kStages * kStageBytes + kResRing + kResPart + 1024;
+  static constexpr int kSmem = 1024 + kStages * kStageBytes + 1024;
   static_assert(kMeta0 + kMetaCols <= 512, "TMEM budget");
   static_assert(kRecBytes % 16 == 0, "bulk copy granularity");
   static_assert(kSmem <= 227 * 1024, "smem");
@@ -162,17 +145,13 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const uint32_t sB = smem_u32(smem);                          // stage s: CPS B tiles (SW128)
   const uint32_t sRec = sB + C::kStages * CPS * C::kBBytes;    // stage s: CPS adjacent records
-  uint8_t* res_ring = smem + C::kStages * C::kStageBytes;              // residual cp.async rings
-  float* res_part = (float*)(res_ring + C::kResRing);                    // split-row partials
-  uint64_t* bars = (uint64_t*)(res_ring + C::kResRing + C::kResPart);
+  uint64_t* bars = (uint64_t*)(smem + C::kStages * C::kStageBytes);
   uint64_t* full_rec = bars;                 // records landed (tx)
   uint64_t* full_b = full_rec + C::kStages;  // gathers landed + metadata written
   uint64_t* empty = full_b + C::kStages;     // MMAs done with the stage (tcgen05.commit)
   uint64_t* tfull = empty + C::kStages;      // accumulator ready
   uint64_t* tempty = tfull + 4;              // accumulator drained
-  uint64_t* rfull = tempty + 4;              // residual rows of a panel written (2-slot ring)
-  uint64_t* rempty = rfull + 2;              // ... and consumed by the epilogue
-  uint32_t* tmem_slot = (uint32_t*)(rempty + 2);
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 4);
   const uint32_t bRec = smem_u32(full_rec), bFull = smem_u32(full_b), bEmpty = smem_u32(empty);
   const uint32_t bTfull = smem_u32(tfull), bTempty = smem_u32(tempty);
   const int warp = threadIdx.x >> 5;
@@ -188,10 +167,6 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
     for (int a = 0; a < 4; ++a) {
       mbar_init(bTfull + 8 * a, 1);
       mbar_init(bTempty + 8 * a, 4);
-    }
-    for (int a = 0; a < 2; ++a) {
-      mbar_init(smem_u32(&rfull[a]), kRW);  // one arrival per residual warp
-      mbar_init(smem_u32(&rempty[a]), 4);   // one arrival per epilogue warp
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -406,7 +381,7 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
         if (++acc == C::kNAcc) { acc = 0; aphase ^= 1; }
       }
     }
-  } else if (warp < kWRes0) {
+  } else {
     // ------------------------------------------------------------ epilogue
     // tcgen05.ld 16x256b: thread t holds rows (t/4) and (t/4 + 8) of a 16-lane block, columns
     // 2*(t%4) + {0,1} of every 8-column repetition -> 8-byte stores, four threads complete a
@@ -417,26 +392,18 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
     uint32_t aphase = 0;
     const bool vec_ok = ((p.ldy & 1) == 0) && ((((uintptr_t)p.Y) & 7) == 0);
     int64_t c0 = pa < pz ? __ldg(p.panel_chunk_ptr + pa) : 0;
-    const uint32_t bRFull = smem_u32(rfull), bREmpty = smem_u32(rempty);
-    int rslot = 0;
-    uint32_t rph = 0;
     for (int pn = pa; pn < pz; ++pn) {
       const int64_t c1 = __ldg(p.panel_chunk_ptr + pn + 1);
       const bool has = c1 > c0;
       c0 = c1;
       int64_t orow[2][2];
-      bool radd[2][2];  // row carries residual entries: Y already holds them, add into it
-      const uint32_t rmask = p.fuse ? __ldg(p.res_rowmask + 4 * (int64_t)pn + quarter) : 0u;
 #pragma unroll
       for (int b = 0; b < 2; ++b)
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
-          const int rl = b * 16 + (lane >> 2) + 8 * h;  // row within the lane quarter
-          const int64_t g = (int64_t)pn * kPanelRows + quarter * 32 + rl;
+          const int64_t g = (int64_t)pn * kPanelRows + quarter * 32 + b * 16 + (lane >> 2) + 8 * h;
           orow[b][h] = g < p.rows ? (p.row_map ? (int64_t)__ldg(p.row_map + g) : g) : -1;
-          radd[b][h] = (rmask >> rl) & 1u;
         }
-      if (p.fuse) mbar_wait_sleep(bRFull + 8 * rslot, rph);  // the panel's residual rows are in Y
       for (int ft = 0; ft < nft; ++ft) {
         const bool full_tile = vec_ok && ft * BN + BN <= p.F;
         mbar_wait_sleep(bTfull + 8 * acc, aphase);
@@ -467,21 +434,6 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
             if (full_tile) {
               float* ylo = p.Y + olo * p.ldy + ft * BN + cc + cpair;
               float* yhi = p.Y + ohi * p.ldy + ft * BN + cc + cpair;
-              if (radd[b][0] | radd[b][1]) {  // residual rows: add into what the residual warps wrote
-#pragma unroll
-                for (int j = 0; j < 8; ++j) {
-                  if (radd[b][0]) {
-                    const float2 r = *(const float2*)(ylo + 8 * j);
-                    v[4 * j] = __float_as_uint(__uint_as_float(v[4 * j]) + r.x);
-                    v[4 * j + 1] = __float_as_uint(__uint_as_float(v[4 * j + 1]) + r.y);
-                  }
-                  if (radd[b][1]) {
-                    const float2 r = *(const float2*)(yhi + 8 * j);
-                    v[4 * j + 2] = __float_as_uint(__uint_as_float(v[4 * j + 2]) + r.x);
-                    v[4 * j + 3] = __float_as_uint(__uint_as_float(v[4 * j + 3]) + r.y);
-                  }
-                }
-              }
 #pragma unroll
               for (int j = 0; j < 8; ++j) {
                 if (olo >= 0)
@@ -496,16 +448,8 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
             for (int j = 0; j < 8; ++j) {
               const int col = ft * BN + cc + 8 * j + cpair;
               if (col >= p.F) continue;
-              float2 lo = make_float2(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]));
-              float2 hi = make_float2(__uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3]));
-              if (radd[b][0] && olo >= 0) {
-                lo.x += p.Y[olo * p.ldy + col];
-                if (col + 1 < p.F) lo.y += p.Y[olo * p.ldy + col + 1];
-              }
-              if (radd[b][1] && ohi >= 0) {
-                hi.x += p.Y[ohi * p.ldy + col];
-                if (col + 1 < p.F) hi.y += p.Y[ohi * p.ldy + col + 1];
-              }
+              const float2 lo = make_float2(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]));
+              const float2 hi = make_float2(__uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3]));
               if (vec_ok && col + 2 <= p.F) {
                 if (olo >= 0) __stcs((float2*)(p.Y + olo * p.ldy + col), lo);
                 if (ohi >= 0) __stcs((float2*)(p.Y + ohi * p.ldy + col), hi);
@@ -527,149 +471,6 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
         if (lane == 0) mbar_arrive(bTempty + 8 * acc);
         if (++acc == C::kNAcc) { acc = 0; aphase ^= 1; }
       }
-      if (p.fuse) {  // the panel's residual rows are consumed: the slot may take panel + 2
-        __syncwarp();
-        if (lane == 0) mbar_arrive(bREmpty + 8 * rslot);
-        if (++rslot == 2) { rslot = 0; rph ^= 1; }
-      }
-    }
-  } else {
-    // ------------------------------------------------------------ fused residual CSR SpMM
-    // Per panel of the CTA's range, the residual entries of its rows (k_residual's scheme,
-    // ops.cu): a row's sum is WRITTEN to Y (before the epilogue, which then adds the
-    // tensor-core result into the rows of res_rowmask).  Split rows (> 256 residual entries)
-    // are run by all residual subgroups together, their partials added in subgroup order
-    // through shared memory (deterministic, no atomics, no global workspace); single-item rows
-    // one subgroup each.  X rows arrive by cp.async into the subgroup's shared-memory ring, two
-    // batches of kRB entries in flight.
-    constexpr int LPR = C::kLPR, SUB = C::kRSub, NSUB = C::kRNSub;
-    const int rw = warp - kWRes0;
-    const int sub = lane / LPR, li = lane % LPR;
-    const int csub = rw * SUB + sub;
-    const unsigned gmask = LPR == 32 ? 0xffffffffu : (((1u << LPR) - 1u) << (sub * LPR));
-    const uint32_t ring = smem_u32(res_ring) + (uint32_t)((rw * 32 + lane) * 2 * kRB * 16);
-    const uint32_t bRFull = smem_u32(rfull), bREmpty = smem_u32(rempty);
-    const bool bf = (p.idesc >> 7) & 1u;
-    int rslot = 0;
-    uint32_t rph = 0;
-    auto item_sum = [&](const ResSeg& g, int f, float acc[8]) {
-      const uint32_t xbytes = f < p.F ? 16u : 0u;
-      const int nb = (g.len + kRB - 1) / kRB;
-      int32_t cn = 0;
-      uint32_t vn = 0u, vc;
-      if (li < kRB && li < g.len) {
-        cn = __ldg(p.res_col + g.kb + li);
-        vn = __ldg(p.res_val + g.kb + li);
-      }
-#pragma unroll
-      for (int j = 0; j < kRB; ++j) {
-        const int32_t cc = __shfl_sync(gmask, cn, j, LPR);
-        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(ring + j * 16),
-                     "l"(p.X + (int64_t)cc * p.ldx + (xbytes ? f : 0)), "r"(j < g.len ? xbytes : 0u)
-                     : "memory");
-      }
-      asm volatile("cp.async.commit_group;" ::: "memory");
-      for (int k = 0; k < nb; ++k) {
-        vc = vn;
-        if (k + 1 < nb) {
-          const int e1 = (k + 1) * kRB;
-          cn = 0;
-          vn = 0u;
-          if (li < kRB && e1 + li < g.len) {
-            cn = __ldg(p.res_col + g.kb + e1 + li);
-            vn = __ldg(p.res_val + g.kb + e1 + li);
-          }
-          const uint32_t rb = ring + ((k + 1) & 1) * kRB * 16;
-#pragma unroll
-          for (int j = 0; j < kRB; ++j) {
-            const int32_t cc = __shfl_sync(gmask, cn, j, LPR);
-            asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(rb + j * 16),
-                         "l"(p.X + (int64_t)cc * p.ldx + (xbytes ? f : 0)), "r"(e1 + j < g.len ? xbytes : 0u)
-                         : "memory");
-          }
-          asm volatile("cp.async.commit_group;" ::: "memory");
-          asm volatile("cp.async.wait_group 1;" ::: "memory");
-        } else {
-          asm volatile("cp.async.wait_group 0;" ::: "memory");
-        }
-        const uint32_t rb = ring + (k & 1) * kRB * 16;
-#pragma unroll
-        for (int j = 0; j < kRB; ++j) {
-          const uint32_t a = __shfl_sync(gmask, vc, j, LPR) & 0xFFFFu;
-          uint32_t wv[4];
-          asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
-                       : "=r"(wv[0]), "=r"(wv[1]), "=r"(wv[2]), "=r"(wv[3])
-                       : "r"(rb + j * 16));
-          const float af = bf ? __uint_as_float(a << 16) : __half2float(__ushort_as_half((unsigned short)a));
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            float x0, x1;
-            if (bf) {
-              x0 = __uint_as_float(wv[q] << 16);
-              x1 = __uint_as_float(wv[q] & 0xFFFF0000u);
-            } else {
-              x0 = __half2float(__ushort_as_half((unsigned short)(wv[q] & 0xFFFFu)));
-              x1 = __half2float(__ushort_as_half((unsigned short)(wv[q] >> 16)));
-            }
-            acc[2 * q] = fmaf(af, x0, acc[2 * q]);
-            acc[2 * q + 1] = fmaf(af, x1, acc[2 * q + 1]);
-          }
-        }
-      }
-    };
-    auto store_row = [&](int64_t yrow, int f, const float acc[8]) {
-      if (f >= p.F) return;
-      float* y = p.Y + yrow * p.ldy + f;
-      if (f + 8 <= p.F && (p.ldy & 3) == 0 && (((uintptr_t)p.Y) & 15) == 0) {
-        __stcg((float4*)y, make_float4(acc[0], acc[1], acc[2], acc[3]));
-        __stcg((float4*)(y + 4), make_float4(acc[4], acc[5], acc[6], acc[7]));
-      } else {
-#pragma unroll
-        for (int q = 0; q < 8; ++q)
-          if (f + q < p.F) y[q] = acc[q];
-      }
-    };
-    for (int pn = pa; pn < pz; ++pn) {
-      if (!p.fuse) break;
-      mbar_wait(bREmpty + 8 * rslot, rph ^ 1);  // the epilogue has consumed panel - 2's rows
-      const int64_t i0 = __ldg(p.res_pptr + pn), i1 = __ldg(p.res_pptr + pn + 1);
-      const int64_t is = __ldg(p.res_psplit + pn);
-      for (int ft = 0; ft < nft; ++ft) {  // slabs of LPR * 8 = BN features
-        const int f = ft * BN + li * 8;
-        // split rows: every subgroup takes every NSUB-th item of the row
-        for (int64_t j0 = i0; j0 < is;) {
-          const ResSeg g0 = p.res_items[j0];
-          const int nseg = g0.nseg;
-          float acc[8];
-#pragma unroll
-          for (int q = 0; q < 8; ++q) acc[q] = 0.f;
-          for (int t = csub; t < nseg; t += NSUB) item_sum(p.res_items[j0 + t], f, acc);
-#pragma unroll
-          for (int q = 0; q < 8; ++q) res_part[(csub * LPR + li) * 8 + q] = acc[q];
-          asm volatile("bar.sync 1, %0;" ::"r"(kRW * 32) : "memory");
-          const int tr = threadIdx.x - kWRes0 * 32;  // 0 .. kRW*32-1
-          if (tr < LPR * 8) {
-            const int ff = ft * BN + tr;
-            float sum = 0.f;
-            for (int k = 0; k < NSUB; ++k) sum += res_part[(k * LPR + tr / 8) * 8 + (tr & 7)];
-            if (ff < p.F) p.Y[(int64_t)g0.yrow * p.ldy + ff] = sum;
-          }
-          asm volatile("bar.sync 1, %0;" ::"r"(kRW * 32) : "memory");
-          j0 += nseg;
-        }
-        // single-item rows, one subgroup each (longest first)
-        for (int64_t j = is + csub; j < i1; j += NSUB) {
-          const ResSeg g = p.res_items[j];
-          float acc[8];
-#pragma unroll
-          for (int q = 0; q < 8; ++q) acc[q] = 0.f;
-          item_sum(g, f, acc);
-          store_row(g.yrow, f, acc);
-        }
-      }
-      __syncwarp();
-      if (lane == 0) mbar_arrive(bRFull + 8 * rslot);  // release: this warp's Y rows are written
-      if (++rslot == 2) { rslot = 0; rph ^= 1; }
     }
   }
 
@@ -694,7 +495,7 @@ uint32_t make_idesc_full(nm_dtype dt, int BN) {
 
 template <int BN>
 nm_status launch_full_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
-                         cudaStream_t s, bool fuse) {
+                         cudaStream_t s) {
   using C = FCfg<BN>;
   static int configured_dev = -1;
   int dev = 0;
@@ -716,13 +517,6 @@ nm_status launch_full_bn(const nm_packed* P, const void* PX, int64_t ldx, float*
   prm.rows = P->row_end - P->row_begin;
   prm.n_ftiles = (F + BN - 1) / BN;
   prm.idesc = make_idesc_full(P->dtype, BN);
-  prm.fuse = fuse && P->res_nnz > 0 && P->res_items != nullptr;
-  prm.res_items = P->res_items;
-  prm.res_pptr = P->res_pptr;
-  prm.res_psplit = P->res_psplit;
-  prm.res_rowmask = P->res_rowmask;
-  prm.res_col = P->res_gather ? P->res_gather : P->res_col;
-  prm.res_val = P->res_val;
   if (P->n_ctas < 1 || P->n_panels < 1) return NM_OK;
   k_spmm_full<BN><<<(unsigned)P->n_ctas, kFThreads, C::kSmem, s>>>(prm);
   NM_CUDA(cudaGetLastError());
@@ -732,11 +526,11 @@ nm_status launch_full_bn(const nm_packed* P, const void* PX, int64_t ldx, float*
 }  // namespace
 
 nm_status launch_spmm_sptc_full(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
-                                cudaStream_t s, bool fuse_residual) {
+                                cudaStream_t s) {
   if (!P->image_full) return fail(NM_ERR_UNSUPPORTED, "nm_spmm: the pack holds no full-record image");
-  if (F <= 64) return launch_full_bn<64>(P, PX, ldx, Yp, ldy, F, s, fuse_residual);
-  if (F <= 128) return launch_full_bn<128>(P, PX, ldx, Yp, ldy, F, s, fuse_residual);
-  return launch_full_bn<256>(P, PX, ldx, Yp, ldy, F, s, fuse_residual);
+  if (F <= 64) return launch_full_bn<64>(P, PX, ldx, Yp, ldy, F, s);
+  if (F <= 128) return launch_full_bn<128>(P, PX, ldx, Yp, ldy, F, s);
+  return launch_full_bn<256>(P, PX, ldx, Yp, ldy, F, s);
 }
 
 }  // namespace nm

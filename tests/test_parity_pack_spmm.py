@@ -395,42 +395,3 @@ def test_sptc_formats_agree_bitwise(kind, seed, V, M, F):
     Y_ref, E, _ = oracle.spmm(ip, ic, v64, x64)
     err = np.abs(outs[0].astype(np.float64) - Y_ref)
     assert (err <= TOL * E).all(), err.max()
-
-
-@pytest.mark.parametrize("graph", ["pl", "hub"])
-@pytest.mark.parametrize("F", [64, 128, 256, 300])
-def test_fused_residual_matches_two_kernel_path(graph, F):
-    """nm_spmm on a full-record pack runs the residual inside the tensor-core kernel (residual
-    warps write the residual rows' sums, the epilogue adds the tensor-core result).  It must
-    meet the oracle bound, and equal the two-launch path (nm_spmm_sptc + nm_spmm_residual)
-    bitwise where no row is split (the same per-row summation order and the same final add)."""
-    dev = _cuda()
-    if graph == "pl":
-        ip, ic = graphs.lmcl_graph(6000, 60000, 2.1, 4, 0.5, 71, self_loops=True)
-    else:
-        ip, ic = _star_plus_er(n=4000, hubs=(0, 17, 1234), m=12000, seed=72)
-    n = len(ip) - 1
-    dtype = "bf16"
-    perm = np.random.default_rng(73).permutation(n).astype(np.int32)
-    v32, bits, v64 = _values(ip, ic, dtype, 74)
-    xbits, x64 = graphs.round16(graphs.features(n, F, 75), dtype)
-    ldx = (F + 7) // 8 * 8
-    Xb = torch.zeros((n, ldx), dtype=torch.int16, device=dev)
-    Xb[:, :F] = torch.from_numpy(xbits.view(np.int16)).to(dev)
-    X = Xb.view(torch.bfloat16)[:, :F]
-    P = api.pack(ip, ic, perm, 1, 2, 4, dtype=dtype, val=v32, order="original", tau=4)
-    st = P.stats()
-    assert st["n_mb"] > 0 and st["residual_nnz"] > 0
-    Yf = torch.full((n, F), float("nan"), device=dev)
-    api.spmm(P, X, Yf)                                   # fused
-    Y2 = torch.full((n, F), float("nan"), device=dev)
-    api.spmm(P, X, Y2, part="sptc")
-    api.spmm(P, X, Y2, part="residual")                 # two launches
-    torch.cuda.synchronize()
-    Y_ref, E, _ = oracle.spmm(ip, ic, v64, x64)
-    yf = Yf.cpu().numpy()
-    assert (np.abs(yf.astype(np.float64) - Y_ref) <= TOL * E).all()
-    if st["residual_split_rows"] == 0:
-        assert np.array_equal(yf, Y2.cpu().numpy())
-    else:
-        np.testing.assert_allclose(yf, Y2.cpu().numpy(), rtol=1e-5, atol=1e-5)
