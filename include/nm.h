@@ -180,10 +180,11 @@ NM_API nm_status nm_pack_hybrid(const nm_csr* A, const int32_t* perm, int V, int
                                 nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags,
                                 int tau, void* stream, nm_packed** out);
 
-/* nm_hybrid_tau -- the tau nm_pack_hybrid should use for an SpMM with F feature columns:
- * the break-even number of kept values at which a meta-block's gathered X bytes (its 4
- * selected rows) equal those of the same values in the residual CSR (6 bytes + 1 gathered X
- * row each): ceil(8F / (2F + 6)), i.e. 4 for F >= 10.  DESIGN.md §6.  Returns 0 for F < 1. */
+/* nm_hybrid_tau -- the tau nm_pack_hybrid should use for an SpMM with F feature columns: the
+ * break-even number of kept values at which a meta-block's share of a tensor-core chunk costs
+ * as much time as the same values in the residual CSR, from a model fitted to B200
+ * measurements: ceil((0.28 + 0.0075 F) / (8 * 0.00016 F)), i.e. 8 at F = 128,
+ * 7 at F = 256.  Returns 0 for F < 1. */
 NM_API int nm_hybrid_tau(int F);
 
 /* Sizes: #meta-blocks, #values kept in MMA slots, #residual nonzeros, device bytes held,

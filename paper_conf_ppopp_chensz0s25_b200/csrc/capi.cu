@@ -198,20 +198,20 @@ const char* nm_last_error(void) { return g_last_error.c_str(); }
 
 int nm_version(void) { return 1; }
 
-// Hybrid-split threshold from a traffic model (reading #27): every byte either
-// path moves passes the L2 slices (LTS), which cap the whole chip's throughput, so compare
-// LTS bytes.  An emitted meta-block costs its share of a chunk record (kChunkBytes / 8) plus
-// its 4 gathered X rows (4 * 2F bytes); a residual value costs its column + value (6 bytes)
-// plus one gathered X row (2F bytes).  Blocks keeping fewer values than the break-even go to
-// the residual.
+// Hybrid-split threshold from a measured time model (reading #27): a meta-block
+// emitted to the tensor-core path costs an eighth of a K = 32 chunk, a residual value one
+// gathered X row.  Fitted on B200 (round 2, full-record kernel + cp.async residual, whole-GPU
+// times): a chunk costs ~0.28 + 0.0075 F ns (the MMA issue interval, ~242 cycles per
+// tcgen05.mma.sp, plus the 4736-B record and the gathers: C3 F = 128 1.24 ns, C4 F = 256
+// 2.2 ns); a residual value ~0.16 F ps (C3 21 ps, C4 40 ps).  Blocks keeping fewer values than
+// the break-even go to the residual: 8 at F = 128, 7 at F = 256, 10 at F = 64.  Measured tau
+// sweeps (profiles/r02_tau_sweep.txt): C4 best at 8, C3 128:2:16 at 6, C3 1:2:4 and C5 flat
+// between 4 and 12.
 int nm_hybrid_tau(int F) {
-  // break-even of the X-row traffic: a meta-block gathers its 4 selected X rows (8F bytes of
-  // 16-bit features) whatever it keeps, a residual value gathers one X row plus its 6-byte
-  // (col, value) entry.  The compressed chunk record adds only ~4 bytes per kept value, so it
-  // is left out; measured on B200: banded n = 2^20, F = 128 -> tau 2 / 3 / 5 / 7
-  // = 0.268 / 0.263 / 0.275 / 0.290 ms per step, and this model gives 4.
   if (F < 1) return 0;
-  return (int)ceil(8.0 * F / (2.0 * F + 6.0));
+  const double t_chunk = 0.28 + 0.0075 * F;   // ns
+  const double t_value = 0.00016 * F;         // ns
+  return (int)ceil(t_chunk / (8.0 * t_value));
 }
 
 void nm_packed_free(nm_packed* P) {

@@ -3,6 +3,8 @@
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 
+#include <mutex>
+
 #include "nm_internal.h"
 
 #ifndef NM_RES_UNROLL
@@ -193,7 +195,7 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
     }
     if (g.slot >= 0) {
       // split row: publish this item's partial, the last arrival reduces in item order
-      float* part = ws + ((int64_t)(g.slot + g.idx) * kResSlab) + li * 8;
+      float* part = ws + ((int64_t)(g.slot + g.idx) * (LPR * 8)) + li * 8;
       *(float4*)part = make_float4(acc[0], acc[1], acc[2], acc[3]);
       *(float4*)(part + 4) = make_float4(acc[4], acc[5], acc[6], acc[7]);
       __threadfence();
@@ -213,7 +215,7 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
           const int i = i0 + u;
           pa[u] = pb[u] = make_float4(0.f, 0.f, 0.f, 0.f);
           if (i < g.nseg) {
-            const float* pi = ws + ((int64_t)(g.slot + i) * kResSlab) + li * 8;
+            const float* pi = ws + ((int64_t)(g.slot + i) * (LPR * 8)) + li * 8;
             pa[u] = __ldcg((const float4*)pi);
             pb[u] = __ldcg((const float4*)(pi + 4));
           }
@@ -310,6 +312,32 @@ nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, floa
   return launch_spmm_sptc_full(P, PX, ldx, Yp, ldy, F, s);
 }
 
+// Per-device pool for the per-call residual workspace: allocations are stream-ordered (so calls
+// on different streams never share a buffer) and the pool keeps its memory between calls (the
+// device's default pool releases at every synchronisation, which made a large workspace cost a
+// fresh device allocation per call: C3 at tau = 8 spent 5 ms of its 6.3 ms residual there).
+// Library state, not handle state: the packed handle stays immutable.
+nm_status workspace_pool(cudaMemPool_t* out) {
+  static std::mutex mu;
+  static cudaMemPool_t pools[64] = {};
+  int dev = 0;
+  NM_CUDA(cudaGetDevice(&dev));
+  if (dev < 0 || dev >= 64) return fail(NM_ERR_UNSUPPORTED, "workspace_pool: device id >= 64");
+  std::lock_guard<std::mutex> lock(mu);
+  if (!pools[dev]) {
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.handleTypes = cudaMemHandleTypeNone;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    NM_CUDA(cudaMemPoolCreate(&pools[dev], &props));
+    uint64_t keep = UINT64_MAX;
+    NM_CUDA(cudaMemPoolSetAttribute(pools[dev], cudaMemPoolAttrReleaseThreshold, &keep));
+  }
+  *out = pools[dev];
+  return NM_OK;
+}
+
 nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
                                cudaStream_t s) {
   const int64_t rows = P->row_end - P->row_begin;
@@ -327,8 +355,10 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
   float* ws = nullptr;
   int32_t* cnt = nullptr;
   if (P->n_res_split > 0) {
-    NM_CUDA(cudaMallocAsync((void**)&ws, sizeof(float) * kResSlab * P->n_res_slots, s));
-    cudaError_t e = cudaMallocAsync((void**)&cnt, sizeof(int32_t) * P->n_res_split * nslab, s);
+    cudaMemPool_t pool;
+    NM_TRY_STATUS(workspace_pool(&pool));
+    NM_CUDA(cudaMallocFromPoolAsync((void**)&ws, sizeof(float) * lpr * 8 * P->n_res_slots, pool, s));
+    cudaError_t e = cudaMallocFromPoolAsync((void**)&cnt, sizeof(int32_t) * P->n_res_split * nslab, pool, s);
     if (e != cudaSuccess) {
       cudaFreeAsync(ws, s);
       return cuda_fail(e, "cudaMallocAsync(residual counters)");
