@@ -199,4 +199,12 @@ nm_status count_violations_dev(const DevCsr& A, const int32_t* perm_dev, int V, 
                                cudaStream_t s);
 nm_status stage1_sort_dev(const DevCsr& A, int32_t* perm_dev, int N, int M, cudaStream_t s);
 
+// Stage-2 gain tables on the device (reorder_gpu.cu): the tables of a primary segment against a
+// batch of targets, entry layout as the host's gain_table (2 int64 per (u, v), u-major).
+struct S2DeviceTables;
+nm_status s2dev_create(const DevCsr& A, int M, int max_batch, cudaStream_t s, S2DeviceTables** out);
+nm_status s2dev_set_perm(S2DeviceTables* t, const int32_t* perm_host);
+nm_status s2dev_tables(S2DeviceTables* t, int64_t p, const int64_t* targets, int nb, int N, int64_t* tabs_out);
+void s2dev_destroy(S2DeviceTables* t);
+
 }  // namespace nm

@@ -300,8 +300,11 @@ Pair pick_from_table(const int64_t* tab, int64_t n, int M, int64_t p, int64_t t,
   return best;
 }
 
+// dev != nullptr: the gain tables come from the device (s2dev_tables, reorder_gpu.cu) -- the
+// same integer sums, so the picks and the resulting order are identical to the host tables'
 int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>& iperm, int N, int M,
-               int maxiter, int gain_rule, int64_t* max_pairs) {
+               int maxiter, int gain_rule, int64_t* max_pairs, S2DeviceTables* dev, nm_status* err) {
+  *err = NM_OK;
   const int64_t n = g.n, S = (n + M - 1) / M;
   int64_t passes = 0;
   std::vector<int32_t> pscore;
@@ -330,6 +333,7 @@ int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>&
     std::fill(used.begin(), used.end(), 0);
     su.clear();
     sv.clear();
+    if (dev && (*err = s2dev_set_perm(dev, perm.data())) != NM_OK) return passes;
     if (I.size() == 1) {
       const int64_t p = I[0];
       if (S == 1) break;
@@ -340,10 +344,14 @@ int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>&
         for (int64_t q = s * M; q < std::min<int64_t>(n, s * M + M); ++q) z += g.deg(perm[q]);
         if (t < 0 || z < tn) { t = s; tn = z; }
       }
-      cp.build(g, perm, p, M);
-      ct.build(g, perm, t, M);
       std::vector<int64_t> tab(2 * (size_t)M * M);
-      gain_table(g, perm, cp, ct, N, M, p, t, used, tab.data());
+      if (dev) {
+        if ((*err = s2dev_tables(dev, p, &t, 1, N, tab.data())) != NM_OK) return passes;
+      } else {
+        cp.build(g, perm, p, M);
+        ct.build(g, perm, t, M);
+        gain_table(g, perm, cp, ct, N, M, p, t, used, tab.data());
+      }
       int64_t npairs = 0;
       for (;;) {
         Pair pr = pick_from_table(tab.data(), n, M, p, t, used, true);  // "beneficial" swaps
@@ -366,7 +374,7 @@ int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>&
         --live;
         // the targets are the live entries of I after the primary, walked lazily: only the
         // target being picked can leave I, so this equals a snapshot taken when p is popped
-        cp.build(g, perm, p, M);
+        if (!dev) cp.build(g, perm, p, M);
         int64_t npairs = 0;
         // targets in batches: their gain tables in parallel, the picks in target order.  Only
         // the target being picked can leave I, so the batch's membership filter is final.
@@ -379,8 +387,11 @@ int64_t stage2(const Graph& g, std::vector<int32_t>& perm, std::vector<int32_t>&
           batch = std::min<size_t>(batch * 2, 256);
           if (tabs.size() < tb.size() * 2 * M * M) tabs.resize(tb.size() * 2 * M * M);
           const int64_t nb = (int64_t)tb.size();
-#pragma omp parallel for schedule(dynamic, 1) num_threads(nthr) if (nb > 1)
-          for (int64_t b = 0; b < nb; ++b) {
+          if (dev) {
+            if ((*err = s2dev_tables(dev, p, tb.data(), (int)nb, N, tabs.data())) != NM_OK) return passes;
+          }
+#pragma omp parallel for schedule(dynamic, 1) num_threads(nthr) if (nb > 1 && !dev)
+          for (int64_t b = 0; b < (dev ? 0 : nb); ++b) {
 #ifdef _OPENMP
             SegCount& c = cts[omp_get_thread_num()];
 #else
@@ -429,6 +440,7 @@ namespace {
 // stays on the host (its greedy is sequential in the recorded pairs).
 struct Backend {
   virtual ~Backend() {}
+  virtual S2DeviceTables* stage2_tables(int /*M*/, nm_status* st) { *st = NM_OK; return nullptr; }
   virtual nm_status stage1(std::vector<int32_t>& perm, std::vector<int32_t>& iperm, int N, int M) = 0;
   virtual nm_status counts(const std::vector<int32_t>& perm, const std::vector<int32_t>& iperm, int V, int N,
                            int M, int64_t* w, int64_t* mb) = 0;
@@ -454,8 +466,25 @@ struct DeviceBackend : Backend {
   const DevCsr& d;
   cudaStream_t s;
   int32_t* dperm = nullptr;
+  S2DeviceTables* s2 = nullptr;
+  int s2_M = 0;
   DeviceBackend(const DevCsr& d_, cudaStream_t s_) : d(d_), s(s_) {}
-  ~DeviceBackend() override { if (dperm) cudaFree(dperm); }
+  ~DeviceBackend() override {
+    if (dperm) cudaFree(dperm);
+    s2dev_destroy(s2);
+  }
+  S2DeviceTables* stage2_tables(int M, nm_status* st) override {
+    *st = NM_OK;
+    if (s2 && s2_M != M) {
+      s2dev_destroy(s2);
+      s2 = nullptr;
+    }
+    if (!s2) {
+      *st = s2dev_create(d, M, 256, s, &s2);  // 256 = the largest target batch of stage2()
+      s2_M = M;
+    }
+    return s2;
+  }
   nm_status upload(const std::vector<int32_t>& perm) {
     if (!dperm) NM_CUDA(cudaMalloc(&dperm, sizeof(int32_t) * d.n));
     NM_CUDA(cudaMemcpyAsync(dperm, perm.data(), sizeof(int32_t) * d.n, cudaMemcpyHostToDevice, s));
@@ -515,7 +544,12 @@ nm_status reorder_core(const Graph& g, Backend& be, int V, int N, int M, const n
       NM_TRY(be.counts(perm, iperm, V, N, M, &w1, &mb1));
     }
     auto tb = now();
-    stats.stage2_passes += stage2(g, perm, iperm, N, M, o.max_stage2, o.gain_rule, &stats.max_pairs_per_primary);
+    nm_status s2st = NM_OK;
+    S2DeviceTables* dev = be.stage2_tables(M, &s2st);
+    NM_TRY(s2st);
+    stats.stage2_passes +=
+        stage2(g, perm, iperm, N, M, o.max_stage2, o.gain_rule, &stats.max_pairs_per_primary, dev, &s2st);
+    NM_TRY(s2st);
     t_s1 += secs(ta, tb);
     t_s2 += secs(tb, now());
     ++it;

@@ -14,6 +14,8 @@
 //      rows' pair sequences — stability gives the "ties keep the current position" rule.
 #include <cub/cub.cuh>
 
+#include <cstring>
+
 #include "nm_internal.h"
 
 namespace nm {
@@ -200,6 +202,167 @@ nm_status stage1_sort_dev(const DevCsr& A, int32_t* perm_dev, int N, int M, cuda
   NM_CUDA(cudaMemcpyAsync(perm_dev, nperm.p, sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
   NM_CUDA(cudaGetLastError());
   NM_CUDA(cudaStreamSynchronize(s));
+  return NM_OK;
+}
+
+}  // namespace nm
+
+namespace nm {
+
+// ---------------------------------------------------------------------------------------------
+// Stage-2 gain tables on the device (Alg. 3 lines 11-14 "GetCandidates",
+// PAPER.md:L459-462; the paper's SOGRE computes them on the GPU, L484).  For a primary segment p
+// and a batch of targets t_1..t_nb, every entry (u, v) of the M x M table of (p, t_b) holds
+//   gp = sum_{w in N(x) \ N(y)} [c_p(w) > N] - [c_p(w) - 1 > N] + sum_{w in N(y) \ N(x)} [c_p(w) > N] - [c_p(w) + 1 > N]
+//   gt = sum_{w in N(x) \ N(y)} [c_t(w) > N] - [c_t(w) + 1 > N] + sum_{w in N(y) \ N(x)} [c_t(w) > N] - [c_t(w) - 1 > N]
+// with x = perm[u], y = perm[v] and c_s(w) = |N(w) ∩ {perm[q] : q in segment s}| -- the same
+// integer sums as the host gain_table (reorder.cpp), so the picks made from them are bit-exact.
+// c_s lives in one int32 array of n counters per segment of the batch, filled by scattering the
+// neighbour lists of the segment's M vertices and emptied the same way after the tables.
+// ---------------------------------------------------------------------------------------------
+namespace {
+
+__global__ void k_s2_count(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
+                           const int32_t* __restrict__ perm, int64_t n, int M, const int64_t* __restrict__ segs,
+                           int nseg, int32_t* __restrict__ cnt, int delta) {
+  // one warp per (segment k, position j)
+  const int64_t wid = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (wid >= (int64_t)nseg * M) return;
+  const int k = (int)(wid / M), j = (int)(wid % M);
+  const int64_t q = segs[k] * M + j;
+  if (q >= n) return;
+  const int32_t x = perm[q];
+  int32_t* c = cnt + (int64_t)k * n;
+  for (int64_t e = rp[x] + lane; e < rp[x + 1]; e += 32) atomicAdd(&c[ci[e]], delta);
+}
+
+__device__ __forceinline__ bool in_sorted(const int32_t* __restrict__ a, int64_t len, int32_t v) {
+  int64_t lo = 0, hi = len;
+  while (lo < hi) {
+    const int64_t mid = (lo + hi) >> 1;
+    if (a[mid] < v) lo = mid + 1; else hi = mid;
+  }
+  return lo < len && a[lo] == v;
+}
+
+__global__ void k_s2_gain(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
+                          const int32_t* __restrict__ perm, int64_t n, int N, int M, const int64_t* __restrict__ segs,
+                          int nb, const int32_t* __restrict__ cnt, int64_t* __restrict__ tabs) {
+  // one warp per (target b, u, v) entry
+  const int64_t wid = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (wid >= (int64_t)nb * M * M) return;
+  const int b = (int)(wid / (M * M)), r = (int)(wid % (M * M)), i = r / M, j = r % M;
+  const int64_t u = segs[0] * M + i, v = segs[b + 1] * M + j;
+  int64_t* e = tabs + 2 * ((int64_t)b * M * M + r);
+  if (u >= n || v >= n) {
+    if (lane == 0) e[0] = e[1] = 0;
+    return;
+  }
+  const int32_t x = perm[u], y = perm[v];
+  const int32_t* cp = cnt;
+  const int32_t* ct = cnt + (int64_t)(b + 1) * n;
+  const int32_t* nx = ci + rp[x];
+  const int32_t* ny = ci + rp[y];
+  const int64_t dx = rp[x + 1] - rp[x], dy = rp[y + 1] - rp[y];
+  long long sp = 0, st = 0;
+  for (int64_t k = lane; k < dx; k += 32) {  // w in N(x) \ N(y): x's column leaves p (d = -1)
+    const int32_t w = nx[k];
+    if (in_sorted(ny, dy, w)) continue;
+    const int c1 = cp[w], c2 = ct[w];
+    sp += (c1 > N) - (c1 - 1 > N);
+    st += (c2 > N) - (c2 + 1 > N);
+  }
+  for (int64_t k = lane; k < dy; k += 32) {  // w in N(y) \ N(x): y's column enters p (d = +1)
+    const int32_t w = ny[k];
+    if (in_sorted(nx, dx, w)) continue;
+    const int c1 = cp[w], c2 = ct[w];
+    sp += (c1 > N) - (c1 + 1 > N);
+    st += (c2 > N) - (c2 - 1 > N);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    sp += __shfl_down_sync(0xffffffffu, sp, o);
+    st += __shfl_down_sync(0xffffffffu, st, o);
+  }
+  if (lane == 0) {
+    e[0] = sp;
+    e[1] = st;
+  }
+}
+
+}  // namespace
+
+struct S2DeviceTables {
+  const DevCsr* A = nullptr;
+  cudaStream_t s = nullptr;
+  int M = 0, max_batch = 0;
+  int32_t* perm = nullptr;   // pass-start order
+  int32_t* cnt = nullptr;    // (max_batch + 1) x n counters, zero between calls
+  int64_t* segs = nullptr;   // [max_batch + 1]
+  int64_t* tabs = nullptr;   // [max_batch * M * M * 2]
+  int64_t* h_segs = nullptr;  // pinned staging
+  int64_t* h_tabs = nullptr;
+};
+
+nm_status s2dev_create(const DevCsr& A, int M, int max_batch, cudaStream_t s, S2DeviceTables** out) {
+  S2DeviceTables* t = new S2DeviceTables();
+  t->A = &A;
+  t->s = s;
+  t->M = M;
+  t->max_batch = max_batch;
+  const size_t ntab = (size_t)max_batch * M * M * 2;
+  cudaError_t e = cudaMalloc(&t->perm, sizeof(int32_t) * A.n);
+  if (e == cudaSuccess) e = cudaMalloc(&t->cnt, sizeof(int32_t) * (size_t)(max_batch + 1) * A.n);
+  if (e == cudaSuccess) e = cudaMalloc(&t->segs, sizeof(int64_t) * (max_batch + 1));
+  if (e == cudaSuccess) e = cudaMalloc(&t->tabs, sizeof(int64_t) * ntab);
+  if (e == cudaSuccess) e = cudaMallocHost(&t->h_segs, sizeof(int64_t) * (max_batch + 1));
+  if (e == cudaSuccess) e = cudaMallocHost(&t->h_tabs, sizeof(int64_t) * ntab);
+  if (e == cudaSuccess) e = cudaMemsetAsync(t->cnt, 0, sizeof(int32_t) * (size_t)(max_batch + 1) * A.n, s);
+  if (e != cudaSuccess) {
+    s2dev_destroy(t);
+    return cuda_fail(e, "s2dev_create");
+  }
+  *out = t;
+  return NM_OK;
+}
+
+void s2dev_destroy(S2DeviceTables* t) {
+  if (!t) return;
+  if (t->s) cudaStreamSynchronize(t->s);
+  cudaFree(t->perm);
+  cudaFree(t->cnt);
+  cudaFree(t->segs);
+  cudaFree(t->tabs);
+  cudaFreeHost(t->h_segs);
+  cudaFreeHost(t->h_tabs);
+  delete t;
+}
+
+nm_status s2dev_set_perm(S2DeviceTables* t, const int32_t* perm_host) {
+  NM_CUDA(cudaMemcpyAsync(t->perm, perm_host, sizeof(int32_t) * t->A->n, cudaMemcpyHostToDevice, t->s));
+  return NM_OK;
+}
+
+nm_status s2dev_tables(S2DeviceTables* t, int64_t p, const int64_t* targets, int nb, int N, int64_t* tabs_out) {
+  if (nb < 1) return NM_OK;
+  if (nb > t->max_batch) return fail(NM_ERR_INVALID_ARG, "s2dev_tables: batch too large");
+  const DevCsr& A = *t->A;
+  const int M = t->M;
+  t->h_segs[0] = p;
+  for (int b = 0; b < nb; ++b) t->h_segs[b + 1] = targets[b];
+  NM_CUDA(cudaMemcpyAsync(t->segs, t->h_segs, sizeof(int64_t) * (nb + 1), cudaMemcpyHostToDevice, t->s));
+  const int B = 256;
+  const int64_t wc = (int64_t)(nb + 1) * M, wg = (int64_t)nb * M * M;
+  k_s2_count<<<(unsigned)((wc * 32 + B - 1) / B), B, 0, t->s>>>(A.rp, A.ci, t->perm, A.n, M, t->segs, nb + 1, t->cnt, 1);
+  k_s2_gain<<<(unsigned)((wg * 32 + B - 1) / B), B, 0, t->s>>>(A.rp, A.ci, t->perm, A.n, N, M, t->segs, nb, t->cnt,
+                                                                t->tabs);
+  k_s2_count<<<(unsigned)((wc * 32 + B - 1) / B), B, 0, t->s>>>(A.rp, A.ci, t->perm, A.n, M, t->segs, nb + 1, t->cnt, -1);
+  NM_CUDA(cudaGetLastError());
+  NM_CUDA(cudaMemcpyAsync(t->h_tabs, t->tabs, sizeof(int64_t) * wg * 2, cudaMemcpyDeviceToHost, t->s));
+  NM_CUDA(cudaStreamSynchronize(t->s));
+  memcpy(tabs_out, t->h_tabs, sizeof(int64_t) * wg * 2);
   return NM_OK;
 }
 

@@ -1,5 +1,8 @@
-"""Host nm_reorder vs nm_reorder_gpu (Stage-1 + counts on the device) on larger graphs: wall
-time and bit-identity of the two permutations.  usage: python tools/reorder_timing.py [out.jsonl]"""
+"""nm_reorder (host Stage-1 + host Stage-2 gain tables) vs nm_reorder_gpu (Stage-1, the counts and
+the Stage-2 gain tables on the device, the picks on the host): wall time, bit-identity of the two
+permutations, violation removal -- on graphs shaped like the paper's workloads, compared with
+Table 7's reordering times (0.01-30.55 s).
+usage: python tools/reorder_timing.py [out.jsonl]"""
 import json
 import os
 import sys
@@ -10,28 +13,43 @@ import torch  # noqa: E402
 
 from paper_conf_ppopp_chensz0s25_b200 import api, graphs  # noqa: E402
 
-CASES = [("band", 262144, 16, 64, 8, 2), ("band", 1048576, 16, 128, 16, 1),
-         ("pl", 262144, 16, 128, 16, 1), ("pl", 65536, 16, 64, 8, 1)]
+# (name, graph builder, V, M, reorder options, run the host version too)
+CASES = [
+    ("banded n=262k d=16", lambda: graphs.banded_graph(262144, 16, 21), 64, 8, dict(max_outer=2), True),
+    ("banded n=1M d=16", lambda: graphs.banded_graph(1 << 20, 16, 21), 1, 4, dict(max_outer=1), True),
+    ("power-law n=262k d=16", lambda: graphs.lmcl_graph(262144, 262144 * 8, 2.1, 1, 0.0, 21, scramble=True),
+     1, 4, dict(max_outer=1), True),
+    ("power-law n=65k d=16", lambda: graphs.lmcl_graph(65536, 65536 * 8, 2.1, 1, 0.0, 21, scramble=True),
+     64, 8, dict(max_outer=1), True),
+    ("C3 reddit 1:2:4, one Alg.1 iteration", lambda: graphs.gnn_graph("reddit"), 1, 4,
+     dict(max_outer=0, max_stage2=0), True),
+    ("C3 reddit 1:2:4, MAXITER = 10", lambda: graphs.gnn_graph("reddit"), 1, 4, dict(), False),
+    ("C4 proteins 128:2:16, MAXITER = 10", lambda: graphs.gnn_graph("proteins"), 128, 16, dict(), False),
+]
 
 
 def main():
     out = open(sys.argv[1], "w") if len(sys.argv) > 1 else None
     torch.cuda.init()
-    for kind, n, d, V, M, outer in CASES:
-        if kind == "band":
-            ip, ic = graphs.banded_graph(n, d, 21)
-        else:
-            ip, ic = graphs.lmcl_graph(n, n * d // 2, 2.1, 1, 0.0, 21, scramble=True)
+    cache = {}
+    for name, make, V, M, opts, host in CASES:
+        key = name.split(",")[0].split(" 1:2")[0]
+        if key not in cache:
+            cache = {key: make()}
+        ip, ic = cache[key]
         t = time.time()
-        pg, sg = api.reorder(ip, ic, V, 2, M, max_outer=outer, device=True)
+        pg, sg = api.reorder(ip, ic, V, 2, M, device=True, **opts)
         tg = time.time() - t
-        t = time.time()
-        ph, sh = api.reorder(ip, ic, V, 2, M, max_outer=outer)
-        th = time.time() - t
-        rec = {"graph": kind, "n": n, "nnz": int(len(ic)), "V": V, "M": M, "max_outer": outer,
-               "host_s": th, "gpu_s": tg, "identical": bool((pg == ph).all()),
-               "stage1_iters": sg["stage1_iters"], "mb": [sg["mb_init"], sg["mb_final"]],
-               "omega": [sg["omega_init"], sg["omega_final"]]}
+        rec = {"graph": name, "n": int(len(ip) - 1), "nnz": int(len(ic)), "V": V, "M": M, "opts": opts, "gpu_s": tg,
+               "omega": [sg["omega_init"], sg["omega_final"]], "mb": [sg["mb_init"], sg["mb_final"]],
+               "outer_iters": sg["outer_iters"], "stage1_iters": sg["stage1_iters"],
+               "stage2_passes": sg["stage2_passes"],
+               "violation_removal": None if sg["omega_init"] == 0 else 1 - sg["omega_final"] / sg["omega_init"]}
+        if host:
+            t = time.time()
+            ph, sh = api.reorder(ip, ic, V, 2, M, **opts)
+            rec["host_s"] = time.time() - t
+            rec["identical"] = bool((pg == ph).all())
         print(json.dumps(rec), flush=True)
         if out:
             out.write(json.dumps(rec) + "\n")
