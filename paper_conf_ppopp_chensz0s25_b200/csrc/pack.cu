@@ -483,10 +483,17 @@ __global__ void k_seg_fill(const int64_t* __restrict__ rrp, int64_t rows, const 
   }
 }
 
+#ifndef NM_RES_ORDER
+#define NM_RES_ORDER 0
+#endif
 __global__ void k_seg_key(const ResSeg* __restrict__ segs, int64_t n, uint32_t* __restrict__ key,
                           int32_t* __restrict__ idx) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+#if NM_RES_ORDER == 0
     key[i] = (uint32_t)(kResSeg - segs[i].len);  // ascending key = longest first
+#else
+    key[i] = segs[i].slot >= 0 ? 0u : 1u;  // split-row items first, then row order (stable)
+#endif
     idx[i] = (int32_t)i;
   }
 }
