@@ -119,16 +119,22 @@ def l2_gather_peak():
     return (best, "measured (tools/probes/probe_gather_rate.b200.txt)") if best else (18944.0, "fallback")
 
 
-def sparse_peak(bf16_tf):
-    """Sparse (2:4) tensor peak, logical TFLOP/s: tools/probes/probe_sparse_peak.b200.txt if it
-    holds a measurement, else 2x the measured dense bf16 rate (NVIDIA's 2:4 ratio), labelled so."""
-    p = os.path.join(ROOT, "tools", "probes", "probe_sparse_peak.b200.txt")
-    if os.path.exists(p):
-        import re
+def sparse_peak(bf16_tf, BN, sm_mhz):
+    """Sparse (2:4) tensor peak for the kernel's MMA shape (M = 128, N = BN, K = 32 logical), logical
+    TFLOP/s at the SM clock the bench ran at: the cycles per tcgen05.mma.sp that
+    tools/probes/probe_mma_issue.cu measured on B200 with the tensor pipe saturated (96 cycles at
+    N = 128, 160 at N = 256, 64 at N = 64) x 148 SMs.  Fallback: 2x the measured dense
+    bf16 rate (NVIDIA's 2:4 ratio), labelled so."""
+    import re
+    p = os.path.join(ROOT, "tools", "probes", "probe_mma_issue.b200.txt")
+    if os.path.exists(p) and sm_mhz:
         for ln in open(p):
-            m = re.match(r"BEST sparse ([\d.]+) TFLOP/s", ln)
-            if m and float(m.group(1)) > 0:
-                return float(m.group(1)), "measured (tools/probes/probe_sparse_peak.b200.txt)"
+            m = re.match(r"sparse N=\s*(\d+) unroll=1 A=noswzK B=sw128MN:\s*([\d.]+) cycles/MMA", ln)
+            if m and int(m.group(1)) == BN:
+                cyc = float(m.group(2))
+                tf = 2.0 * 128 * BN * 32 * 148 * sm_mhz * 1e6 / cyc / 1e12
+                return tf, "measured (tools/probes/probe_mma_issue.b200.txt: %.0f cycles per M128xN%dxK32 " \
+                           "MMA, at %.0f MHz)" % (cyc, BN, sm_mhz)
     return 2.0 * bf16_tf, "assumed 2x measured dense bf16"
 
 
@@ -201,14 +207,14 @@ class OracleSample:
     the same 16-bit-rounded A and X the GPU consumes, rows [0, rows) with rows sized so one
     pass takes ~budget_s seconds (never more than the whole matrix)."""
 
-    def __init__(self, ip, ic, vals, X32, dtype, budget_s):
+    def __init__(self, ip, ic, vals, X32, dtype, budget_s, threads=None):
         import oracle
         from paper_conf_ppopp_chensz0s25_b200 import graphs
         self.oracle = oracle
         self.ip, self.ic = ip, ic
         _, self.v64 = graphs.round16(vals, dtype)
         _, self.x64 = graphs.round16(X32, dtype)
-        self.cores = len(os.sched_getaffinity(0))
+        self.cores = threads or len(os.sched_getaffinity(0))
         n = len(ip) - 1
         rows = max(1, n // 256)
         dt = self._run(rows)[0]
@@ -236,6 +242,10 @@ def cpu_oracle_sample(ip, ic, vals, X32, dtype, budget_s=12.0, passes=3):
     runs = [s() for _ in range(passes)]
     best = sorted(runs, key=lambda r: r["value"])[len(runs) // 2]
     best["sample"] += " (median of %d passes)" % passes
+    # the same oracle on one thread, a smaller row block of ~3 s
+    one = OracleSample(ip, ic, vals, X32, dtype, 3.0, threads=1)()
+    best["single_thread"] = {"value": one["value"], "unit": one["unit"], "cores": one["cores"],
+                             "sample": one["sample"]}
     return best
 
 
@@ -470,7 +480,8 @@ def main():
     nft = (F + BN - 1) // BN
     rec_bytes = pst["full_image_bytes"] if fmt != 2 else pst["image_bytes"]
     l2_gbs, l2_src = l2_gather_peak()
-    sp_tf, sp_src = sparse_peak(bf16_tf)
+    clocks = clk.summary()
+    sp_tf, sp_src = sparse_peak(bf16_tf, BN, clocks.get("sm_mhz") or clocks.get("sm_max_mhz") or 1965.0)
     sptc_terms = {"hbm_bytes": rec_bytes + x_rows_sptc * F * 2 + rows_b * F * 4,
                   "l2_bytes": pst["gather_rows"] * F * 2 + rec_bytes * nft,
                   "mma_flop": 2.0 * chunks * nft * 128 * BN * 32}

@@ -130,14 +130,19 @@ NM_API nm_status nm_count_violations(const nm_csr* A, const int32_t* perm, int V
 
 /* ---------------------------------------------------------------------------------------
  * Packed V:N:M matrix (the SPTC form of L492).  Rows of B are grouped in
- * panels of Vp = 128 rows; columns in segments of Mp columns, Mp = 4 when V == 1 (2:4 at
+ * panels of Vp rows (the V-row meta-block height, L194); columns in segments of Mp columns,
+ * Mp = 4 when V == 1 (2:4 at
  * V = 1) and Mp = M otherwise; per non-empty (panel, segment) meta-block the k = 4 columns
  * with the most nonzeros are selected (vertical constraint, L226-227) and each row keeps
  * its first <= 2 nonzeros among them (N = 2, horizontal constraint L229-230) as two 16-bit
  * values plus a 4-bit index pair.  Everything else goes to a residual CSR.  Device memory
  * holds the MMA-native image consumed by nm_spmm (tcgen05.mma.sp operands).
- * Supported: N = 2; M in {4, 8, 16}; any V >= 1 (V = 1 -> Mp = 4); Vp = 128 (pass 0 or
- * 128); dtype NM_F16 or NM_BF16 (values are rounded from val_dtype to dtype).
+ * Supported: N = 2; M in {4, 8, 16}; any V >= 1 (V = 1 -> Mp = 4); Vp in {64, 128}
+ * (0 = auto: 64 when V == 64, else 128); dtype NM_F16 or NM_BF16 (values are rounded from
+ * val_dtype to dtype).  The tensor-core kernel always runs M = 128 MMAs over 128-row kernel
+ * panels; at Vp = 64 a kernel panel's chunks hold the meta-blocks of both of its 64-row
+ * panels (in canonical order), each k-group carrying the values of one half and no-value
+ * nibbles in the other, so a V = 64 conforming matrix packs with an empty residual.
  * ------------------------------------------------------------------------------------- */
 typedef struct nm_packed nm_packed;
 
@@ -197,7 +202,7 @@ NM_API nm_status nm_packed_info(const nm_packed* P, int64_t* n_mb, int64_t* pack
  * records of the default kernel (4736 B per K = 32 chunk); residual_items = work items of the
  * residual SpMM (<= 256 nonzeros each), residual_split_rows = rows cut into several. */
 typedef struct {
-  int64_t n, row_begin, row_end, n_panels, n_mb, n_chunks, packed_nnz, residual_nnz;
+  int64_t n, row_begin, row_end, n_panels /* 128-row kernel panels */, n_mb, n_chunks, packed_nnz, residual_nnz;
   int64_t image_bytes, device_bytes, residual_items, residual_split_rows;
   int32_t V, M, Mp, Vp, tau, flags;
   int64_t full_image_bytes;  /* full MMA-operand records (what the default kernel streams) */

@@ -127,13 +127,14 @@ class Packed:
         """nm_export_canonical -> dict of host arrays (residual_only: just the residual CSR)."""
         inf = self.info()
         m, r = inf["n_mb"], inf["residual_nnz"]
-        P = (self.rows + 127) // 128
+        Vp = int(self.stats()["Vp"])
+        P = (self.rows + Vp - 1) // Vp
         out = dict(res_rowptr=np.zeros(self.rows + 1, np.int64), res_col=np.zeros(max(r, 1), np.int32),
                    res_val=np.zeros(max(r, 1), np.uint16))
         if not residual_only:
             out.update(panel_ptr=np.zeros(P + 1, np.int64), mb_seg=np.zeros(max(m, 1), np.int32),
-                       sel=np.zeros(max(m, 1) * 4, np.uint8), nib=np.zeros(max(m, 1) * 128, np.uint8),
-                       vals=np.zeros(max(m, 1) * 256, np.uint16))
+                       sel=np.zeros(max(m, 1) * 4, np.uint8), nib=np.zeros(max(m, 1) * Vp, np.uint8),
+                       vals=np.zeros(max(m, 1) * Vp * 2, np.uint16))
         ptr = lambda k, t: out[k].ctypes.data_as(t) if k in out else None
         L.check(L.load().nm_export_canonical(
             self.handle, ptr("panel_ptr", L.P64), ptr("mb_seg", L.P32), ptr("sel", L.PU8), ptr("nib", L.PU8),
@@ -142,11 +143,11 @@ class Packed:
         if not residual_only:
             out["mb_seg"] = out["mb_seg"][:m]
             out["sel"] = out["sel"][:m * 4]
-            out["nib"] = out["nib"][:m * 128]
-            out["vals"] = out["vals"][:m * 256]
+            out["nib"] = out["nib"][:m * Vp]
+            out["vals"] = out["vals"][:m * Vp * 2]
         out["res_col"] = out["res_col"][:r]
         out["res_val"] = out["res_val"][:r]
-        out["n_mb"], out["res_nnz"] = m, r
+        out["n_mb"], out["res_nnz"], out["Vp"] = m, r, Vp
         return out
 
     def free(self):
@@ -162,11 +163,12 @@ class Packed:
 
 
 def pack(indptr, indices, perm, V: int, N: int, M: int, dtype="f16", val=None, val_dtype=None,
-         row_begin=None, row_end=None, stream=None, order="permuted", tau=0):
+         row_begin=None, row_end=None, stream=None, order="permuted", tau=0, Vp=0):
     """nm_pack / nm_pack_rows / nm_pack_ex / nm_pack_hybrid of B = P A P^T.  val: values per CSR
     entry (numpy, dtype val_dtype in {'f16','bf16' (uint16 bits),'f32'}) or None for a binary
     adjacency.  order='original' folds the permutation into the SpMM (NM_PACK_ORIGINAL_ORDER).
-    tau > 0: hybrid split (meta-blocks keeping fewer than tau values go to the residual)."""
+    tau > 0: hybrid split (meta-blocks keeping fewer than tau values go to the residual).
+    Vp: panel height, 64 or 128 (0 = the library's choice: 64 when V == 64, else 128)."""
     if val is not None and val_dtype is None:
         val_dtype = "f32" if val.dtype == np.float32 else ("f16" if val.dtype == np.float16 else "bf16")
     c, keep = _csr_struct(indptr, indices, val, val_dtype or "f16")
@@ -179,15 +181,15 @@ def pack(indptr, indices, perm, V: int, N: int, M: int, dtype="f16", val=None, v
     flags = L.NM_PACK_ORIGINAL_ORDER if order == "original" else 0
     lib = L.load()
     if tau:
-        L.check(lib.nm_pack_hybrid(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], rb, re, flags, int(tau), sp,
+        L.check(lib.nm_pack_hybrid(ctypes.byref(c), pp, V, N, M, int(Vp), _DT[dtype], rb, re, flags, int(tau), sp,
                                    ctypes.byref(h)), "nm_pack_hybrid")
     elif order == "original":
-        L.check(lib.nm_pack_ex(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], rb, re, flags, sp,
+        L.check(lib.nm_pack_ex(ctypes.byref(c), pp, V, N, M, int(Vp), _DT[dtype], rb, re, flags, sp,
                                ctypes.byref(h)), "nm_pack_ex")
     elif row_begin is None:
-        L.check(lib.nm_pack(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], sp, ctypes.byref(h)), "nm_pack")
+        L.check(lib.nm_pack(ctypes.byref(c), pp, V, N, M, int(Vp), _DT[dtype], sp, ctypes.byref(h)), "nm_pack")
     else:
-        L.check(lib.nm_pack_rows(ctypes.byref(c), pp, V, N, M, 128, _DT[dtype], rb, re, sp, ctypes.byref(h)),
+        L.check(lib.nm_pack_rows(ctypes.byref(c), pp, V, N, M, int(Vp), _DT[dtype], rb, re, sp, ctypes.byref(h)),
                 "nm_pack_rows")
     P = Packed(h, c.n, rb, re, dtype)
     P.order = order

@@ -3,6 +3,7 @@
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -272,12 +273,12 @@ nm_status nm_export_canonical(const nm_packed* P, int64_t* panel_ptr, int32_t* m
   NM_CUDA(cudaGetDevice(&cur));
   NM_CUDA(cudaSetDevice(P->device));
   const int64_t rows = P->row_end - P->row_begin;
-  std::vector<int64_t> mbp(P->n_panels + 1), chp(P->n_panels + 1);
-  NM_CUDA(cudaMemcpy(mbp.data(), P->panel_mb_ptr, sizeof(int64_t) * (P->n_panels + 1),
-                     cudaMemcpyDeviceToHost));
+  const int64_t Pc = P->n_cpanels, Vp = P->Vp, ratio = kPanelRows / P->Vp;
+  std::vector<int64_t> mbp(Pc + 1), chp(P->n_panels + 1);
+  NM_CUDA(cudaMemcpy(mbp.data(), P->panel_mb_ptr, sizeof(int64_t) * (Pc + 1), cudaMemcpyDeviceToHost));
   NM_CUDA(cudaMemcpy(chp.data(), P->panel_chunk_ptr, sizeof(int64_t) * (P->n_panels + 1),
                      cudaMemcpyDeviceToHost));
-  if (panel_ptr) memcpy(panel_ptr, mbp.data(), sizeof(int64_t) * (P->n_panels + 1));
+  if (panel_ptr) memcpy(panel_ptr, mbp.data(), sizeof(int64_t) * (Pc + 1));
   if (mb_seg && P->n_mb)
     NM_CUDA(cudaMemcpy(mb_seg, P->mb_seg, sizeof(int32_t) * P->n_mb, cudaMemcpyDeviceToHost));
   if (sel && P->n_mb) {
@@ -324,19 +325,25 @@ nm_status nm_export_canonical(const nm_packed* P, int64_t* panel_ptr, int32_t* m
         }
       }
     }
-    for (int64_t p = 0; p < P->n_panels; ++p) {
-      for (int64_t m = mbp[p]; m < mbp[p + 1]; ++m) {
-        int64_t local = m - mbp[p];
+    // canonical panel pc (Vp rows) = rows [(pc % ratio) * Vp, +Vp) of kernel panel pc / ratio,
+    // whose chunks hold the meta-blocks of its canonical panels in canonical order
+    for (int64_t pc = 0; pc < Pc; ++pc) {
+      const int64_t p = pc / ratio;
+      const int64_t kfirst = mbp[std::min(p * ratio, Pc)];
+      const int r0 = (int)(pc % ratio) * (int)Vp;
+      for (int64_t m = mbp[pc]; m < mbp[pc + 1]; ++m) {
+        int64_t local = m - kfirst;
         int64_t c = chp[p] + local / kChunkMB;
         int g = (int)(local % kChunkMB);
         const uint8_t* cv = img.data() + (size_t)c * kChunkBytes;
         const uint32_t* cm = (const uint32_t*)(cv + kChunkValBytes);
-        for (int r = 0; r < kPanelRows; ++r) {
+        for (int rc = 0; rc < Vp; ++rc) {
+          const int r = r0 + rc;
           int m0 = r % 8, m1 = (r / 8) % 2, m2 = r / 16, k1 = g / 4, q = g % 4;
           int lane = m0 + 8 * k1 + 16 * m2;
           uint32_t w = cm[lane];
           uint8_t nb = (uint8_t)((w >> (16 * m1 + 4 * q)) & 0xF);
-          if (nib) nib[m * kPanelRows + r] = nb;
+          if (nib) nib[m * Vp + rc] = nb;
           if (vals) {
             for (int slot = 0; slot < 2; ++slot) {
               int k = 2 * g + slot;
@@ -344,7 +351,7 @@ nm_status nm_export_canonical(const nm_packed* P, int64_t* panel_ptr, int32_t* m
                            (size_t)(k % 8) * 2;
               uint16_t v;
               memcpy(&v, cv + off, 2);
-              vals[(m * kPanelRows + r) * 2 + slot] = v;
+              vals[(m * Vp + rc) * 2 + slot] = v;
             }
           }
         }

@@ -84,10 +84,12 @@ struct nm_packed {
   int V = 1, N = 2, M = 4, Vp = 128, Mp = 4;
   int tau = 0;                         // hybrid split threshold (0 = plain canonical pack)
   nm_dtype dtype = NM_F16;
-  int64_t n_panels = 0, n_mb = 0, n_chunks = 0, packed_nnz = 0, res_nnz = 0;
+  // n_panels: kernel panels of kPanelRows (= MMA M = 128) rows; n_cpanels: canonical panels of
+  // Vp rows (Vp = 64: two per kernel panel, their meta-blocks share its chunks)
+  int64_t n_panels = 0, n_cpanels = 0, n_mb = 0, n_chunks = 0, packed_nnz = 0, res_nnz = 0;
   // device arrays
-  int64_t* panel_mb_ptr = nullptr;     // [n_panels+1]
-  int64_t* panel_chunk_ptr = nullptr;  // [n_panels+1]
+  int64_t* panel_mb_ptr = nullptr;     // [n_cpanels+1] first meta-block of each canonical panel
+  int64_t* panel_chunk_ptr = nullptr;  // [n_panels+1] first chunk of each kernel panel
   int4* unit_info = nullptr;           // [2 * n_panels] schedule: {panel, #chunks, first chunk lo, hi},
                                        //   {record byte offset lo, hi, record bytes lo, hi}
   uint16_t* rec_len16 = nullptr;       // [n_chunks] compressed record size / 16

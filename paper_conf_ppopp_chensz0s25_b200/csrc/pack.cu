@@ -83,14 +83,14 @@ __global__ void k_split_keys(const uint64_t* __restrict__ key, int32_t* __restri
     Bci[k] = (int32_t)(key[k] & 0xFFFFFFFFu);
 }
 
-// meta-block key of every entry: panel * S + col / Mp (warp per row)
+// meta-block key of every entry: (Vp-row panel) * S + col / Mp (warp per row)
 __global__ void k_mbkey(const int64_t* __restrict__ Brp, const int32_t* __restrict__ Bci,
-                        int64_t rows, int Mp, int64_t S, int64_t* __restrict__ key) {
+                        int64_t rows, int Vp, int Mp, int64_t S, int64_t* __restrict__ key) {
   int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kWarp;
   int lane = threadIdx.x % kWarp;
   int64_t nw = (int64_t)gridDim.x * blockDim.x / kWarp;
   for (int64_t l = warp; l < rows; l += nw) {
-    int64_t panel = l / kPanelRows;
+    int64_t panel = l / Vp;
     for (int64_t k = Brp[l] + lane; k < Brp[l + 1]; k += kWarp)
       key[k] = panel * S + Bci[k] / Mp;
   }
@@ -114,11 +114,19 @@ __global__ void k_panel_ptr(const int64_t* __restrict__ mbkey, int64_t n_mb, int
   }
 }
 
-__global__ void k_chunk_counts(const int64_t* __restrict__ mbp, int64_t P,
+// first meta-block of kernel panel R (kPanelRows rows = `ratio` canonical panels of Vp rows)
+__device__ __forceinline__ int64_t kpanel_mb(const int64_t* __restrict__ mbp, int64_t R, int ratio, int64_t Pc) {
+  const int64_t c = R * ratio;
+  return mbp[c < Pc ? c : Pc];
+}
+
+// chunks of every kernel panel: its meta-blocks (those of its `ratio` canonical panels, in
+// canonical order), kChunkMB per chunk
+__global__ void k_chunk_counts(const int64_t* __restrict__ mbp, int64_t P, int ratio, int64_t Pc,
                                int64_t* __restrict__ nchunk) {
   for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < P;
        r += (int64_t)gridDim.x * blockDim.x)
-    nchunk[r] = (mbp[r + 1] - mbp[r] + kChunkMB - 1) / kChunkMB;
+    nchunk[r] = (kpanel_mb(mbp, r + 1, ratio, Pc) - kpanel_mb(mbp, r, ratio, Pc) + kChunkMB - 1) / kChunkMB;
 }
 
 __global__ void k_meta_init(uint8_t* __restrict__ image, int64_t n_chunks) {
@@ -151,13 +159,13 @@ __global__ void k_xrow_map(const int32_t* __restrict__ perm, uint8_t* __restrict
 
 // per-entry meta-block id and column counts (warp per row)
 __global__ void k_colcount(const int64_t* __restrict__ Brp, const int32_t* __restrict__ Bci,
-                           int64_t rows, int Mp, int64_t S, const int64_t* __restrict__ mbkey,
+                           int64_t rows, int Vp, int Mp, int64_t S, const int64_t* __restrict__ mbkey,
                            int64_t n_mb, int32_t* __restrict__ cnt, int64_t* __restrict__ emb) {
   int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kWarp;
   int lane = threadIdx.x % kWarp;
   int64_t nw = (int64_t)gridDim.x * blockDim.x / kWarp;
   for (int64_t l = warp; l < rows; l += nw) {
-    int64_t panel = l / kPanelRows;
+    int64_t panel = l / Vp;
     for (int64_t k = Brp[l] + lane; k < Brp[l + 1]; k += kWarp) {
       int64_t s = Bci[k] / Mp;
       int64_t m = lower_bound64(mbkey, n_mb, panel * S + s);
@@ -276,16 +284,17 @@ __global__ void k_remap_emb(const int64_t* __restrict__ flag, const int64_t* __r
 // per emitted meta-block: segment id, selection and the X row of each logical k
 __global__ void k_write_sel(const int32_t* __restrict__ cnt, const int64_t* __restrict__ cand_of, int Mp,
                             int64_t n_mb, const int64_t* __restrict__ mbkey, int64_t S, int64_t n,
-                            const int64_t* __restrict__ mbp, const int64_t* __restrict__ chp,
+                            const int64_t* __restrict__ mbp, int ratio, int64_t Pc,
+                            const int64_t* __restrict__ chp,
                             int32_t* __restrict__ mb_seg, uint32_t* __restrict__ mb_sel,
                             uint8_t* __restrict__ image) {
   for (int64_t m = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; m < n_mb;
        m += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t panel = mbkey[m] / S, s = mbkey[m] % S;
+    const int64_t panel = mbkey[m] / S / ratio, s = mbkey[m] % S;  // kernel panel
     mb_seg[m] = (int32_t)s;
     const uint32_t sel = mb_sel[m];
     const int32_t* c = cnt + (cand_of ? cand_of[m] : m) * Mp;
-    const int64_t local = m - mbp[panel];
+    const int64_t local = m - kpanel_mb(mbp, panel, ratio, Pc);
     const int64_t chunk = chp[panel] + local / kChunkMB;
     const int g = (int)(local % kChunkMB);
     int32_t* xrow = (int32_t*)(image + chunk * kChunkBytes + kChunkXrowOff);
@@ -304,8 +313,8 @@ __global__ void k_write_sel(const int32_t* __restrict__ cnt, const int64_t* __re
 __global__ void k_place(const int64_t* __restrict__ Brp, const int32_t* __restrict__ Bci,
                         const uint16_t* __restrict__ Bval, int64_t rows, int Mp,
                         const int64_t* __restrict__ emb, const uint32_t* __restrict__ mb_sel,
-                        const int64_t* __restrict__ mbp, const int64_t* __restrict__ chp,
-                        uint8_t* __restrict__ image, uint8_t* __restrict__ resflag,
+                        const int64_t* __restrict__ mbp, int ratio, int64_t Pc,
+                        const int64_t* __restrict__ chp, uint8_t* __restrict__ image, uint8_t* __restrict__ resflag,
                         unsigned long long* __restrict__ kept_count) {
   int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kWarp;
   int lane = threadIdx.x % kWarp;
@@ -320,8 +329,9 @@ __global__ void k_place(const int64_t* __restrict__ Brp, const int32_t* __restri
       resflag[k] = kept ? 0 : 1;
       if (!kept) continue;
       atomicAdd(kept_count, 1ull);
+      // kernel panel (at Vp = 64 its other 64-row half keeps no-value nibbles in this k-group)
       int64_t panel = l / kPanelRows;
-      int64_t local = m - mbp[panel];
+      int64_t local = m - kpanel_mb(mbp, panel, ratio, Pc);
       int64_t chunk = chp[panel] + local / kChunkMB;
       int g = (int)(local % kChunkMB);
       int r = (int)(l % kPanelRows);
@@ -600,8 +610,9 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   if (N != 2) return fail(NM_ERR_UNSUPPORTED, "nm_pack: N must be 2 (hardware 2:4, L496)");
   if (!(M == 4 || M == 8 || M == 16)) return fail(NM_ERR_UNSUPPORTED, "nm_pack: M must be 4, 8 or 16");
   if (V < 1) return fail(NM_ERR_INVALID_ARG, "nm_pack: V < 1");
-  if (Vp == 0) Vp = kPanelRows;
-  if (Vp != kPanelRows) return fail(NM_ERR_UNSUPPORTED, "nm_pack: Vp must be 128");
+  if (Vp == 0) Vp = (V == 64) ? 64 : kPanelRows;
+  if (Vp != 64 && Vp != kPanelRows) return fail(NM_ERR_UNSUPPORTED, "nm_pack: Vp must be 64 or 128");
+  const int ratio = kPanelRows / Vp;  // canonical panels per kernel panel
   if (dtype != NM_F16 && dtype != NM_BF16) return fail(NM_ERR_UNSUPPORTED, "nm_pack: dtype must be f16 or bf16");
   const int64_t n = A->n;
   if (n <= 0 || A->nnz < 0) return fail(NM_ERR_INVALID_ARG, "nm_pack: empty graph");
@@ -610,7 +621,8 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     return fail(NM_ERR_INVALID_ARG, "nm_pack_rows: bad row range (row_begin must be a multiple of Vp unless the range is empty)");
   const int Mp = (V == 1) ? 4 : M;
   const int64_t rows = re - rb;
-  const int64_t P = (rows + Vp - 1) / Vp;
+  const int64_t P = (rows + kPanelRows - 1) / kPanelRows;  // kernel panels (MMA M = 128)
+  const int64_t Pc = (rows + Vp - 1) / Vp;                 // canonical panels
   const int64_t S = (n + Mp - 1) / Mp;
 
   if (!A->on_device) {
@@ -681,7 +693,7 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   NM_TRY(dalloc(d_mbkey, sizeof(int64_t) * bnnz, s));
   NM_TRY(dalloc(d_runs, sizeof(int64_t) * bnnz, s));
   NM_TRY(dalloc(d_nruns, sizeof(int64_t), s));
-  k_mbkey<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, rows, Mp, S, d_mk.as<int64_t>());
+  k_mbkey<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, rows, Vp, Mp, S, d_mk.as<int64_t>());
   {
     size_t bytes = 0;
     NM_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, bytes, d_mk.as<int64_t>(), d_mk2.as<int64_t>(), bnnz, 0, 64, s));
@@ -712,7 +724,7 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   NM_TRY(dalloc(d_selc, sizeof(uint32_t) * nc1, s));
   NM_CUDA(cudaMemsetAsync(d_cnt.p, 0, sizeof(int32_t) * Mp * nc1, s));
   if (bnnz) {
-    k_colcount<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, rows, Mp, S, d_mbkey.as<int64_t>(), n_cand,
+    k_colcount<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, rows, Vp, Mp, S, d_mbkey.as<int64_t>(), n_cand,
                                                        d_cnt.as<int32_t>(), d_emb.as<int64_t>());
     k_select<<<grid_for(n_cand, 256), 256, 0, s>>>(d_cnt.as<int32_t>(), Mp, n_cand, d_selc.as<uint32_t>());
   }
@@ -750,7 +762,7 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   NM_CUDA(cudaGetDevice(&Pk->device));
   Pk->n = n; Pk->row_begin = rb; Pk->row_end = re;
   Pk->V = V; Pk->N = N; Pk->M = M; Pk->Vp = Vp; Pk->Mp = Mp; Pk->dtype = dtype;
-  Pk->n_panels = P; Pk->n_mb = n_mb; Pk->tau = tau;
+  Pk->n_panels = P; Pk->n_cpanels = Pc; Pk->n_mb = n_mb; Pk->tau = tau;
   struct Guard {
     nm_packed* p;
     bool ok = false;
@@ -761,13 +773,13 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     Pk->device_bytes += bytes;
     return NM_OK;
   };
-  NM_TRY(palloc((void**)&Pk->panel_mb_ptr, sizeof(int64_t) * (P + 1)));
+  NM_TRY(palloc((void**)&Pk->panel_mb_ptr, sizeof(int64_t) * (Pc + 1)));
   NM_TRY(palloc((void**)&Pk->panel_chunk_ptr, sizeof(int64_t) * (P + 1)));
-  k_panel_ptr<<<grid_for(P + 1, 256), 256, 0, s>>>(mbkey, n_mb, P, S, Pk->panel_mb_ptr, nullptr);
+  k_panel_ptr<<<grid_for(Pc + 1, 256), 256, 0, s>>>(mbkey, n_mb, Pc, S, Pk->panel_mb_ptr, nullptr);
   DevBuf d_nch;
   NM_TRY(dalloc(d_nch, sizeof(int64_t) * (P + 1), s));
   NM_CUDA(cudaMemsetAsync(d_nch.p, 0, sizeof(int64_t) * (P + 1), s));
-  k_chunk_counts<<<grid_for(P, 256), 256, 0, s>>>(Pk->panel_mb_ptr, P, d_nch.as<int64_t>());
+  k_chunk_counts<<<grid_for(P, 256), 256, 0, s>>>(Pk->panel_mb_ptr, P, ratio, Pc, d_nch.as<int64_t>());
   NM_TRY(scan_excl(d_nch.as<int64_t>(), Pk->panel_chunk_ptr, P + 1, s));
   std::vector<int64_t> chp(P + 1);
   NM_CUDA(cudaMemcpyAsync(chp.data(), Pk->panel_chunk_ptr, sizeof(int64_t) * (P + 1), cudaMemcpyDeviceToHost, s));
@@ -789,7 +801,7 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   if (n_mb) {
     NM_CUDA(cudaMemcpyAsync(Pk->mb_sel, selv, sizeof(uint32_t) * n_mb, cudaMemcpyDeviceToDevice, s));
     k_write_sel<<<grid_for(n_mb, 256), 256, 0, s>>>(d_cnt.as<int32_t>(), d_cand_of.p ? d_cand_of.as<int64_t>() : nullptr,
-                                                    Mp, n_mb, mbkey, S, n, Pk->panel_mb_ptr, Pk->panel_chunk_ptr,
+                                                    Mp, n_mb, mbkey, S, n, Pk->panel_mb_ptr, ratio, Pc, Pk->panel_chunk_ptr,
                                                     Pk->mb_seg, Pk->mb_sel, full);
   }
   NM_CUDA(cudaGetLastError());
@@ -803,7 +815,7 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   NM_CUDA(cudaMemsetAsync(d_rc.p, 0, sizeof(int64_t) * (rows + 1), s));
   if (bnnz) {
     k_place<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, Bci, Bval, rows, Mp, d_emb.as<int64_t>(), Pk->mb_sel,
-                                                    Pk->panel_mb_ptr, Pk->panel_chunk_ptr, full,
+                                                    Pk->panel_mb_ptr, ratio, Pc, Pk->panel_chunk_ptr, full,
                                                     d_flag.as<uint8_t>(), d_kept.as<unsigned long long>());
     k_res_count<<<grid_for(rows * 32, 256), 256, 0, s>>>(Brp, d_flag.as<uint8_t>(), rows, d_rc.as<int64_t>());
   }
@@ -911,17 +923,12 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
     NM_CUDA(cudaStreamSynchronize(s));
   }
 
-  // unit schedule: natural panel order (consecutive panels run concurrently on the persistent
-  // grid, so their X neighbourhoods are shared in L2); NM_UNIT_ORDER=heavy sorts by chunk
-  // count instead.  One 16-byte descriptor per panel: {panel, #chunks, first chunk}.
+  // unit schedule of the compressed-record kernel: natural panel order (consecutive panels run
+  // concurrently on the persistent grid, so their X neighbourhoods are shared in L2).
+  // Two 16-byte descriptors per panel: {panel, #chunks, first chunk}, {record bytes offset, size}.
   {
     std::vector<int32_t> order(P);
     std::iota(order.begin(), order.end(), 0);
-    const char* ord = getenv("NM_UNIT_ORDER");
-    if (ord && std::string(ord) == "heavy")
-      std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
-        return (chp[a + 1] - chp[a]) > (chp[b + 1] - chp[b]);
-      });
     std::vector<int4> info(2 * P);
     for (int64_t j = 0; j < P; ++j) {
       const int32_t r = order[j];

@@ -55,6 +55,11 @@ def test_counts(kind, seed, V, M):
         assert np.array_equal(ps0, ps1)
 
 
+def _vp(V):
+    """nm_pack's automatic panel height (nm.h): 64 for V = 64 patterns, else 128."""
+    return 64 if V == 64 else 128
+
+
 def _values(ip, ic, dtype, seed):
     v = graphs.symmetric_values(ip, ic, seed)
     bits, v64 = graphs.round16(v, dtype)
@@ -69,7 +74,7 @@ def test_pack_canonical_bit_exact(kind, seed, V, M, dtype):
     perm, _ = api.reorder(ip, ic, V, 2, M)
     v32, bits, _ = _values(ip, ic, dtype, seed)
     Mp = 4 if V == 1 else M
-    ref = oracle.pack(ip, ic, bits, 0, perm, 128, Mp)
+    ref = oracle.pack(ip, ic, bits, 0, perm, _vp(V), Mp)
     P = api.pack(ip, ic, perm, V, 2, M, dtype=dtype, val=v32)  # device rounds f32 -> 16 bit
     got = P.export_canonical()
     for k in ("panel_ptr", "mb_seg", "sel", "nib", "vals", "res_rowptr", "res_col", "res_val"):
@@ -220,7 +225,7 @@ def test_spmm_original_order_fused(kind, seed, V, M, dtype):
     tdt = torch.float16 if dtype == "f16" else torch.bfloat16
     X = torch.from_numpy(xbits.view(np.int16)).to(dev).view(tdt)
     P = api.pack(ip, ic, perm, V, 2, M, dtype=dtype, val=v32, order="original")
-    ref = oracle.pack(ip, ic, bits, 0, perm, 128, 4 if V == 1 else M)
+    ref = oracle.pack(ip, ic, bits, 0, perm, _vp(V), 4 if V == 1 else M)
     got = P.export_canonical()
     for k in ("panel_ptr", "mb_seg", "nib", "vals", "res_rowptr", "res_col", "res_val"):
         assert np.array_equal(ref[k], got[k]), k
@@ -252,7 +257,7 @@ def test_pack_hybrid_canonical_bit_exact(kind, seed, V, M, tau, order):
     perm, _ = api.reorder(ip, ic, V, 2, M)
     v32, bits, _ = _values(ip, ic, "f16", seed)
     Mp = 4 if V == 1 else M
-    ref = oracle.pack(ip, ic, bits, 0, perm, 128, Mp, tau=tau)
+    ref = oracle.pack(ip, ic, bits, 0, perm, _vp(V), Mp, tau=tau)
     P = api.pack(ip, ic, perm, V, 2, M, dtype="f16", val=v32, tau=tau, order=order)
     got = P.export_canonical()
     for k in ("panel_ptr", "mb_seg", "sel", "nib", "vals", "res_rowptr", "res_col", "res_val"):
@@ -395,3 +400,92 @@ def test_sptc_formats_agree_bitwise(kind, seed, V, M, F):
     Y_ref, E, _ = oracle.spmm(ip, ic, v64, x64)
     err = np.abs(outs[0].astype(np.float64) - Y_ref)
     assert (err <= TOL * E).all(), err.max()
+
+
+# ------------------------------------------------------------------------------------------
+# panel height V_p (nm.h: Vp in {64, 128}; at 64 two canonical panels share a 128-row kernel
+# panel's chunks, each k-group holding one half's values)
+# ------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("kind,seed,V,M,Vp", [("band", 5, 64, 8, 64), ("band", 5, 64, 8, 128), ("pl", 3, 1, 4, 64),
+                                              ("pl", 6, 128, 16, 64), ("er", 7, 8, 8, 64), ("tiny", 1, 1, 4, 64)])
+@pytest.mark.parametrize("order", ["permuted", "original"])
+def test_panel_height_vp(kind, seed, V, M, Vp, order):
+    dev = _cuda()
+    ip, ic = _graph(kind, seed)
+    n = len(ip) - 1
+    F = 72
+    perm, _ = api.reorder(ip, ic, V, 2, M)
+    v32, bits, v64 = _values(ip, ic, "bf16", seed)
+    Mp = 4 if V == 1 else M
+    ref = oracle.pack(ip, ic, bits, 0, perm, Vp, Mp)
+    P = api.pack(ip, ic, perm, V, 2, M, dtype="bf16", val=v32, order=order, Vp=Vp)
+    assert P.stats()["Vp"] == Vp
+    got = P.export_canonical()
+    for k in ("panel_ptr", "mb_seg", "sel", "nib", "vals", "res_rowptr", "res_col", "res_val"):
+        assert np.array_equal(ref[k], got[k]), k
+    xbits, x64 = graphs.round16(graphs.features(n, F, seed + 2), "bf16")
+    Y_ref, E, _ = oracle.spmm(ip, ic, v64, x64)
+    X = torch.from_numpy(xbits.view(np.int16)).to(dev).view(torch.bfloat16)
+    if order == "permuted":
+        perm_d = torch.from_numpy(perm.astype(np.int32)).to(dev)
+        PX = torch.empty_like(X)
+        api.permute_rows(X, PX, perm_d, "bf16")
+        Yp = torch.full((n, F), float("nan"), device=dev)
+        api.spmm(P, PX, Yp, F=F)
+        Y = torch.empty_like(Yp)
+        api.unpermute_rows(Yp, Y, perm_d, "f32")
+    else:
+        Y = torch.full((n, F), float("nan"), device=dev)
+        api.spmm(P, X, Y, F=F)
+        # row shards starting at an odd multiple of 64 (legal at Vp = 64 only).  The shard's
+        # 128-row kernel panels pair different 64-row panels than the whole pack's, so the
+        # chunking (and the fp32 summation grouping inside each MMA) differs: checked against
+        # the oracle bound, not bitwise against Y.
+        if Vp == 64 and n > 256:
+            cut = ((n // 2) // 128) * 128 + 64
+            Y2 = torch.full((n, F), float("nan"), device=dev)
+            for a, b in ((0, cut), (cut, n)):
+                Ps = api.pack(ip, ic, perm, V, 2, M, dtype="bf16", val=v32, order="original", Vp=64,
+                              row_begin=a, row_end=b)
+                api.spmm(Ps, X, Y2, F=F)
+            torch.cuda.synchronize()
+            err2 = np.abs(Y2.cpu().numpy().astype(np.float64) - Y_ref)
+            assert (err2 <= TOL * E).all(), err2.max()
+    torch.cuda.synchronize()
+    err = np.abs(Y.cpu().numpy().astype(np.float64) - Y_ref)
+    assert (err <= TOL * E).all(), err.max()
+
+
+def test_vp64_conforming_v64_has_empty_residual():
+    """A 64:2:8-conforming matrix (every 64-row x 8-column meta-block uses <= 4 columns, every
+    row <= 2 per 8-segment, L194 / L226-230) packs losslessly into the tensor-core form at
+    Vp = 64, where 128-row panels would merge two halves' column sets and spill."""
+    _cuda()
+    rng = np.random.default_rng(5)
+    n, M = 1024, 8
+    rows = [[] for _ in range(n)]
+    for p in range(n // 64):
+        for s in range(n // M):
+            if rng.random() < 0.25:
+                cols = s * M + np.sort(rng.choice(M, 4, replace=False))
+                for i in range(p * 64, p * 64 + 64):
+                    if rng.random() < 0.5:
+                        rows[i].extend(rng.choice(cols, 2, replace=False).tolist())
+    ip = np.zeros(n + 1, np.int64)
+    ic = []
+    for i in range(n):
+        r = sorted(set(rows[i]))
+        ic.extend(r)
+        ip[i + 1] = ip[i] + len(r)
+    ic = np.array(ic, np.int32)
+    ident = np.arange(n, dtype=np.int32)
+    P64 = api.pack(ip, ic, ident, 64, 2, M)
+    P128 = api.pack(ip, ic, ident, 64, 2, M, Vp=128)
+    assert P64.stats()["Vp"] == 64 and P128.stats()["Vp"] == 128
+    assert P64.info()["residual_nnz"] == 0
+    assert P128.info()["residual_nnz"] > 0
+    ref = oracle.pack(ip, ic, None, 0x3C00, ident, 64, M)
+    assert ref["res_nnz"] == 0
+    got = P64.export_canonical()
+    for k in ("panel_ptr", "mb_seg", "sel", "nib", "vals"):
+        assert np.array_equal(ref[k], got[k]), k
