@@ -104,13 +104,16 @@ NM_API nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reord
 /* nm_reorder_gpu -- nm_reorder with Stage-1 (Alg. 2 lines 4-13: Hamming position codes of
  * every (row, segment) of B, L339-346 / Listing 1, and the stable lexicographic row
  * sort, L366-384) and the omega / MBscore counts (L203, L382) run on the current CUDA device
- * (the paper's SOGRE is a GPU library, L484).  Stage-2 (Alg. 3) stays on
- * the host: its greedy is sequential in the recorded pairs.  The permutation is bit-identical
- * to nm_reorder's and to the CPU oracle's.
+ * (the paper's SOGRE is a GPU library, L484).  Stage-2 (Alg. 3): the
+ * M x M gain tables of each batch of (primary, target) pairs are computed on the device
+ * (L448-455); the picks (freshtop, the est / I bookkeeping) stay on the host because the
+ * greedy is sequential in the recorded pairs.  The permutation is bit-identical to
+ * nm_reorder's and to the CPU oracle's.
  *   A, V, N, M, opts, perm_out, st : as nm_reorder (A host or device CSR; perm_out host).
  *   stream : cudaStream_t the device work is ordered on (NULL = legacy default stream).
- * Synchronous on return.  Device memory: ~ 60 bytes per stored entry + 60 per vertex,
- * from the default stream-ordered pool, trimmed on return.  Errors: as nm_reorder, plus CUDA / OOM. */
+ * Synchronous on return.  Device memory: ~ 60 bytes per stored entry + 60 per vertex, from a
+ * private stream-ordered pool created and destroyed by the call (the device's default pool is
+ * not touched).  Errors: as nm_reorder, plus CUDA / OOM. */
 NM_API nm_status nm_reorder_gpu(const nm_csr* A, int V, int N, int M, const nm_reorder_opts* opts,
                                 int32_t* perm_out, nm_reorder_stats* st, void* stream);
 
@@ -121,6 +124,18 @@ NM_API nm_status nm_reorder_gpu(const nm_csr* A, int V, int N, int M, const nm_r
  * *V_out / *M_out, its order in perm_out (host int32[n]) and its statistics.  Synchronous. */
 NM_API nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, const nm_reorder_opts* opts,
                                    int32_t* perm_out, int* V_out, int* M_out, nm_reorder_stats* st);
+
+/* nm_score_patterns -- best-V:N:M selection scored by the packed form:
+ * nm_select_pattern keeps the last pattern the reordered graph CONFORMS to (L496, L655); this
+ * scores what the SpMM would move.  For each candidate (V[i], M[i]), N = 2: nm_reorder_gpu with
+ * opts, nm_pack_hybrid at nm_hybrid_tau(F) (Vp auto), score = n_chunks * (0.28 + 0.0075 F) +
+ * residual_nnz * 0.00016 F (ns: the B200 time model nm_hybrid_tau is derived from, DESIGN.md
+ * §6).  scores (double[ncand]), n_chunks / residual_nnz (int64[ncand]): host, nullable.
+ * *best = index of the lowest score (ties: the earlier candidate), perm_out (host int32[n]) its
+ * permutation.  Synchronous.  Errors: as nm_reorder_gpu and nm_pack_hybrid. */
+NM_API nm_status nm_score_patterns(const nm_csr* A, int ncand, const int* V, const int* M, int F, nm_dtype dtype,
+                                   const nm_reorder_opts* opts, void* stream, double* scores,
+                                   int64_t* n_chunks, int64_t* residual_nnz, int* best, int32_t* perm_out);
 
 /* nm_count_violations -- omega (L203), MBscore (L382) and optionally PScore per segment
  * (L396) of B = P A P^T, computed on the GPU.  perm: host int32[n] or NULL (identity).

@@ -65,6 +65,11 @@ SIGNATURES = {
                                          ctypes.POINTER(nm_reorder_opts), P32,
                                          ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.c_int),
                                          ctypes.POINTER(nm_reorder_stats)]),
+    "nm_score_patterns": (ctypes.c_int, [ctypes.POINTER(nm_csr), ctypes.c_int, ctypes.POINTER(ctypes.c_int),
+                                         ctypes.POINTER(ctypes.c_int), ctypes.c_int, ctypes.c_int,
+                                         ctypes.POINTER(nm_reorder_opts), ctypes.c_void_p,
+                                         ctypes.POINTER(ctypes.c_double), P64, P64, ctypes.POINTER(ctypes.c_int),
+                                         P32]),
     "nm_count_violations": (ctypes.c_int, [ctypes.POINTER(nm_csr), P32, ctypes.c_int, ctypes.c_int,
                                            ctypes.c_int, P64, P64, P32]),
     "nm_pack": (ctypes.c_int, [ctypes.POINTER(nm_csr), P32, ctypes.c_int, ctypes.c_int, ctypes.c_int,

@@ -82,6 +82,30 @@ def select_pattern(indptr, indices, max_M=32, max_V=32, max_outer=10, max_stage1
     return V.value, M.value, perm, {f: getattr(st, f) for f, _ in L.nm_reorder_stats._fields_}
 
 
+def score_patterns(indptr, indices, candidates, F, dtype="bf16", val=None, val_dtype=None, stream=None,
+                   max_outer=10, max_stage1=10, max_stage2=10, gain_rule=0, keep_best=1):
+    """nm_score_patterns: candidates = [(V, M), ...] (N = 2).  Returns (best index, perm of the
+    best, [{"V", "M", "score_ns", "n_chunks", "residual_nnz"}, ...])."""
+    if val is not None and val_dtype is None:
+        val_dtype = "f32" if val.dtype == np.float32 else ("f16" if val.dtype == np.float16 else "bf16")
+    c, keep = _csr_struct(indptr, indices, val, val_dtype or "f16")
+    k = len(candidates)
+    Vs = (ctypes.c_int * k)(*[int(v) for v, _ in candidates])
+    Ms = (ctypes.c_int * k)(*[int(m) for _, m in candidates])
+    sc = (ctypes.c_double * k)()
+    ch = np.zeros(k, np.int64)
+    rs = np.zeros(k, np.int64)
+    best = ctypes.c_int()
+    perm = np.zeros(c.n, np.int32)
+    o = L.nm_reorder_opts(max_outer, max_stage1, max_stage2, gain_rule, keep_best)
+    L.check(L.load().nm_score_patterns(ctypes.byref(c), k, Vs, Ms, int(F), _DT[dtype], ctypes.byref(o),
+                                       _stream_ptr(stream), sc, ch.ctypes.data_as(L.P64), rs.ctypes.data_as(L.P64),
+                                       ctypes.byref(best), perm.ctypes.data_as(L.P32)), "nm_score_patterns")
+    rows = [{"V": int(v), "M": int(m), "score_ns": float(sc[i]), "n_chunks": int(ch[i]), "residual_nnz": int(rs[i])}
+            for i, (v, m) in enumerate(candidates)]
+    return best.value, perm, rows
+
+
 def count_violations(indptr, indices, perm, V: int, N: int, M: int):
     """nm_count_violations (GPU): returns (omega, mbscore, pscore int32[ceil(n/M)])."""
     c, keep = _csr_struct(indptr, indices)

@@ -8,9 +8,6 @@
 
 #include "nm_internal.h"
 
-#ifndef NM_RES_KERNEL
-#define NM_RES_KERNEL 0  // residual kernel: 0 = subgroup per item (default, measured faster), 1 = warp per item
-#endif
 #ifndef NM_RES_UNROLL
 #define NM_RES_UNROLL 2  // X rows in flight per lane in k_residual (measured: 2 >= 4 >> 8)
 #endif
@@ -247,219 +244,6 @@ __global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ seg
   }
 }
 
-// Warp-per-item residual SpMM (the default, NM_RES_KERNEL = 1).  The whole warp works on one
-// work item at a time, so every lane runs the same trip counts (no divergent subgroups, every
-// shuffle over the full warp).  The warp is EPS = 32 / LPR lane groups; group g takes the
-// entries e = g (mod EPS) of each batch of BATCH entries, a lane owns 8 consecutive features
-// of the launch's slab and moves them with one 16-byte cp.async per entry into its own slots
-// of the warp's shared-memory ring (a lane reads back only what it copied: cp.async.wait_group
-// is the only synchronisation).  Batches are pipelined ACROSS the warp's items: batch j + 1
-// (possibly the next item's first) is in flight while batch j is accumulated, and the Y row
-// of a single-item row is read when its first batch is issued.  At an item's end the groups'
-// partial sums are added with butterfly shuffles (fixed order: deterministic) and group 0
-// writes Y (single-item rows) or the item's partial (split rows; the last arrival reduces the
-// partials in item order, as in k_residual_sub).
-template <int LPR>
-struct ResW {
-  static constexpr int EPS = 32 / LPR;                      // entries per warp step
-  static constexpr int BATCH = 8 * EPS < 32 ? 8 * EPS : 32;  // entries per batch (<= 32: one per lane)
-  static constexpr int SLOTS = BATCH / EPS;                 // 16-byte slots per lane and batch
-  static constexpr int kWarpBytes = 2 * SLOTS * 32 * 16;    // double-buffered ring per warp
-  static constexpr int kWarps = 8;                          // warps per CTA
-  static constexpr int kSmem = kWarps * kWarpBytes;
-};
-
-template <int BF, int LPR>
-__global__ void __launch_bounds__(256) k_residual_w(const ResSeg* __restrict__ segs, int64_t n_segs,
-                                                    const int32_t* __restrict__ rc, const uint16_t* __restrict__ rv,
-                                                    const uint16_t* __restrict__ X, int64_t ldx,
-                                                    float* __restrict__ Y, int64_t ldy, int F, int f_base,
-                                                    float* __restrict__ ws, int32_t* __restrict__ cnt) {
-  using C = ResW<LPR>;
-  constexpr int EPS = C::EPS, BATCH = C::BATCH, SLOTS = C::SLOTS;
-  extern __shared__ __align__(16) uint8_t res_smem[];
-  const int lane = threadIdx.x & 31;
-  const int grp = lane / LPR, li = lane % LPR;
-  const int f = f_base + li * 8;
-  const bool fin = f < F;  // lanes past the F tail copy nothing (their sums are never stored)
-  // byte address of (row c, feature f) = c * ldxb + xbase: one 32 x 32 -> 64-bit IMAD.WIDE
-  const uint64_t xbase = (uint64_t)(uintptr_t)(X + (fin ? f : 0));
-  const uint32_t ldxb = (uint32_t)ldx * 2u;  // ldx < 2^31 (nm_spmm), rows < 2^31
-  const bool vec_y = ((ldy & 3) == 0) && ((((uintptr_t)Y) & 15) == 0) && f + 8 <= F;
-  const uint32_t ring = (uint32_t)__cvta_generic_to_shared(res_smem) + (threadIdx.x >> 5) * C::kWarpBytes + lane * 16;
-  const int64_t nwarps = (int64_t)gridDim.x * (blockDim.x >> 5);
-  int64_t wi = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  if (wi >= n_segs) return;
-  // slots of a partial batch past the item's end are not copied: they keep an earlier batch's
-  // (finite) X values or these zeros and are multiplied by a zero value
-#pragma unroll
-  for (int i = 0; i < 2 * SLOTS; ++i)
-    asm volatile("st.shared.v4.b32 [%0], {%1, %1, %1, %1};" ::"r"(ring + i * 32 * 16), "r"(0u) : "memory");
-
-  // issue side: item wi (descriptor gi), batch ki
-  ResSeg gi = segs[wi];
-  int ki = 0;
-  // compute side: the batch issued before the current issue position
-  ResSeg gc;
-  int kc = 0;
-  uint32_t vc = 0u, vn = 0u;               // 16-bit values of the compute / in-flight batch (lane t: entry t)
-  float4 yc0 = make_float4(0.f, 0.f, 0.f, 0.f), yc1 = yc0, yn0 = yc0, yn1 = yc0;
-  int bp = 0;                              // ring half of the compute batch
-
-  // issues batch ki of item gi into ring half h; returns the lane's value bits
-  auto issue = [&](const ResSeg& g, int k, int h, uint32_t& vout) {
-    const int e0 = k * BATCH;
-    const int rem = g.len - e0;
-    int32_t col = 0;
-    uint32_t v = 0u;
-    if (lane < BATCH && lane < rem) {
-      col = __ldcs(rc + g.kb + e0 + lane);  // streamed once
-      v = __ldcs(rv + g.kb + e0 + lane);
-    }
-    vout = v;
-    const uint32_t base = ring + (uint32_t)(h * SLOTS * 32 * 16);
-    if (rem >= BATCH) {  // full batch (warp-uniform branch): no per-entry predicate
-#pragma unroll
-      for (int i = 0; i < SLOTS; ++i) {
-        const uint32_t c = (uint32_t)__shfl_sync(0xffffffffu, col, i * EPS + grp);
-        const uint64_t src = (uint64_t)c * ldxb + xbase;
-        asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p cp.async.cg.shared.global [%0], [%1], 16;\n\t}" ::"r"(
-                         base + i * 32 * 16),
-                     "l"(src), "r"((uint32_t)fin)
-                     : "memory");
-      }
-    } else {
-#pragma unroll
-      for (int i = 0; i < SLOTS; ++i) {
-        const int e = i * EPS + grp;
-        const uint32_t c = (uint32_t)__shfl_sync(0xffffffffu, col, e);
-        const uint64_t src = (uint64_t)c * ldxb + xbase;
-        asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p cp.async.cg.shared.global [%0], [%1], 16;\n\t}" ::"r"(
-                         base + i * 32 * 16),
-                     "l"(src), "r"((uint32_t)(fin && e < rem))
-                     : "memory");
-      }
-    }
-    asm volatile("cp.async.commit_group;" ::: "memory");
-  };
-  auto load_y = [&](const ResSeg& g, float4& y0, float4& y1) {
-    if (g.slot < 0 && vec_y && grp == 0) {
-      const float* y = Y + (int64_t)g.yrow * ldy + f;
-      y0 = __ldcs((const float4*)y);
-      y1 = __ldcs((const float4*)(y + 4));
-    }
-  };
-
-  issue(gi, 0, 0, vn);
-  load_y(gi, yn0, yn1);
-  float acc[8];
-#pragma unroll
-  for (int q = 0; q < 8; ++q) acc[q] = 0.f;
-  for (;;) {
-    // the in-flight batch becomes the compute batch; advance the issue position
-    gc = gi;
-    kc = ki;
-    vc = vn;
-    if (kc == 0) { yc0 = yn0; yc1 = yn1; }
-    bool more = true;
-    if (++ki * BATCH >= gi.len) {
-      ki = 0;
-      wi += nwarps;
-      more = wi < n_segs;
-      if (more) gi = segs[wi];
-    }
-    if (more) {
-      issue(gi, ki, bp ^ 1, vn);
-      if (ki == 0) load_y(gi, yn0, yn1);
-      asm volatile("cp.async.wait_group 1;" ::: "memory");
-    } else {
-      asm volatile("cp.async.wait_group 0;" ::: "memory");
-    }
-    // accumulate the compute batch
-    {
-      const uint32_t base = ring + (uint32_t)(bp * SLOTS * 32 * 16);
-#pragma unroll
-      for (int i = 0; i < SLOTS; ++i) {
-        const unsigned short a = (unsigned short)__shfl_sync(0xffffffffu, vc, i * EPS + grp);
-        uint32_t wv[4];
-        asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
-                     : "=r"(wv[0]), "=r"(wv[1]), "=r"(wv[2]), "=r"(wv[3])
-                     : "r"(base + i * 32 * 16));
-#pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          acc[2 * q] = fma16<BF>(a, (unsigned short)(wv[q] & 0xFFFFu), acc[2 * q]);
-          acc[2 * q + 1] = fma16<BF>(a, (unsigned short)(wv[q] >> 16), acc[2 * q + 1]);
-        }
-      }
-    }
-    bp ^= 1;
-    if ((kc + 1) * BATCH >= gc.len) {
-      // item done: add the groups' partial sums (butterfly, fixed order)
-#pragma unroll
-      for (int o = LPR; o < 32; o <<= 1)
-#pragma unroll
-        for (int q = 0; q < 8; ++q) acc[q] += __shfl_xor_sync(0xffffffffu, acc[q], o);
-      float* y = Y + (int64_t)gc.yrow * ldy + f;
-      if (gc.slot < 0) {
-        if (grp == 0 && f < F) {
-          if (vec_y) {
-            yc0.x += acc[0]; yc0.y += acc[1]; yc0.z += acc[2]; yc0.w += acc[3];
-            yc1.x += acc[4]; yc1.y += acc[5]; yc1.z += acc[6]; yc1.w += acc[7];
-            __stcs((float4*)y, yc0);
-            __stcs((float4*)(y + 4), yc1);
-          } else {
-#pragma unroll
-            for (int q = 0; q < 8; ++q)
-              if (f + q < F) y[q] += acc[q];
-          }
-        }
-      } else {
-        // split row: publish this item's partial; the last arrival reduces in item order
-        float* part = ws + ((int64_t)(gc.slot + gc.idx) * (LPR * 8)) + li * 8;
-        if (grp == 0) {
-          *(float4*)part = make_float4(acc[0], acc[1], acc[2], acc[3]);
-          *(float4*)(part + 4) = make_float4(acc[4], acc[5], acc[6], acc[7]);
-        }
-        __threadfence();
-        __syncwarp();
-        int last = 0;
-        if (lane == 0) last = atomicAdd(cnt + gc.split_id, 1) == gc.nseg - 1;
-        last = __shfl_sync(0xffffffffu, last, 0);
-        if (last) {
-          __threadfence();
-          float s[8];
-#pragma unroll
-          for (int q = 0; q < 8; ++q) s[q] = 0.f;
-          if (grp == 0) {
-            for (int i = 0; i < gc.nseg; ++i) {
-              const float* pi = ws + ((int64_t)(gc.slot + i) * (LPR * 8)) + li * 8;
-              const float4 pa = __ldcg((const float4*)pi), pb = __ldcg((const float4*)(pi + 4));
-              s[0] += pa.x; s[1] += pa.y; s[2] += pa.z; s[3] += pa.w;
-              s[4] += pb.x; s[5] += pb.y; s[6] += pb.z; s[7] += pb.w;
-            }
-            if (f < F) {
-              if (vec_y) {
-                float4 a0 = *(float4*)y, a1 = *(float4*)(y + 4);
-                a0.x += s[0]; a0.y += s[1]; a0.z += s[2]; a0.w += s[3];
-                a1.x += s[4]; a1.y += s[5]; a1.z += s[6]; a1.w += s[7];
-                *(float4*)y = a0;
-                *(float4*)(y + 4) = a1;
-              } else {
-#pragma unroll
-                for (int q = 0; q < 8; ++q)
-                  if (f + q < F) y[q] += s[q];
-              }
-            }
-          }
-        }
-      }
-#pragma unroll
-      for (int q = 0; q < 8; ++q) acc[q] = 0.f;
-      if (!more) break;
-    }
-  }
-}
-
 // dst[p] = src[idx[p]] (gather) or dst[idx[p]] = src[p] (scatter); row bytes copied with
 // 16-byte vectors when aligned.  One warp per row.
 template <bool SCATTER>
@@ -566,8 +350,6 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
   const int sub_per_warp = 32 / lpr;
   int64_t g = (P->n_res_segs + 8 * sub_per_warp - 1) / (8 * sub_per_warp);
   if (g > 148 * 16) g = 148 * 16;
-  int sms = 148;
-  NM_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, P->device));
   // this call's split-row workspace: partial-sum slots + arrival counters (one set per slab
   // launch, so the counters need no reset between the launches of one call)
   const int nslab = (F + lpr * 8 - 1) / (lpr * 8);
@@ -589,23 +371,6 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
       return cuda_fail(e, "cudaMemsetAsync(residual counters)");
     }
   }
-#if NM_RES_KERNEL == 1
-#define NM_RES_LAUNCH(BF, LPR)                                                                              \
-  do {                                                                                                      \
-    static int resident = 0;                                                                                \
-    if (!resident) {                                                                                        \
-      if (ResW<LPR>::kSmem > 48 * 1024)                                                                     \
-        cudaFuncSetAttribute(k_residual_w<BF, LPR>, cudaFuncAttributeMaxDynamicSharedMemorySize,            \
-                             ResW<LPR>::kSmem);                                                             \
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&resident, k_residual_w<BF, LPR>, 256, ResW<LPR>::kSmem); \
-      if (resident < 1) resident = 1;                                                                       \
-    }                                                                                                       \
-    const int64_t gw = std::min<int64_t>((P->n_res_segs + 7) / 8, (int64_t)sms * resident);                \
-    k_residual_w<BF, LPR><<<(unsigned)gw, 256, ResW<LPR>::kSmem, s>>>(                                      \
-        P->res_segs, P->n_res_segs, rcol, P->res_val, (const uint16_t*)PX, ldx, Yp, ldy, F, f_base, ws,     \
-        cnt ? cnt + P->n_res_split * (f_base / (lpr * 8)) : nullptr);                                       \
-  } while (0)
-#else
 #define NM_RES_LAUNCH(BF, LPR)                                                                              \
   do {                                                                                                      \
     static bool attr_set = false;                                                                           \
@@ -618,7 +383,6 @@ nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, 
         P->res_segs, P->n_res_segs, rcol, P->res_val, (const uint16_t*)PX, ldx, Yp, ldy, F, f_base, ws,     \
         cnt ? cnt + P->n_res_split * (f_base / (lpr * 8)) : nullptr);                                       \
   } while (0)
-#endif
   for (int f_base = 0; f_base < F; f_base += lpr * 8) {
     switch (lpr * 2 + bf) {
       case 8: NM_RES_LAUNCH(0, 4); break;

@@ -12,6 +12,7 @@
 
 #include <algorithm>
 #include <cstdlib>
+#include <cstring>
 #include <string>
 #include <numeric>
 #include <vector>
@@ -970,8 +971,50 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   return NM_OK;
 }
 
+// Pattern scoring: reorder + hybrid pack per candidate, scored by the
+// library's own time model (the one nm_hybrid_tau is derived from).
+nm_status score_patterns_impl(const nm_csr* A, int ncand, const int* Vs, const int* Ms, int F, nm_dtype dtype,
+                              const nm_reorder_opts* opts, cudaStream_t s, double* scores, int64_t* chunks_out,
+                              int64_t* res_out, int* best, int32_t* perm_out) {
+  if (!A || ncand < 1 || !Vs || !Ms || !best || !perm_out)
+    return fail(NM_ERR_INVALID_ARG, "nm_score_patterns: NULL argument or no candidate");
+  if (F < 1) return fail(NM_ERR_INVALID_ARG, "nm_score_patterns: F < 1");
+  const int64_t n = A->n;
+  std::vector<int32_t> perm(n > 0 ? n : 1);
+  double best_score = 0.0;
+  int best_i = -1;
+  const int tau = nm_hybrid_tau(F);
+  for (int i = 0; i < ncand; ++i) {
+    NM_TRY(nm_reorder_gpu(A, Vs[i], 2, Ms[i], opts, perm.data(), nullptr, s));
+    nm_packed* P = nullptr;
+    NM_TRY(pack_impl(A, perm.data(), Vs[i], 2, Ms[i], 0, dtype, 0, n, 0, tau, s, &P));
+    const double t_chunk = 0.28 + 0.0075 * F, t_value = 0.00016 * F;  // ns (nm_hybrid_tau's model)
+    const double sc = (double)P->n_chunks * t_chunk + (double)P->res_nnz * t_value;
+    if (scores) scores[i] = sc;
+    if (chunks_out) chunks_out[i] = P->n_chunks;
+    if (res_out) res_out[i] = P->res_nnz;
+    nm_packed_free(P);
+    if (best_i < 0 || sc < best_score) {  // ties keep the earlier candidate
+      best_score = sc;
+      best_i = i;
+      memcpy(perm_out, perm.data(), sizeof(int32_t) * n);
+    }
+  }
+  *best = best_i;
+  return NM_OK;
+}
+
 }  // namespace
 }  // namespace nm
+
+extern "C" nm_status nm_score_patterns(const nm_csr* A, int ncand, const int* V, const int* M, int F, nm_dtype dtype,
+                                       const nm_reorder_opts* opts, void* stream, double* scores,
+                                       int64_t* n_chunks, int64_t* residual_nnz, int* best, int32_t* perm_out) {
+  return nm::guarded("nm_score_patterns", [&] {
+    return nm::score_patterns_impl(A, ncand, V, M, F, dtype, opts, (cudaStream_t)stream, scores, n_chunks,
+                                   residual_nnz, best, perm_out);
+  });
+}
 
 extern "C" nm_status nm_pack(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
                              nm_dtype dtype, void* stream, nm_packed** out) {

@@ -55,7 +55,7 @@ def main():
         res["full_sptc_ms"] = timed(lambda: api.spmm(P, X, Y, F=F, part="sptc"), flush)
         res["full_res_ms"] = timed(lambda: api.spmm(P, X, Y, F=F, part="residual"), flush)
         api.spmm(P, X, Y, F=F)
-        for s in (2, 4):
+        for s in ((2, 4) if os.environ.get("FSPLIT", "1") == "1" else ()):
             if F % (8 * s):
                 continue
             fs = F // s
