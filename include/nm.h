@@ -300,6 +300,20 @@ NM_API nm_status nm_gcn_layer(const nm_packed* Ahat, const void* H, const void* 
                        void* Hout, int F_in, int F_out, int flags, void* ws, size_t ws_bytes,
                        void* stream);
 
+/* nm_gcn_layer_bcast -- nm_gcn_layer whose output rows go straight into n_dst (1..16) buffers:
+ * dst is a HOST array of device pointers, each a row-major [* x F_out] buffer of the pack's
+ * dtype, 16-byte aligned; the layer's rows [0, row_end-row_begin) are stored at rows
+ * [dst_row0, dst_row0 + rows) of every dst[i] by the fused bias + activation + down-convert
+ * kernel.  This is the all-gather of the row-sharded multi-GPU GCN (PAPER.md
+ * L426) fused into the layer's last kernel: on one node dst[] holds every rank's
+ * peer-mapped (NVLink, symmetric-memory) copy of the next layer's operand, so the rows reach
+ * each GPU from this kernel's 16-byte stores instead of a separate collective.  The caller
+ * orders the ranks (a barrier after the layer, before anyone reads the buffers).  Stream-
+ * ordered.  Errors: as nm_gcn_layer, plus INVALID_ARG for a bad destination list. */
+NM_API nm_status nm_gcn_layer_bcast(const nm_packed* Ahat, const void* H, const void* W, const float* bias,
+                                    void* const* dst, int n_dst, int64_t dst_row0, int F_in, int F_out,
+                                    int flags, void* ws, size_t ws_bytes, void* stream);
+
 /* nm_gcn_layer_backward -- gradients of nm_gcn_layer (linear-first or aggregate-first give the
  * same Z = Ahat (H W) + b), SURVEY §8(f) item 4:
  *   dZ = dHout * act'(Z) (ReLU: Hout > 0), db = column sums of dZ, dT = Ahat^T dZ = Ahat dZ

@@ -101,6 +101,8 @@ SIGNATURES = {
     "nm_gcn_workspace_bytes": (ctypes.c_size_t, [ctypes.c_int64, ctypes.c_int, ctypes.c_int]),
     "nm_gcn_layer": (ctypes.c_int, [VP, VP, VP, VP, VP, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                     VP, ctypes.c_size_t, VP]),
+    "nm_gcn_layer_bcast": (ctypes.c_int, [VP, VP, VP, VP, ctypes.POINTER(VP), ctypes.c_int, ctypes.c_int64,
+                                          ctypes.c_int, ctypes.c_int, ctypes.c_int, VP, ctypes.c_size_t, VP]),
     "nm_gcn_backward_workspace_bytes": (ctypes.c_size_t, [ctypes.c_int64, ctypes.c_int, ctypes.c_int]),
     "nm_sgc_workspace_bytes": (ctypes.c_size_t, [ctypes.c_int64, ctypes.c_int]),
     "nm_sgc_propagate": (ctypes.c_int, [VP, VP, ctypes.c_int64, VP, ctypes.c_int64, VP, ctypes.c_int, ctypes.c_int,

@@ -268,6 +268,17 @@ def gcn_layer(P: Packed, H, W, bias, Hout, ws, relu=True, order="linear", stream
             "nm_gcn_layer")
 
 
+def gcn_layer_bcast(P: Packed, H, W, bias, dst_ptrs, dst_row0, F_out, ws, relu=True, order="linear",
+                    stream=None):
+    """nm_gcn_layer_bcast: this shard's output rows stored at rows [dst_row0, +rows) of every
+    buffer in dst_ptrs (device addresses, e.g. every rank's symmetric-memory buffer)."""
+    flags = (L.NM_RELU if relu else 0) | _ORDERS[order]
+    arr = (ctypes.c_void_p * len(dst_ptrs))(*[int(p) for p in dst_ptrs])
+    L.check(L.load().nm_gcn_layer_bcast(P.handle, _ptr(H), _ptr(W), _ptr(bias), arr, len(dst_ptrs), int(dst_row0),
+                                        H.shape[1], int(F_out), flags, _ptr(ws), ws.numel(), _stream_ptr(stream)),
+            "nm_gcn_layer_bcast")
+
+
 def gcn_backward_workspace_bytes(n, F_in, F_out):
     return int(L.load().nm_gcn_backward_workspace_bytes(n, F_in, F_out))
 

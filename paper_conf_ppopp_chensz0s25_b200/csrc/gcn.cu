@@ -38,6 +38,51 @@ __global__ void k_bias_act(const float* __restrict__ Y, int64_t rows, int F, con
   }
 }
 
+// bias + activation + down-convert of 8 consecutive features per thread, the 16-byte result
+// stored into every destination buffer (row dst_row0 + l): the fused all-gather of
+// nm_gcn_layer_bcast -- on a multi-GPU node the destinations are the ranks' peer-mapped
+// (NVLink) buffers, so the rows reach every GPU from this kernel's own stores
+constexpr int kMaxDst = 16;
+struct DstList {
+  uint16_t* p[kMaxDst];
+  int n;
+};
+
+template <int BF>
+__global__ void k_bias_act_bcast(const float* __restrict__ Y, int64_t rows, int F, const float* __restrict__ bias,
+                                 int relu, DstList dst, int64_t dst_row0) {
+  const int vpr = F / 8;  // 16-byte vectors per row (F % 8 == 0)
+  const int64_t total = rows * vpr;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / vpr;
+    const int c = (int)(i % vpr) * 8;
+    const float4 a = *(const float4*)(Y + r * F + c), b = *(const float4*)(Y + r * F + c + 4);
+    float v[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+    uint32_t w[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      float x0 = v[2 * q] + (bias ? bias[c + 2 * q] : 0.f), x1 = v[2 * q + 1] + (bias ? bias[c + 2 * q + 1] : 0.f);
+      if (relu) {
+        x0 = fmaxf(x0, 0.f);
+        x1 = fmaxf(x1, 0.f);
+      }
+      uint16_t h0, h1;
+      if (BF) {
+        __nv_bfloat16 t0 = __float2bfloat16_rn(x0), t1 = __float2bfloat16_rn(x1);
+        h0 = *(uint16_t*)&t0;
+        h1 = *(uint16_t*)&t1;
+      } else {
+        __half t0 = __float2half_rn(x0), t1 = __float2half_rn(x1);
+        h0 = *(uint16_t*)&t0;
+        h1 = *(uint16_t*)&t1;
+      }
+      w[q] = (uint32_t)h0 | ((uint32_t)h1 << 16);
+    }
+    const uint4 o = make_uint4(w[0], w[1], w[2], w[3]);
+    for (int d = 0; d < dst.n; ++d) *(uint4*)(dst.p[d] + (dst_row0 + r) * F + c) = o;
+  }
+}
+
 template <int BF>
 __global__ void k_to16(const float* __restrict__ Y, int64_t total, uint16_t* __restrict__ out) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
@@ -214,10 +259,10 @@ extern "C" size_t nm_gcn_workspace_bytes(int64_t n, int F_in, int F_out) {
          kLtWorkspace;
 }
 
-extern "C" nm_status nm_gcn_layer(const nm_packed* Ahat, const void* H, const void* W, const float* bias,
-                                  void* Hout, int F_in, int F_out, int flags, void* ws, size_t ws_bytes,
-                                  void* stream) {
-  if (!Ahat || !H || !W || !Hout || !ws) return fail(NM_ERR_INVALID_ARG, "nm_gcn_layer: NULL argument");
+static nm_status gcn_layer_impl(const nm_packed* Ahat, const void* H, const void* W, const float* bias,
+                                void* Hout, const DstList* bc, int64_t dst_row0, int F_in, int F_out, int flags,
+                                void* ws, size_t ws_bytes, void* stream) {
+  if (!Ahat || !H || !W || !(Hout || bc) || !ws) return fail(NM_ERR_INVALID_ARG, "nm_gcn_layer: NULL argument");
   if (F_in < 1 || F_out < 1 || F_out % 8 != 0 || F_in % 8 != 0)
     return fail(NM_ERR_UNSUPPORTED, "nm_gcn_layer: F_in and F_out must be positive multiples of 8");
   if (flags & ~(NM_RELU | NM_AGG_FIRST | NM_ORDER_AUTO)) return fail(NM_ERR_INVALID_ARG, "nm_gcn_layer: unknown flags");
@@ -252,10 +297,44 @@ extern "C" nm_status nm_gcn_layer(const nm_packed* Ahat, const void* H, const vo
     if (st != NM_OK) return st;
     pre = out32;
   }
-  if (bf) k_bias_act<1><<<grid_for(rows * F_out), 256, 0, s>>>(pre, rows, F_out, bias, flags & NM_RELU, (uint16_t*)Hout);
-  else k_bias_act<0><<<grid_for(rows * F_out), 256, 0, s>>>(pre, rows, F_out, bias, flags & NM_RELU, (uint16_t*)Hout);
+  if (bc) {
+    if (rows > 0) {
+      if (bf)
+        k_bias_act_bcast<1><<<grid_for(rows * (F_out / 8)), 256, 0, s>>>(pre, rows, F_out, bias, flags & NM_RELU, *bc,
+                                                                        dst_row0);
+      else
+        k_bias_act_bcast<0><<<grid_for(rows * (F_out / 8)), 256, 0, s>>>(pre, rows, F_out, bias, flags & NM_RELU, *bc,
+                                                                        dst_row0);
+    }
+  } else if (bf) {
+    k_bias_act<1><<<grid_for(rows * F_out), 256, 0, s>>>(pre, rows, F_out, bias, flags & NM_RELU, (uint16_t*)Hout);
+  } else {
+    k_bias_act<0><<<grid_for(rows * F_out), 256, 0, s>>>(pre, rows, F_out, bias, flags & NM_RELU, (uint16_t*)Hout);
+  }
   NM_CUDA(cudaGetLastError());
   return NM_OK;
+}
+
+extern "C" nm_status nm_gcn_layer(const nm_packed* Ahat, const void* H, const void* W, const float* bias,
+                                  void* Hout, int F_in, int F_out, int flags, void* ws, size_t ws_bytes,
+                                  void* stream) {
+  return gcn_layer_impl(Ahat, H, W, bias, Hout, nullptr, 0, F_in, F_out, flags, ws, ws_bytes, stream);
+}
+
+extern "C" nm_status nm_gcn_layer_bcast(const nm_packed* Ahat, const void* H, const void* W, const float* bias,
+                                        void* const* dst, int n_dst, int64_t dst_row0, int F_in, int F_out,
+                                        int flags, void* ws, size_t ws_bytes, void* stream) {
+  if (!dst || n_dst < 1 || n_dst > kMaxDst)
+    return fail(NM_ERR_INVALID_ARG, "nm_gcn_layer_bcast: need 1 <= n_dst <= 16 destination buffers");
+  if (dst_row0 < 0) return fail(NM_ERR_INVALID_ARG, "nm_gcn_layer_bcast: dst_row0 < 0");
+  DstList bc;
+  bc.n = n_dst;
+  for (int d = 0; d < n_dst; ++d) {
+    if (!dst[d] || ((uintptr_t)dst[d] & 15)) return fail(NM_ERR_INVALID_ARG, "nm_gcn_layer_bcast: NULL or unaligned destination");
+    bc.p[d] = (uint16_t*)dst[d];
+  }
+  for (int d = n_dst; d < kMaxDst; ++d) bc.p[d] = nullptr;
+  return gcn_layer_impl(Ahat, H, W, bias, nullptr, &bc, dst_row0, F_in, F_out, flags, ws, ws_bytes, stream);
 }
 
 // ---- backward ----------------------------------------------------------

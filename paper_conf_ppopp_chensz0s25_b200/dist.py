@@ -14,8 +14,12 @@
   is its send buffer).  Shards are padded to equal row counts so the collective needs no
   reshuffle; with equal shards the padding sits at the end and the gathered buffer is used
   as is, otherwise the padding rows are dropped after the gather.
-* ``local_layer`` is injectable so the host-side logic (sharding, padding, collective order)
-  is testable with the ``gloo`` backend on CPU (tests/test_dist.py).
+* ``gcn_forward_fused``: the same forward with the all-gather fused into each layer's last
+  kernel (``nm_gcn_layer_bcast``): every rank stores its rows straight into all ranks'
+  peer-mapped buffers (torch symmetric memory over NVLink), then one barrier per layer.
+* ``local_layer`` / ``local_layer_bcast`` and the buffer provider are injectable so the host-
+  side logic (sharding, padding, offsets, buffer alternation) is testable with the ``gloo``
+  backend on CPU (tests/test_dist.py).
 """
 from __future__ import annotations
 
@@ -117,5 +121,81 @@ def gcn_forward(H, layers, local_layer, group=None, bounds=None):
         if all(b - a == rows_pad for a, b in bounds[:-1]):
             cur = full[:n]  # equal shards: the padding is all at the end, no copy
         else:  # drop each rank's padding rows
+            cur = torch.cat([full[r * rows_pad: r * rows_pad + (b - a)] for r, (a, b) in enumerate(bounds)], dim=0)
+    return cur
+
+
+class SymmetricBuffers:
+    """Peer-mapped layer buffers for ``gcn_forward_fused`` on one NVLink node: every rank owns
+    a [rows_pad * world x F] buffer, allocated with torch's symmetric memory and exchanged
+    (rendezvous) so each rank holds the device addresses of all ranks' copies."""
+
+    def __init__(self, group=None):
+        self.group = group
+        self._h = {}
+
+    def alloc(self, key, shape, dtype, device):
+        import torch.distributed as dist
+        import torch.distributed._symmetric_memory as symm_mem
+        t = symm_mem.empty(shape, dtype=dtype, device=device)
+        h = symm_mem.rendezvous(t, self.group if self.group is not None else dist.group.WORLD)
+        self._h[key] = h
+        return t, list(h.buffer_ptrs)
+
+    def barrier(self, key):
+        self._h[key].barrier()
+
+
+class LocalBuffers:
+    """Single-process stand-in for SymmetricBuffers (world = 1): the only destination is the
+    local buffer, the barrier is a no-op."""
+
+    def alloc(self, key, shape, dtype, device):
+        import torch
+        t = torch.empty(shape, dtype=dtype, device=device)
+        return t, [t.data_ptr()]
+
+    def barrier(self, key):
+        pass
+
+
+def gcn_forward_fused(H, layers, local_layer_bcast, buffers, group=None, bounds=None):
+    """Multi-layer GCN forward with the all-gather FUSED into each layer's last kernel
+    (nm_gcn_layer_bcast): rank r stores its output rows [rb, re) straight into rows
+    [r * rows_pad, ...) of every rank's copy of the next layer's operand (peer-mapped buffers
+    from ``buffers``), then one barrier orders the ranks -- no separate collective and no
+    staging copy.  Two buffers alternate between layers: a rank writes layer l + 1's rows into
+    peers' buffer (l + 1) % 2 only after the barrier of layer l, i.e. after every rank has
+    finished reading it as layer l - 1's output.
+
+    local_layer_bcast(l, H_full, W, bias, relu, rb, re, dst_ptrs, dst_row0) runs the layer on
+        this rank's rows and stores them at dst_row0 of every buffer in dst_ptrs.
+    Returns the full [n x F_L] output on every rank (a view of the last buffer when the shards
+    are equal, else a compacted copy)."""
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    rank = dist.get_rank(group) if dist.is_initialized() else 0
+    n = H.shape[0]
+    if bounds is None:
+        bounds = [shard_rows(n, world, r) for r in range(world)]
+    assert len(bounds) == world and bounds[0][0] == 0 and bounds[-1][1] == n
+    rb, re = bounds[rank]
+    rows_pad = max(1, max(b - a for a, b in bounds))
+    equal = all(b - a == rows_pad for a, b in bounds[:-1])
+    bufs = {}
+    cur = H
+    for li, (W, bias, relu) in enumerate(layers):
+        f = W.shape[1]
+        key = (li % 2, f)
+        if key not in bufs:
+            bufs[key] = buffers.alloc(key, (rows_pad * world, f), H.dtype, H.device)
+        full, ptrs = bufs[key]
+        local_layer_bcast(li, cur, W, bias, relu, rb, re, ptrs, rank * rows_pad)
+        buffers.barrier(key)
+        if equal:
+            cur = full[:n]
+        else:
             cur = torch.cat([full[r * rows_pad: r * rows_pad + (b - a)] for r, (a, b) in enumerate(bounds)], dim=0)
     return cur

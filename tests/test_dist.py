@@ -124,3 +124,92 @@ def test_gcn_forward_gloo_world2_matches_single_process(balanced):
     for r in range(2):
         assert got[r].shape == ref.shape
         np.testing.assert_allclose(got[r], ref, rtol=1e-12, atol=1e-12)
+
+
+class _EmulatedPeerBuffers:
+    """gloo stand-in for dist.SymmetricBuffers: each rank's buffer is local; the destination
+    'pointers' are labels, and the fused kernel's stores into every rank's copy are emulated by
+    an all-gather of the rows in local_layer_bcast."""
+
+    def __init__(self):
+        self.t = {}
+        self.barriers = 0
+
+    def alloc(self, key, shape, dtype, device):
+        t = torch.full(shape, float("nan"), dtype=dtype, device=device)
+        self.t[key] = t
+        world = dist.get_world_size() if dist.is_initialized() else 1
+        return t, [(key, r) for r in range(world)]
+
+    def barrier(self, key):
+        self.barriers += 1
+        if dist.is_initialized():
+            dist.barrier()
+
+
+def _local_layer_bcast_factory(ip, ic, vals, bufs):
+    layer = _local_layer_factory(ip, ic, vals)
+
+    def local_layer_bcast(l, Hf, W, b, relu, rb, re, dst_ptrs, dst_row0):
+        rows = layer(l, Hf, W, b, relu, rb, re)
+        key = dst_ptrs[0][0]
+        assert [p[1] for p in dst_ptrs] == list(range(len(dst_ptrs)))  # one destination per rank
+        full = bufs.t[key]
+        world = len(dst_ptrs)
+        rows_pad = full.shape[0] // world
+        mine = torch.zeros((rows_pad, full.shape[1]), dtype=full.dtype)
+        mine[: re - rb] = rows
+        parts = [torch.empty_like(mine) for _ in range(world)]
+        if world > 1:
+            dist.all_gather(parts, mine)
+            offs = [None] * world
+            dist.all_gather_object(offs, (dst_row0, re - rb))
+        else:
+            parts, offs = [mine], [(dst_row0, re - rb)]
+        for p, (o, k) in zip(parts, offs):
+            full[o: o + k] = p[:k]
+
+    return local_layer_bcast
+
+
+def _worker_fused(rank, world, port, q, balanced=False):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    ip, ic, vals, H, Ws, bs = _problem()
+    layers = [(Ws[0], bs[0], True), (Ws[1], bs[1], False), (Ws[1].T @ Ws[1][:, :8] * 0 + np.eye(8), bs[1], True)]
+    bufs = _EmulatedPeerBuffers()
+    out = nmdist.gcn_forward_fused(torch.from_numpy(H), layers, _local_layer_bcast_factory(ip, ic, vals, bufs),
+                                   bufs, bounds=_bounds(ip, world, balanced))
+    q.put((rank, out.numpy(), bufs.barriers, sorted(bufs.t)))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("balanced", [False, True])
+def test_gcn_forward_fused_gloo_world2_matches_single_process(balanced):
+    """gcn_forward_fused (all-gather fused into each layer's last kernel): world 2 = world 1 =
+    the collective-based gcn_forward; one barrier per layer; two alternating buffers."""
+    ip, ic, vals, H, Ws, bs = _problem()
+    layers = [(Ws[0], bs[0], True), (Ws[1], bs[1], False), (Ws[1].T @ Ws[1][:, :8] * 0 + np.eye(8), bs[1], True)]
+    ref = nmdist.gcn_forward(torch.from_numpy(H), layers, _local_layer_factory(ip, ic, vals)).numpy()
+    b1 = _EmulatedPeerBuffers()
+    one = nmdist.gcn_forward_fused(torch.from_numpy(H), layers, _local_layer_bcast_factory(ip, ic, vals, b1), b1)
+    np.testing.assert_allclose(one.numpy(), ref, rtol=1e-12, atol=1e-12)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_fused, args=(r, 2, port, q, balanced)) for r in range(2)]
+    for p in procs:
+        p.start()
+    got = {}
+    for _ in range(2):
+        r, out, nbar, keys = q.get(timeout=120)
+        got[r] = out
+        assert nbar == len(layers)
+        assert keys == [(0, 8), (0, 12), (1, 8)]  # layers 0 and 2 share parity 0 only per width
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for r in range(2):
+        np.testing.assert_allclose(got[r], ref, rtol=1e-12, atol=1e-12)

@@ -134,3 +134,67 @@ def test_bench_two_ranks_gloo_on_one_gpu():
     assert len(lines) == 1, r.stdout[-2000:]
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["steps"] == 5
+
+
+def test_gcn_layer_bcast_stores_into_every_destination():
+    """nm_gcn_layer_bcast (the all-gather fused into the layer's last kernel): each of three
+    destination buffers receives exactly nm_gcn_layer's rows at dst_row0, bitwise, and no other
+    row is touched (one GPU: the destinations stand for the ranks' peer-mapped buffers)."""
+    from paper_conf_ppopp_chensz0s25_b200 import api, graphs
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    dev = torch.device("cuda:0")
+    ip, ic, vals, H, Ws, bs = _problem()
+    n = len(ip) - 1
+    perm = np.random.default_rng(3).permutation(n).astype(np.int32)
+    rb, re = 1024, 2304
+    P = api.pack(ip, ic, perm, 1, 2, 4, dtype="bf16", val=vals, row_begin=rb, row_end=re)
+    Hd = torch.from_numpy(graphs.round16(H, "bf16")[0].view(np.int16)).to(dev).view(torch.bfloat16)
+    W = torch.from_numpy(graphs.round16(Ws[0], "bf16")[0].view(np.int16)).to(dev).view(torch.bfloat16)
+    b = torch.from_numpy(bs[0]).to(dev)
+    ws = torch.empty(api.gcn_workspace_bytes(n, 64, 64), dtype=torch.uint8, device=dev)
+    ref = torch.empty((re - rb, 64), dtype=torch.bfloat16, device=dev)
+    api.gcn_layer(P, Hd, W, b, ref, ws, relu=True)
+    sentinel = -12345
+    dsts = [torch.full((4000, 64), sentinel, dtype=torch.int16, device=dev) for _ in range(3)]
+    for order in ("linear", "aggregate"):
+        api.gcn_layer(P, Hd, W, b, ref, ws, relu=True, order=order)
+        api.gcn_layer_bcast(P, Hd, W, b, [d.data_ptr() for d in dsts], 700, 64, ws, relu=True, order=order)
+        torch.cuda.synchronize()
+        for d in dsts:
+            assert torch.equal(d[700:700 + re - rb], ref.view(torch.int16))
+            assert bool((d[:700] == sentinel).all()) and bool((d[700 + re - rb:] == sentinel).all())
+
+
+def test_gcn_forward_fused_world1_equals_collective_forward():
+    """dist.gcn_forward_fused with the real layer (nm_gcn_layer_bcast) and a local buffer at
+    world 1 returns exactly dist.gcn_forward's output."""
+    from paper_conf_ppopp_chensz0s25_b200 import api, graphs
+    from paper_conf_ppopp_chensz0s25_b200 import dist as nmdist
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    dev = torch.device("cuda:0")
+    ip, ic, vals, H, Ws, bs = _problem()
+    n = len(ip) - 1
+    perm = np.random.default_rng(3).permutation(n).astype(np.int32)
+    P = api.pack(ip, ic, perm, 1, 2, 4, dtype="bf16", val=vals)
+
+    def bf(a):
+        return torch.from_numpy(graphs.round16(np.asarray(a, np.float32), "bf16")[0].view(np.int16)).to(dev).view(
+            torch.bfloat16)
+
+    layers = [(bf(W), torch.from_numpy(b).to(dev), relu) for W, b, relu in ((Ws[0], bs[0], True), (Ws[1], bs[1], False))]
+    ws = torch.empty(api.gcn_workspace_bytes(n, 64, 64), dtype=torch.uint8, device=dev)
+
+    def local_layer(li, Hf, W, b, relu, a, z):
+        out = torch.empty((z - a, W.shape[1]), dtype=torch.bfloat16, device=dev)
+        api.gcn_layer(P, Hf, W, b, out, ws, relu=relu)
+        return out
+
+    def local_layer_bcast(li, Hf, W, b, relu, a, z, ptrs, row0):
+        api.gcn_layer_bcast(P, Hf, W, b, ptrs, row0, W.shape[1], ws, relu=relu)
+
+    ref = nmdist.gcn_forward(bf(H), layers, local_layer)
+    got = nmdist.gcn_forward_fused(bf(H), layers, local_layer_bcast, nmdist.LocalBuffers())
+    torch.cuda.synchronize()
+    assert torch.equal(ref.view(torch.int16), got.view(torch.int16))
