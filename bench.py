@@ -287,13 +287,16 @@ def main():
     ap.add_argument("--layout", default="auto", choices=["auto", "reordered", "natural"],
                     help="timed layout: the reorder's, the natural order, or the faster of the two (auto)")
     ap.add_argument("--no-reorder", action="store_true", help="profiling: skip nm_reorder (natural order)")
+    ap.add_argument("--xpad", type=int, default=8, help="X / Y rows padded to a multiple of this many elements "
+                    "(>= 8; e.g. 32 aligns C5's 100-feature rows to 256 B)")
     ap.add_argument("--tau", type=int, default=None, help="hybrid threshold (default: the workload's / nm_hybrid_tau)")
     ap.add_argument("--max-outer", type=int, default=None, help="Alg. 1 cap (default: the workload's, else 10, L496)")
     ap.add_argument("--max-stage1", type=int, default=None)
     ap.add_argument("--max-stage2", type=int, default=None)
     ap.add_argument("--gain-rule", type=int, default=0, help="0 = paper (footnote L440), 1 = positive only")
     ap.add_argument("--sptc-format", type=int, default=0, help="tensor-core kernel: 0 = the pack's choice, 1 = full "
-                    "records, 2 = compressed records (nm_spmm_sptc_format)")
+                    "records, 2 = compressed records, 3 = compressed records with A in tensor memory "
+                    "(nm_spmm_sptc_format)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     w = parse_workload(args.workload)
@@ -353,7 +356,8 @@ def main():
     pack_s = time.perf_counter() - t0
     xbits, _ = graphs.round16(X32, dt)
     tdt = torch.float16 if dt == "f16" else torch.bfloat16
-    Fp = (F + 7) // 8 * 8  # rows padded to 16 B (ldx % 8 == 0; C5's F = 100 -> 104 in memory)
+    xa = max(8, args.xpad)
+    Fp = (F + xa - 1) // xa * xa  # rows padded to 16 B (ldx % 8 == 0; C5's F = 100 -> 104 in memory)
     Xpad = torch.zeros((n, Fp), dtype=torch.int16, device=dev)
     Xpad[:, :F] = torch.from_numpy(xbits.view(np.int16)).to(dev)
     X = Xpad.view(tdt)[:, :F]
@@ -478,7 +482,7 @@ def main():
     fmt = args.sptc_format or 1
     BN = 64 if F <= 64 else (128 if F <= 128 else 256)
     nft = (F + BN - 1) // BN
-    rec_bytes = pst["full_image_bytes"] if fmt != 2 else pst["image_bytes"]
+    rec_bytes = pst["full_image_bytes"] if fmt == 1 else pst["image_bytes"]
     l2_gbs, l2_src = l2_gather_peak()
     clocks = clk.summary()
     sp_tf, sp_src = sparse_peak(bf16_tf, BN, clocks.get("sm_mhz") or clocks.get("sm_max_mhz") or 1965.0)
@@ -488,7 +492,7 @@ def main():
     res_terms = {"hbm_bytes": res["res_nnz"] * 6 + (rows_b + 1) * 8 + res_rows * F * 8,
                  "l2_bytes": res["res_nnz"] * F * 2, "mma_flop": 0.0} if has_res else None
     kern = {"k_spmm_sptc": dict(sptc_terms, ms=statistics.mean(sptc_ms),
-                                format="full" if fmt != 2 else "compressed")}
+                                format={1: "full", 2: "compressed", 3: "compressed-tmem"}[fmt])}
     if has_res:
         kern["k_residual"] = dict(res_terms, ms=statistics.mean(b - a for a, b in zip(sptc_ms, step_ms)))
     for k in kern.values():

@@ -19,7 +19,7 @@ OBJ = os.path.join(PKG, "_build")
 LIB = os.path.join(PKG, "libnm.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
-SOURCES = ["capi.cu", "pack.cu", "spmm_sm100.cu", "spmm_full_sm100.cu", "ops.cu", "models.cu", "counts.cu", "gcn.cu", "reorder.cpp",
+SOURCES = ["capi.cu", "pack.cu", "spmm_sm100.cu", "spmm_full_sm100.cu", "spmm_tm_sm100.cu", "ops.cu", "models.cu", "counts.cu", "gcn.cu", "reorder.cpp",
            "reorder_gpu.cu"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-lineinfo", "-std=c++17", "-I" + os.path.join(ROOT, "include"),

@@ -100,7 +100,7 @@ struct nm_packed {
   uint8_t* image_full = nullptr;       // full chunk records (kChunkBytes each, chunk order)
   int32_t* cta_ptr = nullptr;          // [n_ctas+1] contiguous panel range of each SpMM CTA
   int n_ctas = 0;                      // persistent grid of the full-record kernel (#SMs)
-  int sptc_format = 1;                 // tensor-core kernel nm_spmm uses: 1 full, 2 compressed
+  int sptc_format = 1;                 // tensor-core kernel nm_spmm uses: 1 full, 2 compressed, 3 compressed + A in TMEM
   int64_t gather_rows = 0;             // non-negative gather rows over all chunks
   int64_t* res_rowptr = nullptr;       // [rows+1]
   int32_t* res_col = nullptr;          // [res_nnz] canonical (permuted) column
@@ -191,6 +191,8 @@ nm_status launch_spmm_sptc_full(const nm_packed* P, const void* PX, int64_t ldx,
                                 int64_t ldy, int F, cudaStream_t s);
 nm_status launch_spmm_sptc_compressed(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                                       int64_t ldy, int F, cudaStream_t s);
+nm_status launch_spmm_sptc_tm(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
+                              int64_t ldy, int F, cudaStream_t s);
 nm_status launch_spmm_residual(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                                int64_t ldy, int F, cudaStream_t s);
 nm_status gemm_rm(const void* A, int64_t lda, const void* W, int64_t ldw, void* C, int64_t ldc, int64_t m, int k,

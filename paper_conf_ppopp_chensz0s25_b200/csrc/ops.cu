@@ -310,6 +310,7 @@ nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, floa
                            cudaStream_t s, int format) {
   if (format == 0) format = P->sptc_format;
   if (format == 2) return launch_spmm_sptc_compressed(P, PX, ldx, Yp, ldy, F, s);
+  if (format == 3) return launch_spmm_sptc_tm(P, PX, ldx, Yp, ldy, F, s);
   return launch_spmm_sptc_full(P, PX, ldx, Yp, ldy, F, s);
 }
 
@@ -430,7 +431,7 @@ nm_status nm_spmm_sptc_format(const nm_packed* P, const void* PX, int64_t ldx, f
                               int format, void* stream) {
   nm_status st = check_spmm_args(P, PX, ldx, Yp, ldy, F);
   if (st != NM_OK) return st;
-  if (format < 0 || format > 2) return fail(NM_ERR_INVALID_ARG, "nm_spmm_sptc_format: format must be 0, 1 or 2");
+  if (format < 0 || format > 3) return fail(NM_ERR_INVALID_ARG, "nm_spmm_sptc_format: format must be 0, 1, 2 or 3");
   return launch_spmm_sptc(P, PX, ldx, Yp, ldy, F, (cudaStream_t)stream, format);
 }
 

@@ -373,9 +373,9 @@ def test_concurrent_spmm_on_one_handle(dtype):
 @pytest.mark.parametrize("kind,seed,V,M", CASES)
 @pytest.mark.parametrize("F", [32, 128, 300])
 def test_sptc_formats_agree_bitwise(kind, seed, V, M, F):
-    """The full-record kernel (format 1, nm_spmm's default) and the compressed-record kernel
-    (format 2) feed the tensor core identical operands in the same order: Yp must agree
-    bitwise, and both must meet the oracle bound."""
+    """The full-record kernel (format 1), the compressed-record kernel (format 2) and the
+    compressed-record kernel with A in tensor memory (format 3) feed the tensor core identical
+    operands in the same order: Yp must agree bitwise, and all must meet the oracle bound."""
     dev = _cuda()
     ip, ic = _graph(kind, seed)
     n = len(ip) - 1
@@ -390,13 +390,14 @@ def test_sptc_formats_agree_bitwise(kind, seed, V, M, F):
     X = Xb.view(tdt)[:, :F]
     P = api.pack(ip, ic, perm, V, 2, M, dtype=dtype, val=v32, order="original")
     outs = []
-    for fmt in (1, 2):
+    for fmt in (1, 2, 3):
         Y = torch.full((n, F), float("nan"), device=dev)
         api.spmm(P, X, Y, part="sptc", format=fmt)
         api.spmm(P, X, Y, part="residual")
         torch.cuda.synchronize()
         outs.append(Y.cpu().numpy())
     assert np.array_equal(outs[0], outs[1])
+    assert np.array_equal(outs[0], outs[2])
     Y_ref, E, _ = oracle.spmm(ip, ic, v64, x64)
     err = np.abs(outs[0].astype(np.float64) - Y_ref)
     assert (err <= TOL * E).all(), err.max()
