@@ -152,12 +152,13 @@ NM_API nm_status nm_count_violations(const nm_csr* A, const int32_t* perm, int V
  * its first <= 2 nonzeros among them (N = 2, horizontal constraint L229-230) as two 16-bit
  * values plus a 4-bit index pair.  Everything else goes to a residual CSR.  Device memory
  * holds the MMA-native image consumed by nm_spmm (tcgen05.mma.sp operands).
- * Supported: N = 2; M in {4, 8, 16}; any V >= 1 (V = 1 -> Mp = 4); Vp in {64, 128}
- * (0 = auto: 64 when V == 64, else 128); dtype NM_F16 or NM_BF16 (values are rounded from
- * val_dtype to dtype).  The tensor-core kernel always runs M = 128 MMAs over 128-row kernel
- * panels; at Vp = 64 a kernel panel's chunks hold the meta-blocks of both of its 64-row
- * panels (in canonical order), each k-group carrying the values of one half and no-value
- * nibbles in the other, so a V = 64 conforming matrix packs with an empty residual.
+ * Supported: N = 2; M in {4, 8, 16}; any V >= 1 (V = 1 -> Mp = 4); Vp in {16, 32, 64, 128}
+ * (0 = auto: V when V is 16, 32 or 64, else 128); dtype NM_F16 or NM_BF16 (values are rounded
+ * from val_dtype to dtype).  The tensor-core kernel always runs M = 128 MMAs over 128-row
+ * kernel panels; at Vp < 128 a kernel panel's chunks hold the meta-blocks of its 128 / Vp
+ * canonical panels (in canonical order), each k-group carrying the values of one panel's rows
+ * and no-value nibbles in the others, so a V:2:M conforming matrix (V = Vp) packs with an
+ * empty residual.
  * ------------------------------------------------------------------------------------- */
 typedef struct nm_packed nm_packed;
 

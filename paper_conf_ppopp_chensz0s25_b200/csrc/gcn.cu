@@ -98,122 +98,120 @@ __global__ void k_to16(const float* __restrict__ Y, int64_t total, uint16_t* __r
   }
 }
 
-struct LtHandle {
-  cublasLtHandle_t h = nullptr;
-  ~LtHandle() {
-    if (h) cublasLtDestroy(h);
-  }
-};
-
 nm_status lt_fail(cublasStatus_t s, const char* what) {
   return fail(NM_ERR_CUDA, std::string(what) + ": cublasLt status " + std::to_string((int)s));
 }
 
-// C[m x nc] = A[m x k] * W[k x nc], all row-major; A, W 16-bit, C 16-bit or fp32.  Computed as
-// the column-major product C^T = W^T A^T (no transposes needed).
-nm_status dense_gemm(const void* A, const void* W, void* C, int64_t m, int k, int nc, nm_dtype dt, bool c_f32,
-                     void* ws, cudaStream_t s) {
-  static thread_local LtHandle lt;
-  if (!lt.h) {
-    cublasStatus_t r = cublasLtCreate(&lt.h);
-    if (r != CUBLAS_STATUS_SUCCESS) return lt_fail(r, "cublasLtCreate");
-  }
-  if (m == 0) return NM_OK;
-  const cudaDataType_t ty = dt == NM_BF16 ? CUDA_R_16BF : CUDA_R_16F;
-  const cudaDataType_t cty = c_f32 ? CUDA_R_32F : ty;
+// One cuBLASLt problem: descriptors, layouts and the heuristic's algorithm, built once per
+// shape and kept (per thread) for later calls -- nm_gcn_layer and the models call the same
+// shapes every layer / step.
+struct LtPlan {
+  bool ta, tb, c_f32;
+  int64_t m, nn, k, lda, ldb, ldc;
+  nm_dtype dt;
   cublasLtMatmulDesc_t op = nullptr;
   cublasLtMatrixLayout_t la = nullptr, lb = nullptr, lc = nullptr;
-  cublasLtMatmulPreference_t pref = nullptr;
-  nm_status st = NM_OK;
-  do {
-    if (cublasLtMatmulDescCreate(&op, CUBLAS_COMPUTE_32F, CUDA_R_32F) != CUBLAS_STATUS_SUCCESS) {
-      st = fail(NM_ERR_CUDA, "cublasLtMatmulDescCreate");
-      break;
-    }
-    if (cublasLtMatrixLayoutCreate(&la, ty, nc, k, nc) != CUBLAS_STATUS_SUCCESS ||
-        cublasLtMatrixLayoutCreate(&lb, ty, k, m, k) != CUBLAS_STATUS_SUCCESS ||
-        cublasLtMatrixLayoutCreate(&lc, cty, nc, m, nc) != CUBLAS_STATUS_SUCCESS) {
-      st = fail(NM_ERR_CUDA, "cublasLtMatrixLayoutCreate");
-      break;
-    }
-    if (cublasLtMatmulPreferenceCreate(&pref) != CUBLAS_STATUS_SUCCESS) {
-      st = fail(NM_ERR_CUDA, "cublasLtMatmulPreferenceCreate");
-      break;
-    }
-    size_t wsb = kLtWorkspace;
-    cublasLtMatmulPreferenceSetAttribute(pref, CUBLASLT_MATMUL_PREF_MAX_WORKSPACE_BYTES, &wsb, sizeof(wsb));
-    cublasLtMatmulHeuristicResult_t heur;
-    int nres = 0;
-    if (cublasLtMatmulAlgoGetHeuristic(lt.h, op, la, lb, lc, lc, pref, 1, &heur, &nres) != CUBLAS_STATUS_SUCCESS ||
-        nres == 0) {
-      st = fail(NM_ERR_CUDA, "cublasLt: no algorithm");
-      break;
-    }
-    const float one = 1.f, zero = 0.f;
-    cublasStatus_t r = cublasLtMatmul(lt.h, op, &one, W, la, A, lb, &zero, C, lc, C, lc, &heur.algo, ws, wsb, s);
-    if (r != CUBLAS_STATUS_SUCCESS) st = lt_fail(r, "cublasLtMatmul");
-  } while (0);
-  if (pref) cublasLtMatmulPreferenceDestroy(pref);
-  if (la) cublasLtMatrixLayoutDestroy(la);
-  if (lb) cublasLtMatrixLayoutDestroy(lb);
-  if (lc) cublasLtMatrixLayoutDestroy(lc);
-  if (op) cublasLtMatmulDescDestroy(op);
-  return st;
-}
+  cublasLtMatmulAlgo_t algo;
+  void destroy() {
+    if (la) cublasLtMatrixLayoutDestroy(la);
+    if (lb) cublasLtMatrixLayoutDestroy(lb);
+    if (lc) cublasLtMatrixLayoutDestroy(lc);
+    if (op) cublasLtMatmulDescDestroy(op);
+    la = lb = lc = nullptr;
+    op = nullptr;
+  }
+  bool same(bool ta_, bool tb_, int64_t m_, int64_t nn_, int64_t k_, int64_t lda_, int64_t ldb_, int64_t ldc_,
+            nm_dtype dt_, bool c_) const {
+    return ta == ta_ && tb == tb_ && m == m_ && nn == nn_ && k == k_ && lda == lda_ && ldb == ldb_ && ldc == ldc_ &&
+           dt == dt_ && c_f32 == c_;
+  }
+};
+
+struct LtCache {
+  cublasLtHandle_t h = nullptr;
+  static constexpr int kSlots = 16;
+  LtPlan plans[kSlots];
+  int used = 0, next = 0;
+  ~LtCache() {
+    for (int i = 0; i < used; ++i) plans[i].destroy();
+    if (h) cublasLtDestroy(h);
+  }
+};
 
 // General column-major product C[m x nn] = op(A)[m x k] op(B)[k x nn] (cuBLASLt, fp32
 // accumulation); A/B 16-bit, C 16-bit or fp32; lda/ldb/ldc are column-major leading dims.
 nm_status lt_gemm(bool ta, bool tb, int64_t m, int64_t nn, int64_t k, const void* A, int64_t lda, const void* B,
                   int64_t ldb, void* C, int64_t ldc, nm_dtype dt, bool c_f32, void* ws, cudaStream_t s) {
-  static thread_local LtHandle lt;
+  static thread_local LtCache lt;
   if (!lt.h) {
     cublasStatus_t r = cublasLtCreate(&lt.h);
     if (r != CUBLAS_STATUS_SUCCESS) return lt_fail(r, "cublasLtCreate");
   }
   if (m == 0 || nn == 0) return NM_OK;
-  const cudaDataType_t ty = dt == NM_BF16 ? CUDA_R_16BF : CUDA_R_16F;
-  const cudaDataType_t cty = c_f32 ? CUDA_R_32F : ty;
-  cublasLtMatmulDesc_t op = nullptr;
-  cublasLtMatrixLayout_t la = nullptr, lb = nullptr, lc = nullptr;
-  cublasLtMatmulPreference_t pref = nullptr;
-  nm_status st = NM_OK;
-  do {
-    if (cublasLtMatmulDescCreate(&op, CUBLAS_COMPUTE_32F, CUDA_R_32F) != CUBLAS_STATUS_SUCCESS) {
-      st = fail(NM_ERR_CUDA, "cublasLtMatmulDescCreate");
-      break;
+  LtPlan* plan = nullptr;
+  for (int i = 0; i < lt.used && !plan; ++i)
+    if (lt.plans[i].same(ta, tb, m, nn, k, lda, ldb, ldc, dt, c_f32)) plan = &lt.plans[i];
+  if (!plan) {
+    LtPlan np;
+    np.ta = ta; np.tb = tb; np.c_f32 = c_f32; np.m = m; np.nn = nn; np.k = k;
+    np.lda = lda; np.ldb = ldb; np.ldc = ldc; np.dt = dt;
+    const cudaDataType_t ty = dt == NM_BF16 ? CUDA_R_16BF : CUDA_R_16F;
+    const cudaDataType_t cty = c_f32 ? CUDA_R_32F : ty;
+    cublasLtMatmulPreference_t pref = nullptr;
+    nm_status st = NM_OK;
+    do {
+      if (cublasLtMatmulDescCreate(&np.op, CUBLAS_COMPUTE_32F, CUDA_R_32F) != CUBLAS_STATUS_SUCCESS) {
+        st = fail(NM_ERR_CUDA, "cublasLtMatmulDescCreate");
+        break;
+      }
+      const cublasOperation_t opa = ta ? CUBLAS_OP_T : CUBLAS_OP_N, opb = tb ? CUBLAS_OP_T : CUBLAS_OP_N;
+      cublasLtMatmulDescSetAttribute(np.op, CUBLASLT_MATMUL_DESC_TRANSA, &opa, sizeof(opa));
+      cublasLtMatmulDescSetAttribute(np.op, CUBLASLT_MATMUL_DESC_TRANSB, &opb, sizeof(opb));
+      if (cublasLtMatrixLayoutCreate(&np.la, ty, ta ? k : m, ta ? m : k, lda) != CUBLAS_STATUS_SUCCESS ||
+          cublasLtMatrixLayoutCreate(&np.lb, ty, tb ? nn : k, tb ? k : nn, ldb) != CUBLAS_STATUS_SUCCESS ||
+          cublasLtMatrixLayoutCreate(&np.lc, cty, m, nn, ldc) != CUBLAS_STATUS_SUCCESS) {
+        st = fail(NM_ERR_CUDA, "cublasLtMatrixLayoutCreate");
+        break;
+      }
+      if (cublasLtMatmulPreferenceCreate(&pref) != CUBLAS_STATUS_SUCCESS) {
+        st = fail(NM_ERR_CUDA, "cublasLtMatmulPreferenceCreate");
+        break;
+      }
+      size_t wsb = kLtWorkspace;
+      cublasLtMatmulPreferenceSetAttribute(pref, CUBLASLT_MATMUL_PREF_MAX_WORKSPACE_BYTES, &wsb, sizeof(wsb));
+      cublasLtMatmulHeuristicResult_t heur;
+      int nres = 0;
+      if (cublasLtMatmulAlgoGetHeuristic(lt.h, np.op, np.la, np.lb, np.lc, np.lc, pref, 1, &heur, &nres) !=
+              CUBLAS_STATUS_SUCCESS ||
+          nres == 0) {
+        st = fail(NM_ERR_CUDA, "cublasLt: no algorithm");
+        break;
+      }
+      np.algo = heur.algo;
+    } while (0);
+    if (pref) cublasLtMatmulPreferenceDestroy(pref);
+    if (st != NM_OK) {
+      np.destroy();
+      return st;
     }
-    const cublasOperation_t opa = ta ? CUBLAS_OP_T : CUBLAS_OP_N, opb = tb ? CUBLAS_OP_T : CUBLAS_OP_N;
-    cublasLtMatmulDescSetAttribute(op, CUBLASLT_MATMUL_DESC_TRANSA, &opa, sizeof(opa));
-    cublasLtMatmulDescSetAttribute(op, CUBLASLT_MATMUL_DESC_TRANSB, &opb, sizeof(opb));
-    if (cublasLtMatrixLayoutCreate(&la, ty, ta ? k : m, ta ? m : k, lda) != CUBLAS_STATUS_SUCCESS ||
-        cublasLtMatrixLayoutCreate(&lb, ty, tb ? nn : k, tb ? k : nn, ldb) != CUBLAS_STATUS_SUCCESS ||
-        cublasLtMatrixLayoutCreate(&lc, cty, m, nn, ldc) != CUBLAS_STATUS_SUCCESS) {
-      st = fail(NM_ERR_CUDA, "cublasLtMatrixLayoutCreate");
-      break;
-    }
-    if (cublasLtMatmulPreferenceCreate(&pref) != CUBLAS_STATUS_SUCCESS) {
-      st = fail(NM_ERR_CUDA, "cublasLtMatmulPreferenceCreate");
-      break;
-    }
-    size_t wsb = kLtWorkspace;
-    cublasLtMatmulPreferenceSetAttribute(pref, CUBLASLT_MATMUL_PREF_MAX_WORKSPACE_BYTES, &wsb, sizeof(wsb));
-    cublasLtMatmulHeuristicResult_t heur;
-    int nres = 0;
-    if (cublasLtMatmulAlgoGetHeuristic(lt.h, op, la, lb, lc, lc, pref, 1, &heur, &nres) != CUBLAS_STATUS_SUCCESS ||
-        nres == 0) {
-      st = fail(NM_ERR_CUDA, "cublasLt: no algorithm");
-      break;
-    }
-    const float one = 1.f, zero = 0.f;
-    cublasStatus_t r = cublasLtMatmul(lt.h, op, &one, A, la, B, lb, &zero, C, lc, C, lc, &heur.algo, ws, wsb, s);
-    if (r != CUBLAS_STATUS_SUCCESS) st = lt_fail(r, "cublasLtMatmul");
-  } while (0);
-  if (pref) cublasLtMatmulPreferenceDestroy(pref);
-  if (la) cublasLtMatrixLayoutDestroy(la);
-  if (lb) cublasLtMatrixLayoutDestroy(lb);
-  if (lc) cublasLtMatrixLayoutDestroy(lc);
-  if (op) cublasLtMatmulDescDestroy(op);
-  return st;
+    // keep it: fill free slots, then replace round-robin
+    int slot = lt.used < LtCache::kSlots ? lt.used++ : (lt.next++ % LtCache::kSlots);
+    if (slot < lt.used && lt.plans[slot].op) lt.plans[slot].destroy();
+    lt.plans[slot] = np;
+    plan = &lt.plans[slot];
+  }
+  const float one = 1.f, zero = 0.f;
+  cublasStatus_t r = cublasLtMatmul(lt.h, plan->op, &one, A, plan->la, B, plan->lb, &zero, C, plan->lc, C, plan->lc,
+                                    &plan->algo, ws, kLtWorkspace, s);
+  if (r != CUBLAS_STATUS_SUCCESS) return lt_fail(r, "cublasLtMatmul");
+  return NM_OK;
+}
+
+// C[m x nc] = A[m x k] * W[k x nc], all row-major; A, W 16-bit, C 16-bit or fp32: the
+// column-major product C^T = W^T A^T (no transposes needed).
+nm_status dense_gemm(const void* A, const void* W, void* C, int64_t m, int k, int nc, nm_dtype dt, bool c_f32,
+                     void* ws, cudaStream_t s) {
+  return lt_gemm(false, false, nc, m, k, W, nc, A, k, C, nc, dt, c_f32, ws, s);
 }
 
 // dZ = relu ? dHout * [Hout > 0] : dHout (16-bit in and out, exact), and a 16-bit ones

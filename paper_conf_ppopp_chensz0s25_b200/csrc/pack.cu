@@ -611,8 +611,9 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   if (N != 2) return fail(NM_ERR_UNSUPPORTED, "nm_pack: N must be 2 (hardware 2:4, L496)");
   if (!(M == 4 || M == 8 || M == 16)) return fail(NM_ERR_UNSUPPORTED, "nm_pack: M must be 4, 8 or 16");
   if (V < 1) return fail(NM_ERR_INVALID_ARG, "nm_pack: V < 1");
-  if (Vp == 0) Vp = (V == 64) ? 64 : kPanelRows;
-  if (Vp != 64 && Vp != kPanelRows) return fail(NM_ERR_UNSUPPORTED, "nm_pack: Vp must be 64 or 128");
+  if (Vp == 0) Vp = (V == 16 || V == 32 || V == 64) ? V : kPanelRows;
+  if (Vp != 16 && Vp != 32 && Vp != 64 && Vp != kPanelRows)
+    return fail(NM_ERR_UNSUPPORTED, "nm_pack: Vp must be 16, 32, 64 or 128");
   const int ratio = kPanelRows / Vp;  // canonical panels per kernel panel
   if (dtype != NM_F16 && dtype != NM_BF16) return fail(NM_ERR_UNSUPPORTED, "nm_pack: dtype must be f16 or bf16");
   const int64_t n = A->n;

@@ -58,7 +58,7 @@ def test_reorder_rejects_bad_csr_and_asymmetric():
 
 
 def test_pack_support_set_rejected_cleanly():
-    """nm.h's support set for nm_pack: Vp in {64, 128} (0 = auto), N = 2,
+    """nm.h's support set for nm_pack: Vp in {16, 32, 64, 128} (0 = auto), N = 2,
     M in {4, 8, 16}, 16-bit dtypes.  Anything else is NM_ERR_UNSUPPORTED before any device work."""
     import ctypes
 
@@ -68,7 +68,7 @@ def test_pack_support_set_rejected_cleanly():
     ip, ic = np.array([0, 1, 2], np.int64), np.array([1, 0], np.int32)
     c, keep = api._csr_struct(ip, ic)
     h = ctypes.c_void_p()
-    for V, N, M, Vp, dt in [(1, 2, 4, 32, _lib.NM_F16), (64, 2, 8, 256, _lib.NM_BF16), (1, 3, 4, 128, _lib.NM_F16),
+    for V, N, M, Vp, dt in [(1, 2, 4, 8, _lib.NM_F16), (64, 2, 8, 256, _lib.NM_BF16), (1, 2, 4, 48, _lib.NM_F16), (1, 3, 4, 128, _lib.NM_F16),
                             (1, 2, 32, 128, _lib.NM_F16), (1, 2, 4, 128, _lib.NM_F32)]:
         st = lib.nm_pack(ctypes.byref(c), None, V, N, M, Vp, dt, None, ctypes.byref(h))
         assert st == _lib.NM_ERR_UNSUPPORTED, (V, N, M, Vp, dt, st)

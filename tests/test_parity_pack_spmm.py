@@ -56,8 +56,8 @@ def test_counts(kind, seed, V, M):
 
 
 def _vp(V):
-    """nm_pack's automatic panel height (nm.h): 64 for V = 64 patterns, else 128."""
-    return 64 if V == 64 else 128
+    """nm_pack's automatic panel height (nm.h): V for V = 16, 32, 64 patterns, else 128."""
+    return V if V in (16, 32, 64) else 128
 
 
 def _values(ip, ic, dtype, seed):
@@ -408,7 +408,8 @@ def test_sptc_formats_agree_bitwise(kind, seed, V, M, F):
 # panel's chunks, each k-group holding one half's values)
 # ------------------------------------------------------------------------------------------
 @pytest.mark.parametrize("kind,seed,V,M,Vp", [("band", 5, 64, 8, 64), ("band", 5, 64, 8, 128), ("pl", 3, 1, 4, 64),
-                                              ("pl", 6, 128, 16, 64), ("er", 7, 8, 8, 64), ("tiny", 1, 1, 4, 64)])
+                                              ("pl", 6, 128, 16, 64), ("er", 7, 8, 8, 64), ("tiny", 1, 1, 4, 64),
+                                              ("band", 4, 16, 8, 16), ("pl", 3, 32, 8, 32), ("er", 2, 32, 16, 16)])
 @pytest.mark.parametrize("order", ["permuted", "original"])
 def test_panel_height_vp(kind, seed, V, M, Vp, order):
     dev = _cuda()
@@ -442,11 +443,11 @@ def test_panel_height_vp(kind, seed, V, M, Vp, order):
         # 128-row kernel panels pair different 64-row panels than the whole pack's, so the
         # chunking (and the fp32 summation grouping inside each MMA) differs: checked against
         # the oracle bound, not bitwise against Y.
-        if Vp == 64 and n > 256:
-            cut = ((n // 2) // 128) * 128 + 64
+        if Vp < 128 and n > 256:
+            cut = ((n // 2) // 128) * 128 + Vp
             Y2 = torch.full((n, F), float("nan"), device=dev)
             for a, b in ((0, cut), (cut, n)):
-                Ps = api.pack(ip, ic, perm, V, 2, M, dtype="bf16", val=v32, order="original", Vp=64,
+                Ps = api.pack(ip, ic, perm, V, 2, M, dtype="bf16", val=v32, order="original", Vp=Vp,
                               row_begin=a, row_end=b)
                 api.spmm(Ps, X, Y2, F=F)
             torch.cuda.synchronize()
@@ -457,19 +458,20 @@ def test_panel_height_vp(kind, seed, V, M, Vp, order):
     assert (err <= TOL * E).all(), err.max()
 
 
-def test_vp64_conforming_v64_has_empty_residual():
-    """A 64:2:8-conforming matrix (every 64-row x 8-column meta-block uses <= 4 columns, every
+@pytest.mark.parametrize("V", [16, 64])
+def test_vp64_conforming_v64_has_empty_residual(V):
+    """A V:2:8-conforming matrix (every V-row x 8-column meta-block uses <= 4 columns, every
     row <= 2 per 8-segment, L194 / L226-230) packs losslessly into the tensor-core form at
-    Vp = 64, where 128-row panels would merge two halves' column sets and spill."""
+    Vp = V, where 128-row panels would merge the blocks' column sets and spill."""
     _cuda()
     rng = np.random.default_rng(5)
     n, M = 1024, 8
     rows = [[] for _ in range(n)]
-    for p in range(n // 64):
+    for p in range(n // V):
         for s in range(n // M):
             if rng.random() < 0.25:
                 cols = s * M + np.sort(rng.choice(M, 4, replace=False))
-                for i in range(p * 64, p * 64 + 64):
+                for i in range(p * V, p * V + V):
                     if rng.random() < 0.5:
                         rows[i].extend(rng.choice(cols, 2, replace=False).tolist())
     ip = np.zeros(n + 1, np.int64)
@@ -480,12 +482,12 @@ def test_vp64_conforming_v64_has_empty_residual():
         ip[i + 1] = ip[i] + len(r)
     ic = np.array(ic, np.int32)
     ident = np.arange(n, dtype=np.int32)
-    P64 = api.pack(ip, ic, ident, 64, 2, M)
-    P128 = api.pack(ip, ic, ident, 64, 2, M, Vp=128)
-    assert P64.stats()["Vp"] == 64 and P128.stats()["Vp"] == 128
+    P64 = api.pack(ip, ic, ident, V, 2, M)
+    P128 = api.pack(ip, ic, ident, V, 2, M, Vp=128)
+    assert P64.stats()["Vp"] == V and P128.stats()["Vp"] == 128
     assert P64.info()["residual_nnz"] == 0
     assert P128.info()["residual_nnz"] > 0
-    ref = oracle.pack(ip, ic, None, 0x3C00, ident, 64, M)
+    ref = oracle.pack(ip, ic, None, 0x3C00, ident, V, M)
     assert ref["res_nnz"] == 0
     got = P64.export_canonical()
     for k in ("panel_ptr", "mb_seg", "sel", "nib", "vals"):

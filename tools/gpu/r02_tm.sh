@@ -1,7 +1,7 @@
 # compressed records with A in tensor memory (format 3): parity, then A/B vs full records
 set -x
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
-timeout 900 python -m pytest tests/test_parity_pack_spmm.py -q -x --timeout 600 -p no:cacheprovider -k "formats_agree" > gpurun_out/t_tm.log 2>&1; echo tests=$?; tail -15 gpurun_out/t_tm.log
+timeout 1200 python -m pytest tests/test_parity_pack_spmm.py tests/test_parity_gcn.py tests/test_parity_models.py tests/test_score_patterns.py tests/test_dist_gpu.py -q --timeout 600 -p no:cacheprovider -k "formats_agree or panel_height or conforming or gcn or sgc or sage or cheb or score or bcast or fused" > gpurun_out/t_tm.log 2>&1; echo tests=$?; tail -15 gpurun_out/t_tm.log
 summ() { python - $1 <<'PY'
 import json,sys
 try:
