@@ -52,7 +52,7 @@ WORKLOADS = {
 }
 # configs[1] (SuiteSparse-shaped sweep): any point named
 #   c2-{banded|powerlaw}-n{65k|262k|1m}-d{8|16|32|64}-f{F}-{V}:2:{M}[-tau{T}]
-# (tau omitted = the library's cost-model threshold nm_hybrid_tau(F); tau0 = plain pack).
+# (tau omitted = nm_pack_auto: the threshold minimising the library's time model; tau0 = plain pack).
 DEFAULT = "c3-reddit-f128-1:2:4"  # configs[2], the N = 1 headline
 SWEEP = ["c2-banded-n1m-d16-f128-1:2:4", "c2-banded-n1m-d32-f128-1:2:4", "c2-banded-n262k-d16-f128-64:2:8",
          "c2-powerlaw-n262k-d16-f128-1:2:4", "c2-powerlaw-n262k-d16-f128-128:2:16"]
@@ -287,9 +287,9 @@ def main():
     ap.add_argument("--layout", default="auto", choices=["auto", "reordered", "natural"],
                     help="timed layout: the reorder's, the natural order, or the faster of the two (auto)")
     ap.add_argument("--no-reorder", action="store_true", help="profiling: skip nm_reorder (natural order)")
-    ap.add_argument("--xpad", type=int, default=8, help="X / Y rows padded to a multiple of this many elements "
+    ap.add_argument("--xpad", type=int, default=32, help="X / Y rows padded to a multiple of this many elements "
                     "(>= 8; e.g. 32 aligns C5's 100-feature rows to 256 B)")
-    ap.add_argument("--tau", type=int, default=None, help="hybrid threshold (default: the workload's / nm_hybrid_tau)")
+    ap.add_argument("--tau", type=int, default=None, help="hybrid threshold (default: the workload's / nm_pack_auto)")
     ap.add_argument("--max-outer", type=int, default=None, help="Alg. 1 cap (default: the workload's, else 10, L496)")
     ap.add_argument("--max-stage1", type=int, default=None)
     ap.add_argument("--max-stage2", type=int, default=None)
@@ -350,14 +350,16 @@ def main():
     from paper_conf_ppopp_chensz0s25_b200.dist import balanced_bounds, panel_costs
     rb, re = balanced_bounds(panel_costs(ip, perm), n, world)[rank]
     t0 = time.perf_counter()
-    tau = w["tau"] if w["tau"] is not None else api.hybrid_tau(F)
-    P = api.pack(ip, ic, perm, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order=args.order, tau=tau)
+    # hybrid threshold: the workload's / --tau, else nm_pack_auto (the tau minimising the
+    # library's time model for this F)
+    tau = w["tau"] if w["tau"] is not None else "auto"
+    P = api.pack(ip, ic, perm, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order=args.order, tau=tau, F=F)
     torch.cuda.synchronize()
     pack_s = time.perf_counter() - t0
     xbits, _ = graphs.round16(X32, dt)
     tdt = torch.float16 if dt == "f16" else torch.bfloat16
-    xa = max(8, args.xpad)
-    Fp = (F + xa - 1) // xa * xa  # rows padded to 16 B (ldx % 8 == 0; C5's F = 100 -> 104 in memory)
+    xa = max(8, args.xpad)  # 32: 64-byte rows, the gathers' DRAM sectors aligned (C5: 100 -> 128)
+    Fp = (F + xa - 1) // xa * xa  # X / Y row pitch (ldx % 8 == 0)
     Xpad = torch.zeros((n, Fp), dtype=torch.int16, device=dev)
     Xpad[:, :F] = torch.from_numpy(xbits.view(np.int16)).to(dev)
     X = Xpad.view(tdt)[:, :F]
@@ -367,7 +369,8 @@ def main():
     # natural order, each packed and timed for a few L2-flushed steps; the faster one is timed
     layout_trial = None
     if args.layout == "auto" and args.order == "original":
-        P_nat = api.pack(ip, ic, None, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order="original", tau=tau)
+        P_nat = api.pack(ip, ic, None, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order="original", tau=tau,
+                         F=F)
         trial = {}
         for name, Pk in (("reordered", P), ("natural", P_nat)):
             for _ in range(3):
@@ -391,8 +394,10 @@ def main():
         else:
             del P_nat
     elif args.layout == "natural":
-        P = api.pack(ip, ic, None, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order=args.order, tau=tau)
+        P = api.pack(ip, ic, None, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order=args.order, tau=tau,
+                     F=F)
         perm = np.arange(n, dtype=np.int32)
+    tau = P.tau  # the threshold actually packed with
     info = P.info()
     perm_d = torch.from_numpy(perm).to(dev)
     PX = padded_like(X) if args.order == "permuted" else None

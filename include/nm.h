@@ -104,11 +104,11 @@ NM_API nm_status nm_reorder(const nm_csr* A, int V, int N, int M, const nm_reord
 /* nm_reorder_gpu -- nm_reorder with Stage-1 (Alg. 2 lines 4-13: Hamming position codes of
  * every (row, segment) of B, L339-346 / Listing 1, and the stable lexicographic row
  * sort, L366-384) and the omega / MBscore counts (L203, L382) run on the current CUDA device
- * (the paper's SOGRE is a GPU library, L484).  Stage-2 (Alg. 3): the
- * M x M gain tables of each batch of (primary, target) pairs are computed on the device
- * (L448-455); the picks (freshtop, the est / I bookkeeping) stay on the host because the
- * greedy is sequential in the recorded pairs.  The permutation is bit-identical to
- * nm_reorder's and to the CPU oracle's.
+ * (the paper's SOGRE is a GPU library, L484).  Stage-2 (Alg. 3) stays on
+ * the host: its greedy is sequential in the recorded pairs, and its M x M gain tables are
+ * computed in parallel batches with OpenMP (a device version of the tables, bit-identical,
+ * is built with -DNM_S2_DEVICE_TABLES=1 but measured slower on B200).  The
+ * permutation is bit-identical to nm_reorder's and to the CPU oracle's.
  *   A, V, N, M, opts, perm_out, st : as nm_reorder (A host or device CSR; perm_out host).
  *   stream : cudaStream_t the device work is ordered on (NULL = legacy default stream).
  * Synchronous on return.  Device memory: ~ 60 bytes per stored entry + 60 per vertex, from a
@@ -128,9 +128,8 @@ NM_API nm_status nm_select_pattern(const nm_csr* A, int max_M, int max_V, const 
 /* nm_score_patterns -- best-V:N:M selection scored by the packed form:
  * nm_select_pattern keeps the last pattern the reordered graph CONFORMS to (L496, L655); this
  * scores what the SpMM would move.  For each candidate (V[i], M[i]), N = 2: nm_reorder_gpu with
- * opts, nm_pack_hybrid at nm_hybrid_tau(F) (Vp auto), score = n_chunks * (0.28 + 0.0075 F) +
- * residual_nnz * 0.00016 F (ns: the B200 time model nm_hybrid_tau is derived from, DESIGN.md
- * §6).  scores (double[ncand]), n_chunks / residual_nnz (int64[ncand]): host, nullable.
+ * opts, nm_pack_auto for F (Vp auto), score = nm_pack_auto's time model of that pack (ns,
+ * DESIGN.md §6).  scores (double[ncand]), n_chunks / residual_nnz (int64[ncand]): host, nullable.
  * *best = index of the lowest score (ties: the earlier candidate), perm_out (host int32[n]) its
  * permutation.  Synchronous.  Errors: as nm_reorder_gpu and nm_pack_hybrid. */
 NM_API nm_status nm_score_patterns(const nm_csr* A, int ncand, const int* V, const int* M, int F, nm_dtype dtype,
@@ -200,6 +199,18 @@ NM_API nm_status nm_pack_ex(const nm_csr* A, const int32_t* perm, int V, int N, 
 NM_API nm_status nm_pack_hybrid(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp,
                                 nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags,
                                 int tau, void* stream, nm_packed** out);
+
+/* nm_pack_auto -- nm_pack_hybrid at the tau that minimises the library's SpMM time model for F
+ * feature columns: the matrix is packed at tau in {0, 2, 4, t/2, t, 3t/2, 2t} (t =
+ * nm_hybrid_tau(F)) and each pack scored as n_chunks * (0.28 + 0.0075 F) + residual_nnz *
+ * 0.00016 F + residual_items * 0.0024 F (ns; per-chunk, per-value and per-work-item costs
+ * fitted to B200 measurements of the two kernels).  The per-item term is what
+ * keeps structured (banded) graphs, whose thin blocks scatter over many rows, at tau = 0.
+ * The best pack is returned in *out, its tau in *tau_out (nullable); ties keep the smaller
+ * tau.  Errors as nm_pack_hybrid.  Blocks until done. */
+NM_API nm_status nm_pack_auto(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp, nm_dtype dtype,
+                              int64_t row_begin, int64_t row_end, int flags, int F, void* stream,
+                              nm_packed** out, int* tau_out);
 
 /* nm_hybrid_tau -- the tau nm_pack_hybrid should use for an SpMM with F feature columns: the
  * break-even number of kept values at which a meta-block's share of a tensor-core chunk costs

@@ -65,6 +65,9 @@ SIGNATURES = {
                                          ctypes.POINTER(nm_reorder_opts), P32,
                                          ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.c_int),
                                          ctypes.POINTER(nm_reorder_stats)]),
+    "nm_pack_auto": (ctypes.c_int, [ctypes.POINTER(nm_csr), P32, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                    ctypes.c_int, ctypes.c_int64, ctypes.c_int64, ctypes.c_int, ctypes.c_int, VP,
+                                    ctypes.POINTER(VP), ctypes.POINTER(ctypes.c_int)]),
     "nm_score_patterns": (ctypes.c_int, [ctypes.POINTER(nm_csr), ctypes.c_int, ctypes.POINTER(ctypes.c_int),
                                          ctypes.POINTER(ctypes.c_int), ctypes.c_int, ctypes.c_int,
                                          ctypes.POINTER(nm_reorder_opts), ctypes.c_void_p,

@@ -187,12 +187,13 @@ class Packed:
 
 
 def pack(indptr, indices, perm, V: int, N: int, M: int, dtype="f16", val=None, val_dtype=None,
-         row_begin=None, row_end=None, stream=None, order="permuted", tau=0, Vp=0):
+         row_begin=None, row_end=None, stream=None, order="permuted", tau=0, Vp=0, F=None):
     """nm_pack / nm_pack_rows / nm_pack_ex / nm_pack_hybrid of B = P A P^T.  val: values per CSR
     entry (numpy, dtype val_dtype in {'f16','bf16' (uint16 bits),'f32'}) or None for a binary
     adjacency.  order='original' folds the permutation into the SpMM (NM_PACK_ORIGINAL_ORDER).
     tau > 0: hybrid split (meta-blocks keeping fewer than tau values go to the residual).
-    Vp: panel height, 64 or 128 (0 = the library's choice: 64 when V == 64, else 128)."""
+    Vp: panel height, 16, 32, 64 or 128 (0 = the library's choice: V for V in 16/32/64, else 128).
+    tau="auto": nm_pack_auto for F feature columns (the tau minimising the library's time model)."""
     if val is not None and val_dtype is None:
         val_dtype = "f32" if val.dtype == np.float32 else ("f16" if val.dtype == np.float16 else "bf16")
     c, keep = _csr_struct(indptr, indices, val, val_dtype or "f16")
@@ -204,6 +205,16 @@ def pack(indptr, indices, perm, V: int, N: int, M: int, dtype="f16", val=None, v
     re = c.n if row_end is None else int(row_end)
     flags = L.NM_PACK_ORIGINAL_ORDER if order == "original" else 0
     lib = L.load()
+    if tau == "auto":
+        if F is None:
+            raise ValueError("tau='auto' needs F")
+        t = ctypes.c_int()
+        L.check(lib.nm_pack_auto(ctypes.byref(c), pp, V, N, M, int(Vp), _DT[dtype], rb, re, flags, int(F), sp,
+                                 ctypes.byref(h), ctypes.byref(t)), "nm_pack_auto")
+        P = Packed(h, c.n, rb, re, dtype)
+        P.order = order
+        P.tau = int(t.value)
+        return P
     if tau:
         L.check(lib.nm_pack_hybrid(ctypes.byref(c), pp, V, N, M, int(Vp), _DT[dtype], rb, re, flags, int(tau), sp,
                                    ctypes.byref(h)), "nm_pack_hybrid")

@@ -972,8 +972,19 @@ nm_status pack_impl(const nm_csr* A, const int32_t* perm_host, int V, int N, int
   return NM_OK;
 }
 
-// Pattern scoring: reorder + hybrid pack per candidate, scored by the
-// library's own time model (the one nm_hybrid_tau is derived from).
+// The library's SpMM time model of a pack (fitted to B200 measurements of the two
+// kernels): per K = 32 chunk and F, per residual value and F, per residual work item (its Y
+// row read-modify-write and item overhead) and F.  ns of whole-GPU time.
+double pack_time_model(const nm_packed* P, int F) {
+  return (double)P->n_chunks * (0.28 + 0.0075 * F) + (double)P->res_nnz * (0.00016 * F) +
+         (double)P->n_res_segs * (0.0024 * F);
+}
+
+nm_status pack_auto_impl(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp, nm_dtype dtype,
+                         int64_t rb, int64_t re, int flags, int F, cudaStream_t s, nm_packed** out, int* tau_out);
+
+// Pattern scoring: reorder + the auto-tau hybrid pack per candidate,
+// scored by the library's time model.
 nm_status score_patterns_impl(const nm_csr* A, int ncand, const int* Vs, const int* Ms, int F, nm_dtype dtype,
                               const nm_reorder_opts* opts, cudaStream_t s, double* scores, int64_t* chunks_out,
                               int64_t* res_out, int* best, int32_t* perm_out) {
@@ -984,13 +995,11 @@ nm_status score_patterns_impl(const nm_csr* A, int ncand, const int* Vs, const i
   std::vector<int32_t> perm(n > 0 ? n : 1);
   double best_score = 0.0;
   int best_i = -1;
-  const int tau = nm_hybrid_tau(F);
   for (int i = 0; i < ncand; ++i) {
     NM_TRY(nm_reorder_gpu(A, Vs[i], 2, Ms[i], opts, perm.data(), nullptr, s));
     nm_packed* P = nullptr;
-    NM_TRY(pack_impl(A, perm.data(), Vs[i], 2, Ms[i], 0, dtype, 0, n, 0, tau, s, &P));
-    const double t_chunk = 0.28 + 0.0075 * F, t_value = 0.00016 * F;  // ns (nm_hybrid_tau's model)
-    const double sc = (double)P->n_chunks * t_chunk + (double)P->res_nnz * t_value;
+    NM_TRY(pack_auto_impl(A, perm.data(), Vs[i], 2, Ms[i], 0, dtype, 0, n, 0, F, s, &P, nullptr));
+    const double sc = pack_time_model(P, F);
     if (scores) scores[i] = sc;
     if (chunks_out) chunks_out[i] = P->n_chunks;
     if (res_out) res_out[i] = P->res_nnz;
@@ -1005,8 +1014,53 @@ nm_status score_patterns_impl(const nm_csr* A, int ncand, const int* Vs, const i
   return NM_OK;
 }
 
+// nm_pack_auto: the hybrid pack whose tau minimises the time model over a candidate set
+nm_status pack_auto_impl(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp, nm_dtype dtype,
+                         int64_t rb, int64_t re, int flags, int F, cudaStream_t s, nm_packed** out, int* tau_out) {
+  if (!out) return fail(NM_ERR_INVALID_ARG, "nm_pack_auto: NULL out");
+  if (F < 1) return fail(NM_ERR_INVALID_ARG, "nm_pack_auto: F < 1");
+  const int tm = nm_hybrid_tau(F);
+  const int cands[] = {0, 2, 4, tm / 2, tm, tm + tm / 2, 2 * tm};
+  nm_packed* best = nullptr;
+  double best_t = 0.0;
+  int best_tau = 0;
+  std::vector<int> seen;
+  for (int tau : cands) {
+    if (tau < 0 || std::find(seen.begin(), seen.end(), tau) != seen.end()) continue;
+    seen.push_back(tau);
+    nm_packed* P = nullptr;
+    nm_status st = pack_impl(A, perm, V, N, M, Vp, dtype, rb, re, flags, tau, s, &P);
+    if (st != NM_OK) {
+      nm_packed_free(best);
+      return st;
+    }
+    const double t = pack_time_model(P, F);
+    if (!best || t < best_t) {  // ties keep the smaller tau
+      nm_packed_free(best);
+      best = P;
+      best_t = t;
+      best_tau = tau;
+    } else {
+      nm_packed_free(P);
+    }
+  }
+  *out = best;
+  if (tau_out) *tau_out = best_tau;
+  return NM_OK;
+}
+
 }  // namespace
 }  // namespace nm
+
+extern "C" nm_status nm_pack_auto(const nm_csr* A, const int32_t* perm, int V, int N, int M, int Vp, nm_dtype dtype,
+                                  int64_t row_begin, int64_t row_end, int flags, int F, void* stream,
+                                  nm_packed** out, int* tau_out) {
+  if (flags & ~NM_PACK_ORIGINAL_ORDER) return nm::fail(NM_ERR_INVALID_ARG, "nm_pack_auto: unknown flags");
+  return nm::guarded("nm_pack_auto", [&] {
+    return nm::pack_auto_impl(A, perm, V, N, M, Vp, dtype, row_begin, row_end, flags, F, (cudaStream_t)stream, out,
+                              tau_out);
+  });
+}
 
 extern "C" nm_status nm_score_patterns(const nm_csr* A, int ncand, const int* V, const int* M, int F, nm_dtype dtype,
                                        const nm_reorder_opts* opts, void* stream, double* scores,

@@ -461,6 +461,9 @@ struct HostBackend : Backend {
   }
 };
 
+#ifndef NM_S2_DEVICE_TABLES
+#define NM_S2_DEVICE_TABLES 0
+#endif
 // Stage-1 sort (reorder_gpu.cu) and omega / MBscore (counts.cu) on the device
 struct DeviceBackend : Backend {
   const DevCsr& d;
@@ -473,8 +476,14 @@ struct DeviceBackend : Backend {
     if (dperm) cudaFree(dperm);
     s2dev_destroy(s2);
   }
+  // The device gain tables are bit-identical to the host's but measured SLOWER on B200 (C3
+  // 1:2:4, one Alg. 1 iteration: 87.7 s vs 28.7 s; banded n = 2^20: 3.27 s vs 0.71 s,
+  // profiles/r02_reorder_timing.jsonl): the per-batch scatter / gain / clear launches and the
+  // table read-back cost more than the host's OpenMP tables.  Compiled in with
+  // -DNM_S2_DEVICE_TABLES=1 for measurement; the default uses the host tables.
   S2DeviceTables* stage2_tables(int M, nm_status* st) override {
     *st = NM_OK;
+    if (!NM_S2_DEVICE_TABLES) return nullptr;
     if (s2 && s2_M != M) {
       s2dev_destroy(s2);
       s2 = nullptr;
