@@ -529,6 +529,11 @@ def main():
             if tr and tr.get("kernel", "").startswith(dom) and tr.get("tau", tau) == tau:
                 roofline["traffic"] = tr["dram_bytes_per_launch"]
                 roofline["traffic_source"] = "profiles/ncu_traffic.json (%s)" % tr.get("round", "")
+            if tr and tr.get("tau", tau) == tau and "k_spmm_sptc" in tr:  # tensor-pipe evidence (ncu)
+                ks = tr["k_spmm_sptc"]
+                kern["k_spmm_sptc"]["ncu"] = {"dram_bytes_per_launch": ks.get("dram_bytes_per_launch"),
+                                              "tensor_pipe": ks.get("tensor_pipe"),
+                                              "source": ks.get("source")}
         except Exception:
             pass
 
