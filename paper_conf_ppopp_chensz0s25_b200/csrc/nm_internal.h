@@ -187,8 +187,15 @@ nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, floa
                            int64_t ldy, int F, cudaStream_t s);
 nm_status launch_spmm_sptc(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy,
                            int F, cudaStream_t s, int format);
+// fused epilogue of the full-record kernel: out16[row * ldo + col] = 16-bit act(Y + bias)
+struct FusedAct {
+  void* out16;
+  int64_t ldo;
+  const float* bias;
+  int relu;
+};
 nm_status launch_spmm_sptc_full(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
-                                int64_t ldy, int F, cudaStream_t s);
+                                int64_t ldy, int F, cudaStream_t s, const FusedAct* fa = nullptr);
 nm_status launch_spmm_sptc_compressed(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,
                                       int64_t ldy, int F, cudaStream_t s);
 nm_status launch_spmm_sptc_tm(const nm_packed* P, const void* PX, int64_t ldx, float* Yp,

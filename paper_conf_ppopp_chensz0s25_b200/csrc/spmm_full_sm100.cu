@@ -61,7 +61,30 @@ struct FullParams {
   int64_t rows;
   int n_ftiles;
   uint32_t idesc;
+  // fused GCN epilogue (nm_gcn_layer on a pack without residual): H16 != nullptr stores
+  // act(Y + bias) as 16-bit values (bf16 if bf16_out) instead of Y (F even)
+  uint16_t* H16;
+  int64_t ldh;
+  const float* bias;
+  int relu, bf16_out;
 };
+
+__device__ __forceinline__ uint32_t pack_act16(float a, float b, const FullParams& p, int col) {
+  if (p.bias) {
+    a += __ldg(p.bias + col);
+    b += __ldg(p.bias + col + 1);
+  }
+  if (p.relu) {
+    a = fmaxf(a, 0.f);
+    b = fmaxf(b, 0.f);
+  }
+  uint32_t r;
+  if (p.bf16_out)
+    asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
+  else
+    asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
+  return r;  // a in the low half
+}
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -431,6 +454,20 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
 #pragma unroll
               for (int j = 0; j < 32; ++j) v[j] = 0u;
             }
+            if (p.H16) {  // fused bias + activation + 16-bit store (F even, 4-byte aligned pairs)
+#pragma unroll
+              for (int j = 0; j < 8; ++j) {
+                const int col = ft * BN + cc + 8 * j + cpair;
+                if (col >= p.F) continue;
+                if (olo >= 0)
+                  *(uint32_t*)(p.H16 + olo * p.ldh + col) =
+                      pack_act16(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]), p, col);
+                if (ohi >= 0)
+                  *(uint32_t*)(p.H16 + ohi * p.ldh + col) =
+                      pack_act16(__uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3]), p, col);
+              }
+              continue;
+            }
             if (full_tile) {
               float* ylo = p.Y + olo * p.ldy + ft * BN + cc + cpair;
               float* yhi = p.Y + ohi * p.ldy + ft * BN + cc + cpair;
@@ -495,7 +532,7 @@ uint32_t make_idesc_full(nm_dtype dt, int BN) {
 
 template <int BN>
 nm_status launch_full_bn(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
-                         cudaStream_t s) {
+                         cudaStream_t s, const FusedAct* fa) {
   using C = FCfg<BN>;
   static int configured_dev = -1;
   int dev = 0;
@@ -517,6 +554,11 @@ nm_status launch_full_bn(const nm_packed* P, const void* PX, int64_t ldx, float*
   prm.rows = P->row_end - P->row_begin;
   prm.n_ftiles = (F + BN - 1) / BN;
   prm.idesc = make_idesc_full(P->dtype, BN);
+  prm.H16 = fa ? (uint16_t*)fa->out16 : nullptr;
+  prm.ldh = fa ? fa->ldo : 0;
+  prm.bias = fa ? fa->bias : nullptr;
+  prm.relu = fa ? fa->relu : 0;
+  prm.bf16_out = P->dtype == NM_BF16;
   if (P->n_ctas < 1 || P->n_panels < 1) return NM_OK;
   k_spmm_full<BN><<<(unsigned)P->n_ctas, kFThreads, C::kSmem, s>>>(prm);
   NM_CUDA(cudaGetLastError());
@@ -526,11 +568,11 @@ nm_status launch_full_bn(const nm_packed* P, const void* PX, int64_t ldx, float*
 }  // namespace
 
 nm_status launch_spmm_sptc_full(const nm_packed* P, const void* PX, int64_t ldx, float* Yp, int64_t ldy, int F,
-                                cudaStream_t s) {
+                                cudaStream_t s, const FusedAct* fa) {
   if (!P->image_full) return fail(NM_ERR_UNSUPPORTED, "nm_spmm: the pack holds no full-record image");
-  if (F <= 64) return launch_full_bn<64>(P, PX, ldx, Yp, ldy, F, s);
-  if (F <= 128) return launch_full_bn<128>(P, PX, ldx, Yp, ldy, F, s);
-  return launch_full_bn<256>(P, PX, ldx, Yp, ldy, F, s);
+  if (F <= 64) return launch_full_bn<64>(P, PX, ldx, Yp, ldy, F, s, fa);
+  if (F <= 128) return launch_full_bn<128>(P, PX, ldx, Yp, ldy, F, s, fa);
+  return launch_full_bn<256>(P, PX, ldx, Yp, ldy, F, s, fa);
 }
 
 }  // namespace nm

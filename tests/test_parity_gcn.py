@@ -156,3 +156,52 @@ def test_gcn_layer_backward(n, fin, fout, V, M, relu):
     got_dh = np.empty_like(dh_p)
     got_dh[perm] = dh_p
     assert np.linalg.norm(got_dh - dH_ref) <= 1e-2 * np.linalg.norm(dH_ref)
+
+
+@pytest.mark.parametrize("fout,relu", [(64, True), (200, False), (128, True)])
+def test_gcn_layer_fused_epilogue_without_residual(fout, relu):
+    """A pack with an empty residual (banded graph, reordered to conform at 1:2:4, tau = 0):
+    nm_gcn_layer applies bias, activation and the bf16 down-convert in the tensor-core kernel's
+    epilogue.  The result equals the unfused path (nm_spmm to fp32 + the separate bias/act
+    kernel, here through nm_gcn_layer_bcast with one destination) bitwise, and the oracle within
+    the GCN bound."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    dev = torch.device("cuda:0")
+    n, fin = 2600, 96
+    ip, ic = graphs.banded_graph(n, 6, 11, self_loops=True)
+    vals = _gcn_norm(ip, ic)
+    vbits, v64 = graphs.round16(vals, "bf16")
+    perm, _ = api.reorder(ip, ic, 1, 2, 4)
+    P = api.pack(ip, ic, perm, 1, 2, 4, dtype="bf16", val=vals)
+    assert P.info()["residual_nnz"] == 0
+    rng = np.random.default_rng(4)
+    hb, _ = graphs.round16(rng.standard_normal((n, fin)).astype(np.float32), "bf16")
+    wb, _ = graphs.round16((rng.standard_normal((fin, fout)) / np.sqrt(fin)).astype(np.float32), "bf16")
+    b = rng.standard_normal(fout).astype(np.float32)
+    H = torch.from_numpy(hb.view(np.int16)).to(dev).view(torch.bfloat16)
+    W = torch.from_numpy(wb.view(np.int16)).to(dev).view(torch.bfloat16)
+    pd = torch.from_numpy(perm).to(dev)
+    PH = torch.empty_like(H)
+    api.permute_rows(H, PH, pd, "bf16")
+    ws = torch.empty(api.gcn_workspace_bytes(n, fin, fout), dtype=torch.uint8, device=dev)
+    bias = torch.from_numpy(b).to(dev)
+    fused = torch.empty((n, fout), dtype=torch.bfloat16, device=dev)
+    api.gcn_layer(P, PH, W, bias, fused, ws, relu=relu)
+    unfused = torch.empty((n, fout), dtype=torch.bfloat16, device=dev)
+    api.gcn_layer_bcast(P, PH, W, bias, [unfused.data_ptr()], 0, fout, ws, relu=relu)
+    torch.cuda.synchronize()
+    assert torch.equal(fused.view(torch.int16), unfused.view(torch.int16))
+    xw_bits = ws[: n * fout * 2].view(torch.int16).cpu().numpy().view(np.uint16).reshape(n, fout)
+    xw = np.empty((n, fout))
+    xw[perm] = graphs.bf16_bits_to_f64(xw_bits)
+    Y, E, _ = oracle.spmm(ip, ic, v64, xw)
+    ref = Y + b
+    if relu:
+        ref = np.maximum(ref, 0.0)
+    out = torch.empty_like(fused)
+    api.unpermute_rows(fused, out, pd, "bf16")
+    torch.cuda.synchronize()
+    got = graphs.bf16_bits_to_f64(out.view(torch.int16).cpu().numpy().view(np.uint16))
+    bound = 1e-3 * E + 2.0 ** -8 * np.abs(ref) + 1e-30
+    assert (np.abs(got - ref) <= bound).all(), np.abs(got - ref).max()
