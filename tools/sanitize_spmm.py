@@ -20,7 +20,7 @@ def run(ip, ic, V, M, F, dtype, tau):
     xb, _ = graphs.round16(graphs.features(n, F, 6), dtype)
     X = torch.from_numpy(xb.view(np.int16)).cuda().view(torch.float16 if dtype == "f16" else torch.bfloat16)
     Y = torch.empty((n, F), device="cuda")
-    for fmt in (1, 2):
+    for fmt in (1, 2, 3):
         api.spmm(P, X, Y, part="sptc", format=fmt)
     api.spmm(P, X, Y)
     torch.cuda.synchronize()
@@ -29,7 +29,27 @@ def run(ip, ic, V, M, F, dtype, tau):
                                                             st["residual_split_rows"], bool(torch.isfinite(Y).all())))
 
 
+def run_gcn_fused():
+    """nm_gcn_layer on a pack without residual (fused epilogue) and nm_gcn_layer_bcast."""
+    n, fin, fout = 2600, 96, 64
+    ip, ic = graphs.banded_graph(n, 6, 11, self_loops=True)
+    vals = graphs.gcn_norm_values(ip, ic)
+    perm, _ = api.reorder(ip, ic, 1, 2, 4)
+    P = api.pack(ip, ic, perm, 1, 2, 4, dtype="bf16", val=vals)
+    H = torch.randn((n, fin), device="cuda").to(torch.bfloat16)
+    W = (torch.randn((fin, fout), device="cuda") / 10).to(torch.bfloat16)
+    b = torch.randn(fout, device="cuda")
+    ws = torch.empty(api.gcn_workspace_bytes(n, fin, fout), dtype=torch.uint8, device="cuda")
+    out = torch.empty((n, fout), dtype=torch.bfloat16, device="cuda")
+    api.gcn_layer(P, H, W, b, out, ws, relu=True)
+    dsts = [torch.empty((n + 100, fout), dtype=torch.bfloat16, device="cuda") for _ in range(2)]
+    api.gcn_layer_bcast(P, H, W, b, [d.data_ptr() for d in dsts], 100, fout, ws, relu=True)
+    torch.cuda.synchronize()
+    print("gcn fused residual=%d equal=%s" % (P.info()["residual_nnz"], bool(torch.equal(out, dsts[0][100:]))))
+
+
 if __name__ == "__main__":
+    run_gcn_fused()
     ip, ic = graphs.er_graph(2048, 16384, 1)
     run(ip, ic, 1, 4, 32, "f16", 4)
     ip, ic = graphs.banded_graph(300 * 128 + 77, 12, 91)
