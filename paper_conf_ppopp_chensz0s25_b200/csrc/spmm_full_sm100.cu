@@ -11,13 +11,13 @@
 //   B (32 gathered rows of X x BN, SWIZZLE_128B MN-major)  <- cp.async 16-byte gathers
 //   E (metadata, 128 lanes x 32 b)        <- tcgen05.st of the record's lane words
 //   D (fp32, 128 x BN)                    in tensor memory (tcgen05.ld out)
-// Warp roles (persistent, one CTA per SM, 14 warps):
+// Warp roles (persistent, one CTA per SM, 22 warps):
 //   w0     record producer: waits for a free stage, one bulk copy per chunk, L2 prefetch of
 //          the next unit's first records
-//   w1-8   two gather groups of 4 warps (one per TMEM lane quarter); group g owns the stages
-//          s = g (mod 2): X gathers of the chunk's 32 rows + its metadata column
-//   w9     MMA issuer (+ TMEM allocation): warp-uniform loop, one elected lane issues
-//   w10-13 epilogue, one warp per TMEM lane quarter: tcgen05.ld 16x256b -> 8-byte stores
+//   w1-16  four gather groups of 4 warps (one per TMEM lane quarter); group g owns the stages
+//          s = g (mod 4): X gathers of the chunk's 32 rows + its metadata column
+//   w17    MMA issuer (+ TMEM allocation): warp-uniform loop, one elected lane issues
+//   w18-21 epilogue, one warp per TMEM lane quarter: tcgen05.ld 16x256b -> 8-byte stores
 // Work distribution: each CTA walks a CONTIGUOUS range of panels (pack time: balanced by chunk
 // count, nm_packed::cta_ptr), so the grid has no tail of idle SMs on skewed (power-law) graphs
 // and consecutive panels of one CTA share their X neighbourhoods in L2.
@@ -32,7 +32,7 @@ namespace nm {
 namespace {
 
 #ifndef NM_FULL_GROUPS
-#define NM_FULL_GROUPS 2
+#define NM_FULL_GROUPS 4
 #endif
 #ifndef NM_FULL_MAX_STAGES
 #define NM_FULL_MAX_STAGES 16
@@ -44,7 +44,7 @@ constexpr int kFGroups = NM_FULL_GROUPS;            // gather groups (4 warps ea
 #define NM_FULL_MMA_ONLY_ON 0
 #endif
 constexpr int kWProd = 0, kWG0 = 1, kWMma = kWG0 + 4 * kFGroups, kWEpi0 = kWMma + 1;
-constexpr int kFThreads = (kWEpi0 + 4) * 32;        // 14 warps
+constexpr int kFThreads = (kWEpi0 + 4) * 32;        // 22 warps (4 groups)
 constexpr int kGThreads = 128;                      // threads per gather group
 constexpr int kPfChunks = 24;                       // records L2-prefetched for the next unit
 
