@@ -372,23 +372,34 @@ def main():
         P_nat = api.pack(ip, ic, None, V, 2, M, dtype=dt, val=vals, row_begin=rb, row_end=re, order="original", tau=tau,
                          F=F)
         trial = {}
+        # (layout, tensor-core kernel) pairs: full records (format 1) or compressed records with
+        # A in TMEM (format 3) -- the faster depends on the graph
+        fmts = (args.sptc_format,) if args.sptc_format else (1, 3)
         for name, Pk in (("reordered", P), ("natural", P_nat)):
-            for _ in range(3):
-                api.spmm(Pk, X, Y)
-            ts = []
-            for _ in range(8):
-                flush.zero_()
-                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                a.record()
-                api.spmm(Pk, X, Y)
-                b.record()
-                ts.append((a, b))
-            torch.cuda.synchronize()
-            t = torch.tensor([statistics.median(x.elapsed_time(y) for x, y in ts)], dtype=torch.float64, device=cdev)
-            if world > 1:
-                dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            trial[name] = float(t.item())
-        layout_trial = dict(trial_ms=trial, chosen=min(trial, key=trial.get))
+            for fmt in fmts:
+                def run():
+                    api.spmm(Pk, X, Y, part="sptc", format=fmt)
+                    if Pk.info()["residual_nnz"]:
+                        api.spmm(Pk, X, Y, part="residual")
+                for _ in range(3):
+                    run()
+                ts = []
+                for _ in range(8):
+                    flush.zero_()
+                    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a.record()
+                    run()
+                    b.record()
+                    ts.append((a, b))
+                torch.cuda.synchronize()
+                t = torch.tensor([statistics.median(x.elapsed_time(y) for x, y in ts)], dtype=torch.float64,
+                                 device=cdev)
+                if world > 1:
+                    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                trial["%s/format%d" % (name, fmt)] = float(t.item())
+        best = min(trial, key=trial.get)
+        layout_trial = dict(trial_ms=trial, chosen=best.split("/")[0])
+        args.sptc_format = int(best.split("format")[1])
         if layout_trial["chosen"] == "natural":
             P, perm = P_nat, np.arange(n, dtype=np.int32)
         else:
@@ -540,7 +551,7 @@ def main():
     # ---------------- end-to-end through the public API with host buffers ----------------
     e2e = None
     if world == 1 and args.order == "original":
-        e2e = e2e_pipelined(P, X, Y, F, max(4, args.steps // 4), useful_flop)
+        e2e = e2e_pipelined(P, X, Y, F, max(4, args.steps // 4), useful_flop, fmt=args.sptc_format)
 
     # ---------------- cuSPARSE on the same box (original order, same rounded inputs) ----------
     cus = None
@@ -573,6 +584,7 @@ def main():
                 "config": {"workload": args.workload, "graph": w.get("graph", w["kind"]), "n": n, "nnz": nnz, "F": F,
                            "layout": (layout_trial or {}).get("chosen", args.layout),
                            "pattern": "%d:2:%d" % (V, M), "order": args.order, "tau": tau,
+                           "sptc_format": args.sptc_format or 1,
                            "parallelism": "row-shard x%d" % world,
                            "l2": "flushed between steps (256 MiB write outside the event-timed intervals)"},
                 "gpu_launches": launches_per_step * args.steps,
@@ -610,7 +622,7 @@ def padded_like(t):
     return base[:, :t.shape[1]]
 
 
-def e2e_pipelined(P, X, Y, F, steps, useful_flop):
+def e2e_pipelined(P, X, Y, F, steps, useful_flop, fmt=0):
     """End to end through the public API with host buffers: every step copies its X from
     pinned host memory, runs nm_spmm and reads Y back to pinned host memory.  Serving-style
     pipelining: device X/Y are double-buffered and H2D, SpMM and D2H run on three streams, so
@@ -643,7 +655,11 @@ def e2e_pipelined(P, X, Y, F, steps, useful_flop):
             s_cmp.wait_event(h2d_done[b])
             if d2h_done[b] is not None:
                 s_cmp.wait_event(d2h_done[b])          # step k-2's Y read back
-            api.spmm(P, Xd[b], Yd[b], stream=s_cmp)
+            if fmt:  # the tensor-core kernel the layout trial chose, then the residual (nm.h calls)
+                api.spmm(P, Xd[b], Yd[b], stream=s_cmp, part="sptc", format=fmt)
+                api.spmm(P, Xd[b], Yd[b], stream=s_cmp, part="residual")
+            else:
+                api.spmm(P, Xd[b], Yd[b], stream=s_cmp)
             cmp_done[b] = ev()
             cmp_done[b].record(s_cmp)
             s_d2h.wait_event(cmp_done[b])

@@ -11,20 +11,22 @@
 // lane words (two rows' nibbles per lane, nm_internal.h) come from two shuffles of the rows'
 // nibble words.  The MMA reads A from TMEM (tcgen05.mma.sp [d], [a], b-desc, [e]), so no
 // shared-memory expansion pass and no A tile in shared memory.
-// Warp roles (persistent, one CTA per SM, 14 warps):
+// Warp roles (persistent, one CTA per SM, 6 + 4 x NM_TM_GROUPS warps):
 //   w0     record producer: one bulk copy of the stage's (1-2 adjacent) compressed records
-//   w1-8   two gather groups of 4 warps (one per TMEM lane quarter): X gathers (cp.async, as the
+//   w1..   gather groups of 4 warps (one per TMEM lane quarter): X gathers (cp.async, as the
 //          full kernel) + A and metadata expansion into TMEM
-//   w9     MMA issuer (+ TMEM allocation)
-//   w10-13 epilogue (as the full kernel)
+//   then   the MMA issuer (+ TMEM allocation) and 4 epilogue warps (as the full kernel)
 #include "nm_internal.h"
 
 namespace nm {
 namespace {
 
-constexpr int kTGroups = 2;
+#ifndef NM_TM_GROUPS
+#define NM_TM_GROUPS 4
+#endif
+constexpr int kTGroups = NM_TM_GROUPS;  // gather + expansion groups (4 warps each)
 constexpr int kWProd = 0, kWG0 = 1, kWMma = kWG0 + 4 * kTGroups, kWEpi0 = kWMma + 1;
-constexpr int kTThreads = (kWEpi0 + 4) * 32;  // 14 warps
+constexpr int kTThreads = (kWEpi0 + 4) * 32;  // 22 warps at 4 groups
 constexpr int kGThreads = 128;
 constexpr int kPfBytes = 96 * 1024;           // records L2-prefetched ahead of the stream
 
