@@ -45,14 +45,19 @@ def test_bench_config_sampled_rows(workload):
     w = bench.parse_workload(workload)
     ip, ic, vals, X32 = bench.make_graph(w)
     perm, st = api.reorder(ip, ic, w["V"], 2, w["M"])
-    P = api.pack(ip, ic, perm, w["V"], 2, w["M"], dtype=w["dtype"], val=vals, order="original")
+    P = api.pack(ip, ic, perm, w["V"], 2, w["M"], dtype=w["dtype"], val=vals, order="original", tau="auto",
+                 F=w["F"])  # bench.py's pack (nm_pack_auto)
     assert P.info()["packed_nnz"] + P.info()["residual_nnz"] == ip[-1]
     xbits, x64 = graphs.round16(X32, w["dtype"])
     _, v64 = graphs.round16(vals, w["dtype"])
     X = torch.from_numpy(xbits.view(np.int16)).cuda().view(torch.float16)
     Y = torch.full((w["n"], w["F"]), float("nan"), device="cuda")
     api.spmm(P, X, Y)
+    Y3 = torch.full((w["n"], w["F"]), float("nan"), device="cuda")  # the A-in-TMEM kernel the bench may pick
+    api.spmm(P, X, Y3, part="sptc", format=3)
+    api.spmm(P, X, Y3, part="residual")
     torch.cuda.synchronize()
+    assert torch.equal(Y, Y3)
     Yh = Y.cpu().numpy()
     assert np.isfinite(Yh).all()
     rng = np.random.default_rng(7)

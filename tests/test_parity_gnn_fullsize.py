@@ -1,5 +1,6 @@
 """Full-size parity at the GNN-shaped configs of BASELINE.json (configs[2..4]) in the launch
-configuration bench.py times (fused original-order pack, hybrid split at the library's tau,
+configuration bench.py times (fused original-order pack, nm_pack_auto's hybrid split, both
+tensor-core kernels the bench's trial chooses from (bitwise equal),
 bench's reorder options), plus multi-unit parity of the wide-M patterns: sampled output rows
 (random + the heaviest rows + first/last) are recomputed one by one by the oracle in fp64 and
 must satisfy |Y - Y_ref| <= 1e-3 * (|A| |X|) (north star); every row of Y must be finite and
@@ -19,11 +20,12 @@ def _cuda():
     return torch.device("cuda:0")
 
 
-def _sampled_parity(ip, ic, vals, X32, perm, V, M, dtype, tau, order="original", nsample=3000, seed=7):
+def _sampled_parity(ip, ic, vals, X32, perm, V, M, dtype, tau, order="original", nsample=3000, seed=7,
+                    formats=False):
     from paper_conf_ppopp_chensz0s25_b200 import api, graphs
     dev = _cuda()
     n, F = X32.shape
-    P = api.pack(ip, ic, perm, V, 2, M, dtype=dtype, val=vals, order=order, tau=tau)
+    P = api.pack(ip, ic, perm, V, 2, M, dtype=dtype, val=vals, order=order, tau=tau, F=F)
     info = P.info()
     assert info["packed_nnz"] + info["residual_nnz"] == ip[-1]
     xbits, x64 = graphs.round16(X32, dtype)
@@ -37,6 +39,12 @@ def _sampled_parity(ip, ic, vals, X32, perm, V, M, dtype, tau, order="original",
         Y = torch.full((n, Fp), float("nan"), device=dev)[:, :F]
         api.spmm(P, X, Y)
         Yh = Y.cpu().numpy()
+        if formats:  # the other tensor-core kernel the bench may pick (A in TMEM): bitwise equal
+            Y3 = torch.full((n, Fp), float("nan"), device=dev)[:, :F]
+            api.spmm(P, X, Y3, part="sptc", format=3)
+            api.spmm(P, X, Y3, part="residual")
+            torch.cuda.synchronize()
+            assert torch.equal(Y, Y3)
     else:
         pd = torch.from_numpy(perm).to(dev)
         PXb = torch.zeros_like(Xb)
@@ -65,8 +73,8 @@ def test_gnn_config_bench_launch(workload):
     w = bench.parse_workload(workload)
     ip, ic, vals, X32 = bench.make_graph(w)
     perm, _ = api.reorder(ip, ic, w["V"], 2, w["M"], device=True, **bench.default_reorder_opts(w))
-    tau = w["tau"] if w["tau"] is not None else api.hybrid_tau(w["F"])
-    P = _sampled_parity(ip, ic, vals, X32, perm, w["V"], w["M"], w["dtype"], tau)
+    tau = w["tau"] if w["tau"] is not None else "auto"  # bench.py: nm_pack_auto
+    P = _sampled_parity(ip, ic, vals, X32, perm, w["V"], w["M"], w["dtype"], tau, formats=True)
     st = P.stats()
     assert st["n_chunks"] > 4 * 148  # many chunks per CTA: stage ring wrap-around, parity flips
 
