@@ -281,13 +281,15 @@ __global__ void __launch_bounds__(kTThreads, 1) k_spmm_tm(const TmParams p) {
                 const uint32_t mask = lds8(rec + kRecMaskOff + row);
                 const uint32_t tot = lds32(rec + kRecTotOff);
                 const uint32_t ne = tot & 0xFFFFu;
-                uint32_t cnt = __popc(mask), has = mask ? 1u : 0u;
-                uint32_t pv = cnt, pn_ = has;  // inclusive warp scans
+                const uint32_t cnt = __popc(mask), has = mask ? 1u : 0u;
+                // both inclusive warp scans in one register (counts <= 256 per quarter)
+                uint32_t sc = cnt | (has << 16);
 #pragma unroll
                 for (int o = 1; o < 32; o <<= 1) {
-                  const uint32_t a = __shfl_up_sync(0xffffffffu, pv, o), b = __shfl_up_sync(0xffffffffu, pn_, o);
-                  if (lane >= o) { pv += a; pn_ += b; }
+                  const uint32_t a = __shfl_up_sync(0xffffffffu, sc, o);
+                  if (lane >= o) sc += a;
                 }
+                const uint32_t pv = sc & 0xFFFFu, pn_ = sc >> 16;
                 const uint32_t qv = lds16(rec + kRecQvOff + 2 * quarter), qn = lds16(rec + kRecQnOff + 2 * quarter);
                 uint32_t e = qv + pv - cnt;
                 const uint32_t vbase = rec + kRecHdrBytes;
