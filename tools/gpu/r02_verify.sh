@@ -10,3 +10,5 @@ for wl in c2-banded-n1m-d16-f128-1:2:4; do
 import json; d=json.loads(open('gpurun_out/v_${fmt}_$wl.json').read().strip().splitlines()[-1]); print('fmt $fmt', d['ms_per_step'], {k:v['ms'] for k,v in d['roofline']['kernels'].items()})"
   done
 done
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_spmm_tm" -s 2 -c 1 -o gpurun_out/r02_c3_tm -f \
+  python bench.py --steps 2 --warmup 3 --no-cpu --no-cusparse --layout natural --no-reorder --sptc-format 3 > gpurun_out/ncu_tm.log 2>&1; echo ncu=$?
