@@ -62,6 +62,52 @@ constexpr int kRecMaxBytes = kRecHdrBytes + 4 * (kPanelRows + kPanelRows * kChun
 // workspace and the counters are allocated per nm_spmm call, stream-ordered (launch time),
 // never stored in the handle -- the packed matrix stays immutable, so concurrent calls on one
 // handle are safe.
+#ifdef __CUDACC__
+// The stage sequence of one CTA of the persistent tensor-core kernels: for each panel of its
+// range, for each F tile, the panel's chunks CPS at a time (panels without chunks have no
+// stages).  The gather groups own every G-th stage; advance(G) steps G stages.
+template <int CPS>
+struct StageIter {
+  int pn, pz, ft, nft, c, nch;
+  int64_t c0, c1;
+  const int64_t* pcp;
+  __device__ __forceinline__ void init(const int64_t* panel_chunk_ptr, int pa, int pz_, int nft_) {
+    pcp = panel_chunk_ptr;
+    pn = pa;
+    pz = pz_;
+    ft = 0;
+    nft = nft_;
+    c = 0;
+    nch = 0;
+    c0 = c1 = pa < pz_ ? __ldg(pcp + pa) : 0;
+    load_panel();
+  }
+  __device__ __forceinline__ bool valid() const { return pn < pz; }
+  __device__ __forceinline__ void load_panel() {
+    while (pn < pz) {
+      c1 = __ldg(pcp + pn + 1);
+      nch = (int)(c1 - c0);
+      if (nch > 0) return;
+      ++pn;
+      c0 = c1;
+    }
+  }
+  __device__ __forceinline__ void next() {
+    c += CPS;
+    if (c < nch) return;
+    c = 0;
+    if (++ft < nft) return;
+    ft = 0;
+    ++pn;
+    c0 = c1;
+    load_panel();
+  }
+  __device__ __forceinline__ void advance(int g) {
+    for (int k = 0; k < g && pn < pz; ++k) next();
+  }
+};
+#endif
+
 constexpr int kResSeg = 256;   // max residual nonzeros per work item
 constexpr int kResSlab = 256;  // features per residual launch (partial-sum slot width)
 struct ResSeg {

@@ -271,79 +271,71 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
     const uint32_t mword = 4u * (uint32_t)(quarter * 32 + lane);  // this lane's metadata word
     uint64_t pol_x;  // gathered X rows stay in L2 (reused by the other panels' meta-blocks)
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_x));
-    int64_t i = 0;  // CTA stage counter
-    int s = 0;
-    uint32_t ph = 0;
-    int64_t c0 = pa < pz ? __ldg(p.panel_chunk_ptr + pa) : 0;
-    for (int pn = pa; pn < pz; ++pn) {
-      const int64_t c1 = __ldg(p.panel_chunk_ptr + pn + 1);
-      const int nch = (int)(c1 - c0);
-      c0 = c1;
-      for (int ft = 0; ft < nft; ++ft) {
-        const int col0 = ft * BN + c16 * 8;
-        const uint32_t colbytes = col0 >= p.F ? 0u : (p.F - col0 >= 8 ? 16u : (uint32_t)(p.F - col0) * 2u);
-        const uint16_t* xcol = p.X + (colbytes ? col0 : 0);
-        for (int c = 0; c < nch; c += CPS, ++i) {
-          if ((int)(i % kFGroups) == group) {  // kFGroups divides kStages: group g owns s = g (mod kFGroups)
-            const int sub = min(CPS, nch - c);
-            mbar_wait(bRec + 8 * s, ph);  // records landed (gather rows, metadata, A)
-            const uint32_t rec0 = sRec + s * CPS * C::kRecBytes;
-            uint32_t mw[CPS];
+    // this group's stages only: i = group, group + kFGroups, ... (stage s = i mod kStages)
+    StageIter<CPS> it;
+    it.init(p.panel_chunk_ptr, pa, pz, nft);
+    it.advance(group);
+    for (int i = group; it.valid(); i += kFGroups, it.advance(kFGroups)) {
+      const int s = i % C::kStages;
+      const uint32_t ph = (uint32_t)((i / C::kStages) & 1);
+      const int col0 = it.ft * BN + c16 * 8;
+      const uint32_t colbytes = col0 >= p.F ? 0u : (p.F - col0 >= 8 ? 16u : (uint32_t)(p.F - col0) * 2u);
+      const uint16_t* xcol = p.X + (colbytes ? col0 : 0);
+      const int sub = min(CPS, it.nch - it.c);
+      mbar_wait(bRec + 8 * s, ph);  // records landed (gather rows, metadata, A)
+      const uint32_t rec0 = sRec + s * CPS * C::kRecBytes;
+      uint32_t mw[CPS];
 #pragma unroll
-            for (int j = 0; j < CPS; ++j) {
-              if (j < sub) {
-                const uint32_t rec = rec0 + j * C::kRecBytes;
-                const uint32_t sbase = sB + (s * CPS + j) * C::kBBytes + dcol;
+      for (int j = 0; j < CPS; ++j) {
+        if (j < sub) {
+          const uint32_t rec = rec0 + j * C::kRecBytes;
+          const uint32_t sbase = sB + (s * CPS + j) * C::kBBytes + dcol;
 #ifdef NM_FULL_MMA_ONLY  // timing experiment (results invalid): no gathers
-                if (false) {
+          if (false) {
 #else
-                if (colbytes == 16u) {
+          if (colbytes == 16u) {
 #endif
 #pragma unroll
-                  for (int q = 0; q < kPer; ++q) {
-                    const int kk = q * kRowsPerPass + kk0;
-                    const int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * kk);
-                    asm volatile(
-                        "{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %2, 0;\n\t"
-                        "cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, q, %3;\n\t}" ::"r"(
-                            sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
-                        "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(xr), "l"(pol_x)
-                        : "memory");
-                  }
-                } else if (!NM_FULL_MMA_ONLY_ON) {  // the F tail: partial or empty pieces
-#pragma unroll
-                  for (int q = 0; q < kPer; ++q) {
-                    const int kk = q * kRowsPerPass + kk0;
-                    const int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * kk);
-                    const uint32_t nb = xr >= 0 ? colbytes : 0u;
-                    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(
-                                     sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
-                                 "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(nb), "l"(pol_x)
-                                 : "memory");
-                  }
-                }
-                mw[j] = lds32(rec + kChunkValBytes + mword);
-              } else {
-                mw[j] = 0x44444444u;  // unused column (legal no-value nibbles)
-              }
+            for (int q = 0; q < kPer; ++q) {
+              const int kk = q * kRowsPerPass + kk0;
+              const int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * kk);
+              asm volatile(
+                  "{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %2, 0;\n\t"
+                  "cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, q, %3;\n\t}" ::"r"(
+                      sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
+                  "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(xr), "l"(pol_x)
+                  : "memory");
             }
-            asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bFull + 8 * s) : "memory");
-            // metadata: this lane's words of the stage's records into its TMEM columns
-            const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + CPS * s;
-            if constexpr (CPS == 2)
-              asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1, %2};" ::"r"(taddr), "r"(mw[0]),
-                           "r"(mw[CPS - 1])
+          } else if (!NM_FULL_MMA_ONLY_ON) {  // the F tail: partial or empty pieces
+#pragma unroll
+            for (int q = 0; q < kPer; ++q) {
+              const int kk = q * kRowsPerPass + kk0;
+              const int32_t xr = (int32_t)lds32(rec + kChunkXrowOff + 4 * kk);
+              const uint32_t nb = xr >= 0 ? colbytes : 0u;
+              asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(
+                               sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
+                           "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(nb), "l"(pol_x)
                            : "memory");
-            else
-              asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(mw[0]) : "memory");
-            asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-            asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-            __syncwarp();
-            if (lane == 0) mbar_arrive(bFull + 8 * s);
+            }
           }
-          if (++s == C::kStages) { s = 0; ph ^= 1; }
+          mw[j] = lds32(rec + kChunkValBytes + mword);
+        } else {
+          mw[j] = 0x44444444u;  // unused column (legal no-value nibbles)
         }
       }
+      asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bFull + 8 * s) : "memory");
+      // metadata: this lane's words of the stage's records into its TMEM columns
+      const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + CPS * s;
+      if constexpr (CPS == 2)
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1, %2};" ::"r"(taddr), "r"(mw[0]),
+                     "r"(mw[CPS - 1])
+                     : "memory");
+      else
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(mw[0]) : "memory");
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(bFull + 8 * s);
     }
   } else if (warp == kWMma) {
     // ------------------------------------------------------------ MMA issuer

@@ -243,92 +243,84 @@ __global__ void __launch_bounds__(kTThreads, 1) k_spmm_tm(const TmParams p) {
     const int src_a = (lane & 7) + 16 * (lane >> 4), src_b = src_a + 8, k1 = (lane >> 3) & 1;
     uint64_t pol_x;
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_x));
-    int64_t i = 0;
-    int s = 0;
-    uint32_t ph = 0;
-    int64_t c0 = pa < pz ? __ldg(p.panel_chunk_ptr + pa) : 0;
-    for (int pn = pa; pn < pz; ++pn) {
-      const int64_t c1 = __ldg(p.panel_chunk_ptr + pn + 1);
-      const int nch = (int)(c1 - c0);
-      c0 = c1;
-      for (int ft = 0; ft < nft; ++ft) {
-        const int col0 = ft * BN + c16 * 8;
-        const uint32_t colbytes = col0 >= p.F ? 0u : (p.F - col0 >= 8 ? 16u : (uint32_t)(p.F - col0) * 2u);
-        const uint16_t* xcol = p.X + (colbytes ? col0 : 0);
-        for (int c = 0; c < nch; c += CPS, ++i) {
-          if ((int)(i % kTGroups) == group) {
-            const int sub = min(CPS, nch - c);
-            mbar_wait(bRec + 8 * s, ph);
-            uint32_t rec = sRec + s * kSlot;
-            uint32_t mw[CPS];
+    // this group's stages only: i = group, group + kTGroups, ... (stage s = i mod kStages)
+    StageIter<CPS> it;
+    it.init(p.panel_chunk_ptr, pa, pz, nft);
+    it.advance(group);
+    for (int i = group; it.valid(); i += kTGroups, it.advance(kTGroups)) {
+      const int s = i % C::kStages;
+      const uint32_t ph = (uint32_t)((i / C::kStages) & 1);
+      const int col0 = it.ft * BN + c16 * 8;
+      const uint32_t colbytes = col0 >= p.F ? 0u : (p.F - col0 >= 8 ? 16u : (uint32_t)(p.F - col0) * 2u);
+      const uint16_t* xcol = p.X + (colbytes ? col0 : 0);
+      const int sub = min(CPS, it.nch - it.c);
+      mbar_wait(bRec + 8 * s, ph);
+      uint32_t rec = sRec + s * kSlot;
+      uint32_t mw[CPS];
 #pragma unroll
-            for (int j = 0; j < CPS; ++j) {
-              uint32_t w[8];
-              if (j < sub) {
-                // X gathers of the chunk's 32 rows (gather row list at the record's start)
-                const uint32_t sbase = sB + (s * CPS + j) * C::kBBytes + dcol;
+      for (int j = 0; j < CPS; ++j) {
+        uint32_t w[8];
+        if (j < sub) {
+          // X gathers of the chunk's 32 rows (gather row list at the record's start)
+          const uint32_t sbase = sB + (s * CPS + j) * C::kBBytes + dcol;
 #pragma unroll
-                for (int q = 0; q < kPer; ++q) {
-                  const int kk = q * kRowsPerPass + kk0;
-                  const int32_t xr = (int32_t)lds32(rec + 4 * kk);
-                  const uint32_t nb = xr >= 0 ? colbytes : 0u;
-                  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(
-                                   sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
-                               "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(nb), "l"(pol_x)
-                               : "memory");
-                }
-                // A row and nibble word of this thread's row
-                const uint32_t mask = lds8(rec + kRecMaskOff + row);
-                const uint32_t tot = lds32(rec + kRecTotOff);
-                const uint32_t ne = tot & 0xFFFFu;
-                const uint32_t cnt = __popc(mask), has = mask ? 1u : 0u;
-                // both inclusive warp scans in one register (counts <= 256 per quarter)
-                uint32_t sc = cnt | (has << 16);
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                  const uint32_t a = __shfl_up_sync(0xffffffffu, sc, o);
-                  if (lane >= o) sc += a;
-                }
-                const uint32_t pv = sc & 0xFFFFu, pn_ = sc >> 16;
-                const uint32_t qv = lds16(rec + kRecQvOff + 2 * quarter), qn = lds16(rec + kRecQnOff + 2 * quarter);
-                uint32_t e = qv + pv - cnt;
-                const uint32_t vbase = rec + kRecHdrBytes;
-#pragma unroll
-                for (int g = 0; g < 8; ++g) {
-                  w[g] = 0u;
-                  if (mask & (1u << g)) w[g] = lds32(vbase + 4 * e++);
-                }
-                const uint32_t W = has ? lds32(vbase + 4 * (ne + qn + pn_ - 1)) : kMetaNone;
-                const uint32_t Wa = __shfl_sync(0xffffffffu, W, src_a), Wb = __shfl_sync(0xffffffffu, W, src_b);
-                mw[j] = ((Wa >> (16 * k1)) & 0xFFFFu) | (((Wb >> (16 * k1)) & 0xFFFFu) << 16);
-                rec += 16u * (uint32_t)((kRecHdrBytes + 4 * (ne + (tot >> 16)) + 15) / 16);
-              } else {
-#pragma unroll
-                for (int g = 0; g < 8; ++g) w[g] = 0u;
-                mw[j] = kMetaNone;
-              }
-              const uint32_t ta = tbase + ((uint32_t)(quarter * 32) << 16) + C::kA0 + 8 * (CPS * s + j);
-              asm volatile(
-                  "tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"r"(ta), "r"(w[0]),
-                  "r"(w[1]), "r"(w[2]), "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7])
-                  : "memory");
-            }
-            asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bFull + 8 * s) : "memory");
-            const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + CPS * s;
-            if constexpr (CPS == 2)
-              asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1, %2};" ::"r"(taddr), "r"(mw[0]),
-                           "r"(mw[CPS - 1])
-                           : "memory");
-            else
-              asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(mw[0]) : "memory");
-            asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-            asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-            __syncwarp();
-            if (lane == 0) mbar_arrive(bFull + 8 * s);
+          for (int q = 0; q < kPer; ++q) {
+            const int kk = q * kRowsPerPass + kk0;
+            const int32_t xr = (int32_t)lds32(rec + 4 * kk);
+            const uint32_t nb = xr >= 0 ? colbytes : 0u;
+            asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(
+                             sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
+                         "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(nb), "l"(pol_x)
+                         : "memory");
           }
-          if (++s == C::kStages) { s = 0; ph ^= 1; }
+          // A row and nibble word of this thread's row
+          const uint32_t mask = lds8(rec + kRecMaskOff + row);
+          const uint32_t tot = lds32(rec + kRecTotOff);
+          const uint32_t ne = tot & 0xFFFFu;
+          const uint32_t cnt = __popc(mask), has = mask ? 1u : 0u;
+          // both inclusive warp scans in one register (counts <= 256 per quarter)
+          uint32_t sc = cnt | (has << 16);
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t a = __shfl_up_sync(0xffffffffu, sc, o);
+            if (lane >= o) sc += a;
+          }
+          const uint32_t pv = sc & 0xFFFFu, pn_ = sc >> 16;
+          const uint32_t qv = lds16(rec + kRecQvOff + 2 * quarter), qn = lds16(rec + kRecQnOff + 2 * quarter);
+          uint32_t e = qv + pv - cnt;
+          const uint32_t vbase = rec + kRecHdrBytes;
+#pragma unroll
+          for (int g = 0; g < 8; ++g) {
+            w[g] = 0u;
+            if (mask & (1u << g)) w[g] = lds32(vbase + 4 * e++);
+          }
+          const uint32_t W = has ? lds32(vbase + 4 * (ne + qn + pn_ - 1)) : kMetaNone;
+          const uint32_t Wa = __shfl_sync(0xffffffffu, W, src_a), Wb = __shfl_sync(0xffffffffu, W, src_b);
+          mw[j] = ((Wa >> (16 * k1)) & 0xFFFFu) | (((Wb >> (16 * k1)) & 0xFFFFu) << 16);
+          rec += 16u * (uint32_t)((kRecHdrBytes + 4 * (ne + (tot >> 16)) + 15) / 16);
+        } else {
+#pragma unroll
+          for (int g = 0; g < 8; ++g) w[g] = 0u;
+          mw[j] = kMetaNone;
         }
+        const uint32_t ta = tbase + ((uint32_t)(quarter * 32) << 16) + C::kA0 + 8 * (CPS * s + j);
+        asm volatile(
+            "tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"r"(ta), "r"(w[0]),
+            "r"(w[1]), "r"(w[2]), "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7])
+            : "memory");
       }
+      asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bFull + 8 * s) : "memory");
+      const uint32_t taddr = tbase + ((uint32_t)(quarter * 32) << 16) + C::kMeta0 + CPS * s;
+      if constexpr (CPS == 2)
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1, %2};" ::"r"(taddr), "r"(mw[0]),
+                     "r"(mw[CPS - 1])
+                     : "memory");
+      else
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(mw[0]) : "memory");
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(bFull + 8 * s);
     }
   } else if (warp == kWMma) {
     // ------------------------------------------------------------ MMA issuer (A from TMEM)
