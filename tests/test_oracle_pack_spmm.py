@@ -56,7 +56,7 @@ def _pack_cases():
 
 
 @pytest.mark.parametrize("ci", range(4))
-@pytest.mark.parametrize("Vp,Mp", [(64, 4), (128, 4), (64, 8), (128, 16), (128, 8)])
+@pytest.mark.parametrize("Vp,Mp", [(64, 4), (128, 4), (64, 8), (128, 16), (128, 8), (16, 8), (32, 4)])
 def test_unpack_plus_residual_is_B_bitwise(ci, Vp, Mp):
     indptr, indices = _pack_cases()[ci]
     n = len(indptr) - 1
