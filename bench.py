@@ -310,6 +310,12 @@ def main():
     if args.impl == "reference":
         return run_reference(args, w)
 
+    if int(os.environ.get("WORLD_SIZE", "1")) > 1 and os.environ.get("OMP_NUM_THREADS", "1") == "1":
+        # the ranks of one node share the host cores for the (untimed) reorder's OpenMP Stage-2
+        # and the packer's host steps: split them (torchrun's default of 1 thread per rank would
+        # make the C3 reorder ~16x slower) -- set before torch, libnm and the oracle load their
+        # OpenMP runtimes
+        os.environ["OMP_NUM_THREADS"] = str(max(1, len(os.sched_getaffinity(0)) // int(os.environ["WORLD_SIZE"])))
     import torch
     import torch.distributed as dist
     from paper_conf_ppopp_chensz0s25_b200 import api, graphs
