@@ -46,7 +46,15 @@ __device__ __forceinline__ float fma16(unsigned short a, unsigned short b, float
 #ifndef NM_RES_CPASYNC
 #define NM_RES_CPASYNC 1  // X rows via cp.async into a per-subgroup shared-memory ring (0: registers)
 #endif
-constexpr int kResBatch = 8;  // entries per cp.async batch (two batches in flight per subgroup)
+#ifndef NM_RES_BATCH
+#define NM_RES_BATCH 8
+#endif
+#ifdef NM_RES_MINB  // tuning experiments: minimum resident CTAs per SM for k_residual
+#define NM_RES_BOUNDS __launch_bounds__(256, NM_RES_MINB)
+#else
+#define NM_RES_BOUNDS __launch_bounds__(256)
+#endif
+constexpr int kResBatch = NM_RES_BATCH;  // entries per cp.async batch (two batches in flight per subgroup)
 
 template <int LPR>
 constexpr int res_smem_bytes() {
@@ -58,7 +66,7 @@ __device__ __forceinline__ void cp_async16_z(uint32_t dst, const void* src, uint
 }
 
 template <int BF, int LPR>
-__global__ void __launch_bounds__(256) k_residual(const ResSeg* __restrict__ segs, int64_t n_segs,
+__global__ void NM_RES_BOUNDS k_residual(const ResSeg* __restrict__ segs, int64_t n_segs,
                                                   const int32_t* __restrict__ rc, const uint16_t* __restrict__ rv,
                                                   const uint16_t* __restrict__ X, int64_t ldx,
                                                   float* __restrict__ Y, int64_t ldy, int F, int f_base,
