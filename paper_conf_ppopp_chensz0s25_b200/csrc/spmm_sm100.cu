@@ -10,18 +10,22 @@
 //   D (fp32, 128 x BN)                              in tensor memory (tcgen05.ld out)
 // The record is the paper's matrix put "into the SPTC required form on the fly" (L492): HBM
 // holds only the non-empty (row, meta-block) slots; the dense operand exists only in SMEM.
-// Warp roles (persistent, one CTA per SM, 22 warps):
-//   w0 record TMA (own ring of kRecSlots) + L2 prefetch of the next units' records
-//   w1-12 loaders, three groups of 4 warps, group g owns the stages s = g (mod 3): X gathers,
-//         record expansion into the A tile, metadata into TMEM
-//   w13 MMA issuer (+ TMEM allocation)
-//   w14-21 epilogue, two warps per TMEM lane quarter: tcgen05.ld 16x256b -> 32-byte
-//   sector-aligned stores of Y rows (no shared-memory staging).
+// Warp roles (persistent, one CTA per SM, 23 warps with the defaults NM_LOAD_GROUPS = 4,
+// NM_EPI_WARPS = 4, NM_PRODUCERS = 2):
+//   w0      record producer 0 (bulk copies into its half of the byte ring) + L2 prefetch of
+//           the next units' records
+//   w1-16   loaders, four groups of 4 warps, group g owns the stages s = g (mod 4): X gathers,
+//           record expansion into the A tile, metadata into TMEM
+//   w17     MMA issuer (+ TMEM allocation)
+//   w18-21  epilogue, one warp per TMEM lane quarter: tcgen05.ld 16x256b -> sector-aligned
+//           stores of Y rows (no shared-memory staging)
+//   w22     record producer 1 (alternate units, the other ring half)
 // All hand-offs are mbarriers; the pipeline runs across work units, so consecutive panels
 // overlap, and every role prefetches the next unit's schedule entry.  Design evidence
 // (DESIGN.md §6): TMA tile::gather4 costs ~57 cycles per instruction on B200, so X rows are
 // gathered with cp.async; one loader group spent ~950 cycles per chunk (clock64 timeline,
-// tools/trace_spmm.py), so three groups share the stages.
+// tools/trace_spmm.py), so several groups share the stages.  (nm_spmm_sptc_format 2; the
+// default tensor-core kernel is spmm_full_sm100.cu.)
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_bf16.h>
