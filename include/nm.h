@@ -200,14 +200,6 @@ NM_API nm_status nm_pack_hybrid(const nm_csr* A, const int32_t* perm, int V, int
                                 nm_dtype dtype, int64_t row_begin, int64_t row_end, int flags,
                                 int tau, void* stream, nm_packed** out);
 
-/* nm_l2_persist -- keep the gathered operand resident in L2 across SpMM calls on `stream`: sets
- * the device's persisting-L2 carve-out to min(bytes, the device maximum) and the stream's
- * access-policy window to [ptr, ptr + bytes) (persisting hits, streaming misses), so the chunk
- * records and the residual's (col, val) stream, both read once, do not evict X.  ptr = NULL or
- * bytes = 0 resets the window and the persisting lines.  Affects the stream (and the device's
- * L2 carve-out) until reset.  Errors: UNSUPPORTED without persisting L2, CUDA. */
-NM_API nm_status nm_l2_persist(const void* ptr, size_t bytes, void* stream);
-
 /* nm_pack_auto -- nm_pack_hybrid at the tau that minimises the library's SpMM time model for F
  * feature columns: the matrix is packed at tau in {0, 2, 4, t/2, t, 3t/2, 2t} (t =
  * nm_hybrid_tau(F)) and each pack scored as n_chunks * (0.28 + 0.0075 F) + residual_nnz *

@@ -65,7 +65,6 @@ SIGNATURES = {
                                          ctypes.POINTER(nm_reorder_opts), P32,
                                          ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.c_int),
                                          ctypes.POINTER(nm_reorder_stats)]),
-    "nm_l2_persist": (ctypes.c_int, [VP, ctypes.c_size_t, VP]),
     "nm_pack_auto": (ctypes.c_int, [ctypes.POINTER(nm_csr), P32, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                     ctypes.c_int, ctypes.c_int64, ctypes.c_int64, ctypes.c_int, ctypes.c_int, VP,
                                     ctypes.POINTER(VP), ctypes.POINTER(ctypes.c_int)]),

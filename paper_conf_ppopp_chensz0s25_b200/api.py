@@ -232,16 +232,6 @@ def pack(indptr, indices, perm, V: int, N: int, M: int, dtype="f16", val=None, v
     return P
 
 
-def l2_persist(t=None, stream=None):
-    """nm_l2_persist: keep tensor t (e.g. the SpMM's X) resident in L2 for work on `stream`;
-    t=None resets."""
-    if t is None:
-        L.check(L.load().nm_l2_persist(None, 0, _stream_ptr(stream)), "nm_l2_persist")
-    else:
-        L.check(L.load().nm_l2_persist(_ptr(t), t.untyped_storage().nbytes() - t.storage_offset() * t.element_size(),
-                                       _stream_ptr(stream)), "nm_l2_persist")
-
-
 def hybrid_tau(F: int) -> int:
     """nm_hybrid_tau: the library's break-even hybrid-split threshold for F feature columns."""
     return int(L.load().nm_hybrid_tau(int(F)))

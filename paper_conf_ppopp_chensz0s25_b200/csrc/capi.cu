@@ -199,36 +199,6 @@ const char* nm_last_error(void) { return g_last_error.c_str(); }
 
 int nm_version(void) { return 1; }
 
-nm_status nm_l2_persist(const void* ptr, size_t bytes, void* stream) {
-  cudaStream_t s = (cudaStream_t)stream;
-  cudaStreamAttrValue v = {};
-  if (!ptr || bytes == 0) {  // reset: no window, persisting lines back to normal
-    v.accessPolicyWindow.base_ptr = nullptr;
-    v.accessPolicyWindow.num_bytes = 0;
-    v.accessPolicyWindow.hitRatio = 0.f;
-    v.accessPolicyWindow.hitProp = cudaAccessPropertyNormal;
-    v.accessPolicyWindow.missProp = cudaAccessPropertyNormal;
-    NM_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v));
-    NM_CUDA(cudaCtxResetPersistingL2Cache());
-    return NM_OK;
-  }
-  int dev = 0, max_persist = 0, max_window = 0;
-  NM_CUDA(cudaGetDevice(&dev));
-  NM_CUDA(cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, dev));
-  NM_CUDA(cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, dev));
-  if (max_persist <= 0 || max_window <= 0) return fail(NM_ERR_UNSUPPORTED, "nm_l2_persist: no persisting L2 on this device");
-  const size_t carve = std::min(bytes, (size_t)max_persist);
-  NM_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, carve));
-  const size_t win = std::min(bytes, (size_t)max_window);
-  v.accessPolicyWindow.base_ptr = const_cast<void*>(ptr);
-  v.accessPolicyWindow.num_bytes = win;
-  v.accessPolicyWindow.hitRatio = std::min(1.f, (float)carve / (float)win);
-  v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-  v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-  NM_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v));
-  return NM_OK;
-}
-
 // Hybrid-split threshold from a measured time model (reading #27): a meta-block
 // emitted to the tensor-core path costs an eighth of a K = 32 chunk, a residual value one
 // gathered X row.  Fitted on B200 (round 2, full-record kernel + cp.async residual, whole-GPU
