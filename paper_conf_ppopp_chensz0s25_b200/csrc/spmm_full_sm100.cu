@@ -267,7 +267,7 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
     constexpr int kRowsPerPass = kGThreads / kRowPieces;
     const int c16 = t % kRowPieces, kk0 = t / kRowPieces;
     const uint32_t dcol = (uint32_t)(c16 >> 3) * 4096u;  // 64-column slab of the SW128 tile
-    const int32_t ldx32 = (int32_t)p.ldx;
+    const uint32_t ldxb = (uint32_t)p.ldx * 2u;  // row pitch in bytes
     const uint32_t mword = 4u * (uint32_t)(quarter * 32 + lane);  // this lane's metadata word
     uint64_t pol_x;  // gathered X rows stay in L2 (reused by the other panels' meta-blocks)
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_x));
@@ -303,7 +303,7 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
                   "{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %2, 0;\n\t"
                   "cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, q, %3;\n\t}" ::"r"(
                       sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
-                  "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(xr), "l"(pol_x)
+                  "l"((uint64_t)(uint32_t)max(xr, 0) * ldxb + (uint64_t)(uintptr_t)xcol), "r"(xr), "l"(pol_x)
                   : "memory");
             }
           } else if (!NM_FULL_MMA_ONLY_ON) {  // the F tail: partial or empty pieces
@@ -314,7 +314,7 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
               const uint32_t nb = xr >= 0 ? colbytes : 0u;
               asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(
                                sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
-                           "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(nb), "l"(pol_x)
+                           "l"((uint64_t)(uint32_t)max(xr, 0) * ldxb + (uint64_t)(uintptr_t)xcol), "r"(nb), "l"(pol_x)
                            : "memory");
             }
           }

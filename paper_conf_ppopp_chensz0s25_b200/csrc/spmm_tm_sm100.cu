@@ -236,7 +236,7 @@ __global__ void __launch_bounds__(kTThreads, 1) k_spmm_tm(const TmParams p) {
     constexpr int kRowsPerPass = kGThreads / kRowPieces;
     const int c16 = t % kRowPieces, kk0 = t / kRowPieces;
     const uint32_t dcol = (uint32_t)(c16 >> 3) * 4096u;
-    const int32_t ldx32 = (int32_t)p.ldx;
+    const uint32_t ldxb = (uint32_t)p.ldx * 2u;  // row pitch in bytes
     const int row = quarter * 32 + lane;   // the A row (TMEM lane) this thread expands
     // metadata lane word of this lane: rows ra = (lane % 8) + 16 (lane / 16) and ra + 8 of the
     // quarter, K-half k1 = (lane / 8) % 2 (nm_internal.h meta layout)
@@ -267,11 +267,20 @@ __global__ void __launch_bounds__(kTThreads, 1) k_spmm_tm(const TmParams p) {
           for (int q = 0; q < kPer; ++q) {
             const int kk = q * kRowsPerPass + kk0;
             const int32_t xr = (int32_t)lds32(rec + 4 * kk);
-            const uint32_t nb = xr >= 0 ? colbytes : 0u;
-            asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(
-                             sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4)),
-                         "l"(xcol + (int64_t)max(xr, 0) * ldx32), "r"(nb), "l"(pol_x)
-                         : "memory");
+            // byte address of row xr: one 32 x 32 -> 64-bit multiply-add (rows, ldx < 2^31)
+            const uint64_t src = (uint64_t)(uint32_t)max(xr, 0) * ldxb + (uint64_t)(uintptr_t)xcol;
+            const uint32_t dst =
+                sbase + (kk >> 3) * 1024 + (kk & 7) * 128 + ((((uint32_t)c16 ^ (uint32_t)kk) & 7u) << 4);
+            if (colbytes == 16u)  // full 16-byte piece: ignore-src zero fill for the -1 rows
+              asm volatile(
+                  "{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %2, 0;\n\t"
+                  "cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, q, %3;\n\t}" ::"r"(dst),
+                  "l"(src), "r"(xr), "l"(pol_x)
+                  : "memory");
+            else  // the F tail: partial or empty pieces
+              asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(dst), "l"(src),
+                           "r"(xr >= 0 ? colbytes : 0u), "l"(pol_x)
+                           : "memory");
           }
           // A row and nibble word of this thread's row
           const uint32_t mask = lds8(rec + kRecMaskOff + row);
