@@ -282,7 +282,7 @@ static nm_status gcn_layer_impl(const nm_packed* Ahat, const void* H, const void
   if (!agg_first) {
     st = dense_gemm(H, W, buf16, n, F_in, F_out, Ahat->dtype, false, lt_ws, s);  // XW (n x F_out)
     if (st != NM_OK) return st;
-    if (!bc && Ahat->res_nnz == 0 && Ahat->sptc_format == 1) {
+    if (!bc && Ahat->res_nnz == 0 && Ahat->sptc_format == 1 && (((uintptr_t)Hout) & 3) == 0) {
       // no residual: the tensor-core kernel's epilogue is the last writer of every row, so bias,
       // activation and the 16-bit down-convert run there (no fp32 Y round trip, no extra pass)
       FusedAct fa{Hout, F_out, bias, flags & NM_RELU};
