@@ -46,7 +46,10 @@ constexpr int kFGroups = NM_FULL_GROUPS;            // gather groups (4 warps ea
 constexpr int kWProd = 0, kWG0 = 1, kWMma = kWG0 + 4 * kFGroups, kWEpi0 = kWMma + 1;
 constexpr int kFThreads = (kWEpi0 + 4) * 32;        // 22 warps (4 groups)
 constexpr int kGThreads = 128;                      // threads per gather group
-constexpr int kPfChunks = 24;                       // records L2-prefetched for the next unit
+#ifndef NM_FULL_PF
+#define NM_FULL_PF 24
+#endif
+constexpr int kPfChunks = NM_FULL_PF;               // records L2-prefetched ahead (chunks)
 
 struct FullParams {
   const uint8_t* image;            // full records, kChunkBytes each, in chunk order
@@ -209,7 +212,12 @@ __global__ void __launch_bounds__(kFThreads, 1) k_spmm_full(const FullParams p) 
     // records are streamed once: L2 evict-first, so they do not push the gathered X rows
     // (evict-last) out of L2 (ncu, C3: DRAM reads 4.08 GB for 2.57 GB of records without it)
     uint64_t pol_stream;
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_stream));
+#ifndef NM_FULL_REC_FRAC
+#define NM_FULL_REC_FRAC 1.0
+#endif
+#define NM_STR2(x) #x
+#define NM_STR(x) NM_STR2(x)
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, " NM_STR(NM_FULL_REC_FRAC) ";" : "=l"(pol_stream));
     int s = 0;
     uint32_t ph = 0;
     int64_t c0 = pa < pz ? __ldg(p.panel_chunk_ptr + pa) : 0;
