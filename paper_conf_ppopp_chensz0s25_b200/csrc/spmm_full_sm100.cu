@@ -47,7 +47,7 @@ constexpr int kWProd = 0, kWG0 = 1, kWMma = kWG0 + 4 * kFGroups, kWEpi0 = kWMma 
 constexpr int kFThreads = (kWEpi0 + 4) * 32;        // 22 warps (4 groups)
 constexpr int kGThreads = 128;                      // threads per gather group
 #ifndef NM_FULL_PF
-#define NM_FULL_PF 24
+#define NM_FULL_PF 4
 #endif
 constexpr int kPfChunks = NM_FULL_PF;               // records L2-prefetched ahead (chunks)
 
