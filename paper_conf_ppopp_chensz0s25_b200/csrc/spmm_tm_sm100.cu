@@ -28,7 +28,10 @@ constexpr int kTGroups = NM_TM_GROUPS;  // gather + expansion groups (4 warps ea
 constexpr int kWProd = 0, kWG0 = 1, kWMma = kWG0 + 4 * kTGroups, kWEpi0 = kWMma + 1;
 constexpr int kTThreads = (kWEpi0 + 4) * 32;  // 22 warps at 4 groups
 constexpr int kGThreads = 128;
-constexpr int kPfBytes = 96 * 1024;           // records L2-prefetched ahead of the stream
+#ifndef NM_TM_PF_KB
+#define NM_TM_PF_KB 96
+#endif
+constexpr int kPfBytes = NM_TM_PF_KB * 1024;  // records L2-prefetched ahead of the stream
 
 struct TmParams {
   const uint8_t* image;            // compressed records, chunk order
