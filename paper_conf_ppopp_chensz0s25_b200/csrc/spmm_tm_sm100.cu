@@ -29,7 +29,7 @@ constexpr int kWProd = 0, kWG0 = 1, kWMma = kWG0 + 4 * kTGroups, kWEpi0 = kWMma 
 constexpr int kTThreads = (kWEpi0 + 4) * 32;  // 22 warps at 4 groups
 constexpr int kGThreads = 128;
 #ifndef NM_TM_PF_KB
-#define NM_TM_PF_KB 96
+#define NM_TM_PF_KB 16
 #endif
 constexpr int kPfBytes = NM_TM_PF_KB * 1024;  // records L2-prefetched ahead of the stream
 
